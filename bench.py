@@ -1,0 +1,444 @@
+#!/usr/bin/env python
+"""bench.py -- MPress D2D stripe swap on B200 (BASELINE.json metric).
+
+Metric: "D2D swap GB/s per source GPU vs 900 GB/s NVLink; GEMM slowdown while
+swapping".  One step = one pass of the whole hot path:
+  a1 PLAN      mpress_plan of the stage-0 micro-batch (host, integer);
+  a3/a4 OUT    one swap-out per in-flight micro-batch (8, 1F1B) + its event;
+  a5 IN        the matching swap-ins;
+  a6 WAIT      the compute stream waits on the last swap-in's event.
+(a2 MAP -- cuMem pool export/import/map -- is set-up, done once before timing.)
+
+Workload (BASELINE.json configs[1], BJ:8): Bert-large stage-0 activations
+(seq 512, micro-batch 8; 47 tensors, 900 MiB per micro-batch, 8 micro-batches
+in flight = 7.03 GiB) striped over 3 light-load peers.
+  * N = 1 (one GPU): the 3 peers are disjoint cuMem pools on the same B200
+    ("loopback", mpress_init_local); the bytes cross HBM instead of NVLink, so
+    the roofline is the measured HBM copy bandwidth.
+  * N > 1 (torchrun, one process per GPU): every rank is a source striping
+    its batch over all N-1 other ranks and an importer for theirs
+    (mpress_init: POSIX-fd pool exchange + cuMemMap peer access over
+    NVLink); value = all ranks' swapped bytes / max-over-ranks time.
+value counts swapped tensor bytes, out + in (the round trip of P:332's
+"time cost", reading R15), per second.  Inputs (7 GiB) exceed the 126 MB L2,
+so no flush is needed between steps.
+"""
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+GiB = 1 << 30
+MICRO_BATCHES = 8
+SPARE_PER_PEER = 24 * GiB          # cfg2: 24 GiB spare per peer
+FALLBACK_HBM = 6650.0              # B200_PROFILING.md fallback, GB/s
+NVLINK_MEASURED = 770.0            # B200_PROFILING.md: measured peer copy per direction
+NVLINK_NOMINAL = 900.0
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="mpress", choices=["mpress", "reference"])
+    ap.add_argument("--path", default="direct", choices=["direct", "bulk", "ce"])
+    ap.add_argument("--max-ctas", type=int, default=0)
+    ap.add_argument("--micro-batches", type=int, default=MICRO_BATCHES)
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=10.0)
+    return ap.parse_args()
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            return json.load(f), "measured"
+    return {"hbm_gbs": FALLBACK_HBM}, "fallback"
+
+
+# --------------------------------------------------------------- clocks
+
+class Clocks:
+    FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+        self.file = None
+
+    def start(self):
+        try:
+            self.file = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), "--query-gpu=" + self.FIELDS,
+                 "--format=csv,noheader,nounits", "-lms", "200"],
+                stdout=self.file, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return None
+        time.sleep(0.25)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.file.flush()
+        self.file.seek(0)
+        rows = [r.strip().split(", ") for r in self.file.read().splitlines() if r.strip()]
+        os.unlink(self.file.name)
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in rows:
+            try:
+                sm.append(float(r[0]))
+                mx = float(r[1])
+            except (ValueError, IndexError):
+                continue
+            for n, v in zip(names, r[3:7]):
+                if v.strip().lower() == "active":
+                    reasons.add(n)
+        if not sm:
+            return None
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+# --------------------------------------------------------------- oracle (cpu)
+
+def oracle_sample(seconds):
+    """The oracle as it stands (plain Python planner + numpy byte model), one
+    micro-batch of the workload per pass, single-threaded, >= `seconds`."""
+    import numpy as np
+    import oracle
+    from synth import splitmix64_bytes, workloads
+    sizes = workloads.cfg2_sizes(1)
+    world, peers = 4, [1, 2, 3]
+    spare = workloads.spare_vector(world, 0, peers, spare=SPARE_PER_PEER)
+    bw = workloads.bw_vector(world, 0, peers)
+    host = [splitmix64_bytes(2000, i, 0, s) for i, s in enumerate(sizes)]
+    passes, moved = 0, 0
+    t0 = time.perf_counter()
+    while True:
+        pl = oracle.plan(world, 0, spare, bw, sizes)
+        stash = oracle.swap_out(pl, host)
+        back = oracle.swap_in(pl, stash)
+        passes += 1
+        moved += 2 * sum(sizes)
+        if time.perf_counter() - t0 >= seconds:
+            break
+    el = time.perf_counter() - t0
+    assert all(np.array_equal(a, b) for a, b in zip(host, back))
+    return {"value": moved / el / 1e9, "unit": "GB/s", "cores": 1, "kind": "oracle",
+            "sample": "%d pass(es) of plan + swap-out + swap-in of 1 of the 8 Bert stage-0 "
+                      "micro-batches (47 tensors, 900 MiB), 3 peers, numpy on one host thread"
+                      % passes}
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    seconds = max(1.0, 60.0 / max(1, args.steps + args.warmup))
+    for _ in range(args.warmup):
+        oracle_sample(0.0)
+    vals = [oracle_sample(seconds / 2)["value"] for _ in range(args.steps)]
+    v = statistics.median(vals)
+    cb = oracle_sample(0.0)
+    cb["value"] = v
+    cb["cores"] = 1
+    line = {"impl": "reference", "metric": "D2D swap GB/s per source GPU (round trip, out+in)",
+            "value": v, "unit": "GB/s", "n_gpus": args.gpus, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": 2 * 900 * (1 << 20) / (v * 1e9) * 1e3,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u8",
+            "data": "synthetic", "config": workload_config(args, args.gpus),
+            "cpu_baseline": cb,
+            "e2e": {"value": v, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line))
+    return 0
+
+
+# --------------------------------------------------------------- the GPU bench
+
+def workload_config(args, n):
+    if n == 1:
+        wl = "cfg2 Bert-large stage-0 activations x%d micro-batches -> 3 peers (1-GPU loopback: " \
+             "peers are cuMem pools on the same B200)" % args.micro_batches
+    else:
+        wl = "cfg2 Bert-large stage-0 activations x%d micro-batches per rank -> all %d other " \
+             "ranks over NVLink (every rank a source and an importer)" % (args.micro_batches, n - 1)
+    return {"workload": wl, "tensors_per_micro_batch": 47, "micro_batch_bytes": 900 << 20,
+            "micro_batches": args.micro_batches, "peers": 3 if n == 1 else n - 1,
+            "path": args.path, "max_ctas": args.max_ctas,
+            "l2": "inputs %.2f GiB per rank > 126 MB L2: no flush needed" %
+                  (args.micro_batches * 900 / 1024)}
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import torch.distributed as dist
+
+    world_env = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    n = world_env
+    torch.cuda.set_device(local_rank)
+    if n > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+
+    import paper_conf_hpca_zhouwylbyx23_b200 as mp
+    from synth import device as synth_dev
+    from synth import workloads
+
+    sizes = workloads.cfg2_sizes(1)
+    mb = args.micro_batches
+    G = mp.DEFAULT_GRANULE
+    path = {"direct": mp.PATH_DIRECT, "bulk": mp.PATH_BULK, "ce": mp.PATH_CE}[args.path]
+
+    if n == 1:
+        world, source = 4, 0
+        peers = [1, 2, 3]
+        spare = workloads.spare_vector(world, source, peers, spare=SPARE_PER_PEER)
+        bw = workloads.bw_vector(world, source, peers)
+        pl0 = mp.plan(world, source, spare, bw, sizes)
+        part = [[0] * world for _ in range(world)]
+        part[source] = [mb * u * G for u in pl0.units]
+        ctx = mp.Context.local(world, source, [local_rank] * world, part)
+        per_copy = spare
+    else:
+        world, source = n, rank
+        spare = [SPARE_PER_PEER] * world
+        bwm = [[0 if s == p else 1 for p in range(world)] for s in range(world)]
+        bw = bwm[source]
+        reqs = [(s, sizes, mb) for s in range(world)]
+        part = mp.partition_sequential(world, spare, bwm, reqs)
+        ctx = mp.Context.distributed(local_rank, world, rank, part)
+        # what source s planned against inside partition_sequential
+        rem = list(spare)
+        for s in range(world):
+            pc = [r // mb for r in rem]
+            if s == source:
+                per_copy = pc
+            for p in range(world):
+                rem[p] -= part[s][p]
+    ctx.set_option(mp.OPT_PATH, path)
+    ctx.set_option(mp.OPT_MAX_CTAS, args.max_ctas)
+
+    seed0 = 2000 + 100 * rank
+    src = [[torch.empty(s, dtype=torch.uint8, device="cuda") for s in sizes] for _ in range(mb)]
+    dst = [[torch.empty(s, dtype=torch.uint8, device="cuda") for s in sizes] for _ in range(mb)]
+    for m in range(mb):
+        for i, t in enumerate(src[m]):
+            synth_dev.fill(t, seed0 + m, i)
+    torch.cuda.synchronize()
+    swap_stream = torch.cuda.Stream()
+    compute = torch.cuda.current_stream()
+    bytes_per_mb = sum(sizes)
+
+    timing = {"out": [], "in": []}
+    launches = [0]
+
+    def step(record=False):
+        pl = mp.plan(world, source, per_copy, bw, sizes)              # a1
+        hs = []
+        for m in range(mb):                                            # a3 + a4
+            if record:
+                e0 = torch.cuda.Event(enable_timing=True); e0.record(swap_stream)
+            hs.append(ctx.swap_out(pl, src[m], stream=swap_stream))
+            launches[0] += ctx.last_launches
+            if record:
+                e1 = torch.cuda.Event(enable_timing=True); e1.record(swap_stream)
+                timing["out"].append((e0, e1))
+        for m in range(mb):                                            # a5
+            if record:
+                e0 = torch.cuda.Event(enable_timing=True); e0.record(swap_stream)
+            ctx.swap_in(hs[m], dst[m], stream=swap_stream)
+            launches[0] += ctx.last_launches
+            if record:
+                e1 = torch.cuda.Event(enable_timing=True); e1.record(swap_stream)
+                timing["in"].append((e0, e1))
+        ctx.wait(hs[-1], compute)                                      # a6
+        for h in hs:
+            h.free()
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    if n > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clocks = Clocks(local_rank)
+    clocks.start()
+    launches[0] = 0
+    t_start = torch.cuda.Event(enable_timing=True)
+    t_end = torch.cuda.Event(enable_timing=True)
+    t_start.record(compute)
+    swap_stream.wait_stream(compute)
+    for _ in range(args.steps):
+        step(record=True)
+    t_end.record(compute)
+    torch.cuda.synchronize()
+    if n > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clk = clocks.stop()
+    ms = t_start.elapsed_time(t_end)
+    ms_t = torch.tensor([ms], dtype=torch.float64, device="cuda")
+    if n > 1:
+        dist.all_reduce(ms_t, op=dist.ReduceOp.MAX)
+    ms_max = float(ms_t.item())
+    ms_step = ms_max / args.steps
+    swapped_per_step_rank = 2 * mb * bytes_per_mb
+    value = n * swapped_per_step_rank / (ms_step / 1e3) / 1e9
+
+    # correctness of what was timed: every restored tensor == the generator
+    bad = 0
+    for m in range(mb):
+        for i, t in enumerate(dst[m]):
+            bad += synth_dev.check(t, seed0 + m, i)
+    bad_t = torch.tensor([bad], dtype=torch.int64, device="cuda")
+    if n > 1:
+        dist.all_reduce(bad_t)
+    if int(bad_t.item()) != 0:
+        raise SystemExit("round trip mismatch: %d bytes" % int(bad_t.item()))
+
+    # per-kernel durations (each swap call here is exactly one kernel launch)
+    dur = {k: [a.elapsed_time(b) for a, b in v] for k, v in timing.items()}
+    tot = {k: sum(v) for k, v in dur.items()}
+    dom = max(tot, key=tot.get)
+    avg_ms = statistics.mean(dur[dom])
+    peaks, peaks_src = measured_peaks()
+    if n == 1:
+        algo_bytes = 2 * bytes_per_mb       # HBM read + HBM write per swapped byte
+        achieved = algo_bytes / (avg_ms / 1e3) / 1e9
+        peak = float(peaks.get("hbm_gbs", FALLBACK_HBM))
+        roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                "frac": achieved / peak, "traffic": traffic_from_profile(),
+                "kernel": "mp_swap_%s<%s>" % (args.path, "kDirIn" if dom == "in" else "kDirOut"),
+                "algorithmic_bytes_per_launch": algo_bytes,
+                "avg_launch_ms": avg_ms, "peak_source": "%s hbm_gbs (MEASURED_PEAKS.json)" % peaks_src,
+                "share_of_step": (tot["in"] + tot["out"]) / ms * 1.0 if ms > 0 else None}
+    else:
+        algo_bytes = bytes_per_mb           # bytes over NVLink per launch (one direction)
+        achieved = algo_bytes / (avg_ms / 1e3) / 1e9
+        roof = {"bound": "nvlink", "achieved": achieved, "peak": NVLINK_MEASURED, "unit": "GB/s",
+                "frac": achieved / NVLINK_MEASURED, "traffic": None,
+                "nominal_peak": NVLINK_NOMINAL, "frac_of_nominal": achieved / NVLINK_NOMINAL,
+                "kernel": "mp_swap_%s<%s>" % (args.path, "kDirIn" if dom == "in" else "kDirOut"),
+                "algorithmic_bytes_per_launch": algo_bytes, "avg_launch_ms": avg_ms,
+                "peak_source": "B200_PROFILING.md measured peer copy per direction"}
+    per_dir = {k: bytes_per_mb / (statistics.mean(v) / 1e3) / 1e9 for k, v in dur.items()}
+
+    e2e = run_e2e(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap_stream, n, dist)
+
+    cpu = None
+    if rank == 0 and n == 1 and not args.no_cpu_baseline:
+        cpu = oracle_sample(args.cpu_seconds)
+
+    if rank == 0:
+        line = {
+            "metric": "D2D swap GB/s per source GPU (round trip, out+in)",
+            "value": value, "unit": "GB/s", "n_gpus": n, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+            "config": workload_config(args, n),
+            "per_direction_gbs": per_dir,
+            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
+            "gpu_launches": launches[0], "clocks": clk,
+            "parity": "round trip bit-exact vs generator (all %d tensors x %d ranks)" % (47 * mb, n),
+        }
+        print(json.dumps(line))
+    ctx.finalize()
+    if n > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def traffic_from_profile():
+    """dram read+write bytes per launch of the dominant kernel from the
+    committed ncu --set full summary, if one exists for this round."""
+    p = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(p):
+        try:
+            with open(p) as f:
+                return json.load(f).get("dram_bytes_per_launch")
+        except Exception:
+            return None
+    return None
+
+
+def run_e2e(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, stream, n, dist):
+    """Same metric through the public API with pinned HOST buffers: each step
+    copies the micro-batches' inputs host->device, swaps them out and in, and
+    reads the restored tensors back device->host."""
+    import torch
+    mb = len(src)
+    steps = max(1, args.e2e_steps)
+    hsrc = [[torch.empty(s, dtype=torch.uint8, pin_memory=True) for s in sizes] for _ in range(mb)]
+    hdst = [[torch.empty(s, dtype=torch.uint8, pin_memory=True) for s in sizes] for _ in range(mb)]
+    for m in range(mb):
+        for i in range(len(sizes)):
+            hsrc[m][i].copy_(src[m][i])
+    torch.cuda.synchronize()
+
+    def step():
+        with torch.cuda.stream(stream):
+            for m in range(mb):
+                for i in range(len(sizes)):
+                    src[m][i].copy_(hsrc[m][i], non_blocking=True)
+        pl = mp.plan(world, source, per_copy, bw, sizes)
+        hs = [ctx.swap_out(pl, src[m], stream=stream) for m in range(mb)]
+        for m in range(mb):
+            ctx.swap_in(hs[m], dst[m], stream=stream)
+        with torch.cuda.stream(stream):
+            for m in range(mb):
+                for i in range(len(sizes)):
+                    hdst[m][i].copy_(dst[m][i], non_blocking=True)
+        for h in hs:
+            h.free()
+
+    step()
+    torch.cuda.synchronize()
+    if n > 1:
+        dist.barrier()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(steps):
+        step()
+    e1.record(stream)
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1)
+    t = torch.tensor([ms], dtype=torch.float64, device="cuda")
+    if n > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms = float(t.item()) / steps
+    per = 2 * mb * sum(sizes)
+    import numpy as np
+    ok = all(np.array_equal(hdst[m][i].numpy(), hsrc[m][i].numpy())
+             for m in (0, mb - 1) for i in range(len(sizes)))
+    return {"value": n * per / (ms / 1e3) / 1e9, "unit": "GB/s",
+            "h2d_bytes_per_step": mb * sum(sizes), "d2h_bytes_per_step": mb * sum(sizes),
+            "steps": steps, "ms_per_step": ms, "round_trip_ok": bool(ok)}
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,307 @@
+/*
+ * mpress.h -- C ABI of libmpress: MPress's device-to-device (D2D) stripe swap
+ * (Zhou et al., "MPress", HPCA 2023), built B200-native.
+ *
+ * Citations: P:<n> = line n of the paper text (§III-C "D2D Swap"
+ * unless stated), R<n> = a reading of the paper recorded in DESIGN.md §3.
+ *
+ * What the library does:
+ *   A GPU with high memory pressure (an early pipeline stage, the "source" or
+ *   "exporter") moves a batch of tensors into the spare HBM of light-load
+ *   peers ("importers") over NVLink, striping each batch into sub-blocks whose
+ *   sizes follow the per-link bandwidth and never exceed a peer's spare
+ *   memory, then streams them back before the next use.
+ *
+ *   mpress_plan      -- the stripe planner (P:151, P:153, P:209, P:213,
+ *                       Fig. 6 lines 2-8 P:156-170).  Host only, integers only.
+ *   mpress_init*     -- the peer-memory layer: each importer reserves a stash
+ *                       pool out of its spare HBM (cuMemCreate), exports it,
+ *                       and every source maps the pools it uses (cuMemMap +
+ *                       cuMemSetAccess over NVLink / NVSwitch).
+ *   mpress_swap_out  -- hand-written sm_100a copy kernel: local tensor bytes
+ *                       -> peer stash ("swap-out" operator).
+ *   mpress_swap_in   -- peer stash -> caller's destination buffers (P:145
+ *                       "swap-in" operator), guided by the handle = the
+ *                       metadata-table entry of P:211.
+ *   mpress_wait / mpress_query -- completion is signalled with CUDA events,
+ *                       so the compute stream overlaps the swap and the host
+ *                       never blocks.
+ *
+ * Conventions
+ *   - Every entry point returns int: MPRESS_OK (0) or a negative MPRESS_ERR_*;
+ *     mpress_last_error() then returns a thread-local message.  No C++
+ *     exception crosses this boundary.
+ *   - Sizes and offsets are bytes (uint64_t).  "Device pointer" = a CUDA
+ *     device address valid on the context's device.
+ *   - CUDA handles are passed as void*: a `cudaStream_t` / `cudaEvent_t`
+ *     (NULL stream = the legacy default stream).
+ *   - Ownership: the caller owns tensors, destination buffers, streams and
+ *     events it passes in.  The library owns plans, contexts, handles, the
+ *     events inside handles, the stash pools and the peer mappings.
+ *   - A context is single-threaded: calls on one context must not race.
+ *     Different contexts are independent.
+ */
+#ifndef MPRESS_H_
+#define MPRESS_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define MPRESS_VERSION 1
+
+#if defined(__GNUC__)
+#define MPRESS_API __attribute__((visibility("default")))
+#else
+#define MPRESS_API
+#endif
+
+/* ---- status codes --------------------------------------------------------- */
+#define MPRESS_OK             0
+#define MPRESS_ERR_ARG       -1  /* null pointer, granule % 256 != 0, source out
+                                    of range, n_tensors == 0, size overflow     */
+#define MPRESS_ERR_NO_SPACE  -2  /* peers' spare cannot hold the batch (P:295,
+                                    R9) or the stash partition is full (R21)   */
+#define MPRESS_ERR_ALIGN     -3  /* tensor / destination not 16-byte aligned    */
+#define MPRESS_ERR_STATE     -4  /* illegal handle transition (R13)             */
+#define MPRESS_ERR_PEER      -5  /* peer not mapped / no peer access            */
+#define MPRESS_ERR_CUDA      -6  /* a CUDA runtime or driver call failed        */
+#define MPRESS_ERR_SYS       -7  /* socket / fd-passing failure at init         */
+
+#define MPRESS_ALIGN            256u    /* virtual tensor alignment (R6)        */
+#define MPRESS_DEFAULT_GRANULE  65536u  /* planning unit G (R3)                 */
+
+/* ---- the plan (metadata table) ------------------------------------- */
+
+/* One sub-block: bytes [src_off, src_off+len) of tensor `tensor` live at
+ * [dst_off, dst_off+len) of the source's slice on peer `peer`.
+ * src_off and dst_off are multiples of 256 (R6).                           */
+typedef struct mpress_stripe {
+  uint32_t tensor;
+  uint32_t peer;
+  uint64_t src_off;
+  uint64_t dst_off;
+  uint64_t len;
+} mpress_stripe;
+
+typedef struct mpress_plan_info {
+  int32_t  world;          /* number of devices the plan spans               */
+  int32_t  source;         /* the exporter                                   */
+  uint32_t n_tensors;
+  uint32_t n_stripes;
+  uint64_t granule;        /* G                                              */
+  uint64_t virtual_bytes;  /* V = sum_i roundup(S_i, 256)                    */
+  uint64_t units;          /* K = ceil(V / G)                                */
+} mpress_plan_info;
+
+typedef struct mpress_plan_s   mpress_plan_t;    /* opaque, library-owned */
+typedef struct mpress_ctx_s    mpress_ctx_t;     /* opaque, library-owned */
+typedef struct mpress_handle_s mpress_handle_t;  /* opaque, library-owned */
+
+/*
+ * mpress_plan -- stripe assignment of one source's tensor batch over its
+ * peers (P:151 equal sub-blocks on symmetric links; P:153/P:209 sub-block
+ * sizes proportional to link bandwidth, tensors batched; Fig. 6 line 3 P:160
+ * spare = MEM_CAP - MEM_USE bounds each peer; P:213 best score = minimum of the
+ * maximal swap time).
+ *
+ *   world         number of devices, >= 1
+ *   source        exporter index in [0, world)
+ *   spare_bytes   [world] spare HBM of each device; the source's entry is ignored.
+ *                 Usable = floor(spare/G)*G (R8).
+ *   link_bw       [world] integer bandwidth weight of link source->p; 0 = not an
+ *                 NVLink neighbour (R10).  Only ratios matter.
+ *   n_tensors     >= 1;  tensor_bytes [n_tensors], each >= 1
+ *   granule       G; 0 -> MPRESS_DEFAULT_GRANULE; must be a multiple of 256
+ *   out           receives a new plan; free with mpress_plan_free
+ *
+ * Result (R1-R7): the batch is laid out virtually (tensor i at a 256-aligned
+ * offset, list order), cut into K units of G bytes, and peer p receives k_p
+ * units minimising max_p k_p/B_p subject to k_p*G <= spare_p, ties to the lower
+ * device index; peer p stores one contiguous range of the virtual batch
+ * (peers ascending).  Integer arithmetic only: the result is bit-identical on
+ * every rank and every call.
+ * Errors: MPRESS_ERR_ARG, MPRESS_ERR_NO_SPACE (no partial plans, R9).
+ */
+MPRESS_API int mpress_plan(int world, int source, const uint64_t* spare_bytes,
+                const uint64_t* link_bw, uint32_t n_tensors,
+                const uint64_t* tensor_bytes, uint64_t granule,
+                mpress_plan_t** out);
+
+/* Borrow the plan's stripe list (sorted by peer, then tensor) and the
+ * per-peer byte counts [world].  Pointers stay valid until mpress_plan_free. */
+MPRESS_API int mpress_plan_stripes(const mpress_plan_t* plan, const mpress_stripe** stripes,
+                        uint32_t* n_stripes, const uint64_t** peer_bytes);
+/* Borrow the per-peer unit counts k_p [world]. */
+MPRESS_API int mpress_plan_units(const mpress_plan_t* plan, const uint64_t** units);
+MPRESS_API int mpress_plan_get_info(const mpress_plan_t* plan, mpress_plan_info* info);
+MPRESS_API void mpress_plan_free(mpress_plan_t* plan);
+
+/*
+ * mpress_partition_sequential -- the stash partition of several sources
+ * (Fig. 6 lines 2-8 P:156-170, reading R12): sources are planned in ascending
+ * index, each against floor(remaining_p / copies_s) per peer, and reserve
+ * copies_s * k_p * G bytes of peer p.
+ *   bw_matrix     [world*world] row s = link_bw of source s
+ *   n_sources     entries in sources / n_tensors / copies
+ *   sizes_flat    concatenated tensor_bytes of the sources, in the order given
+ *   partition     [world*world] out: partition[s*world+p] = bytes of p's pool
+ *                 owned by source s (0 for non-sources)
+ * Errors: as mpress_plan for any source.
+ */
+MPRESS_API int mpress_partition_sequential(int world, const uint64_t* spare_bytes,
+                                const uint64_t* bw_matrix, uint32_t n_sources,
+                                const int32_t* sources, const uint32_t* n_tensors,
+                                const uint64_t* sizes_flat, const uint32_t* copies,
+                                uint64_t granule, uint64_t* partition);
+
+/* ---- peer-memory layer ----------------------------------------------------- */
+
+/* All-gather callback, implemented by the caller over its process group:
+ * every rank passes `len` bytes in `mine`; on return `all` holds world*len
+ * bytes, rank r's at all + r*len.  Must act as a barrier.  Return 0 on success. */
+typedef int (*mpress_exchange_fn)(void* user, const void* mine, size_t len, void* all);
+
+/*
+ * mpress_init -- collective over `world` processes, one per GPU (torchrun).
+ *   device     CUDA ordinal this rank runs on
+ *   partition  [world*world], identical on all ranks (see
+ *              mpress_partition_sequential).  Rank p creates a stash pool of
+ *              sum_s partition[s*world+p] bytes (rounded up to the VMM
+ *              granularity) in its own HBM; source s's partition starts at
+ *              sum_{s'<s} partition[s'*world+p].
+ *   exchange   all-gather used to swap process ids and to synchronise; the
+ *              pool handles themselves travel as POSIX file descriptors over
+ *              Unix-domain sockets (SCM_RIGHTS).
+ * Every rank maps each peer pool it owns a partition in, with read/write
+ * access for `device` (peer access over NVLink).
+ * Errors: MPRESS_ERR_ARG, MPRESS_ERR_CUDA, MPRESS_ERR_PEER, MPRESS_ERR_SYS.
+ */
+MPRESS_API int mpress_init(int device, int world, int rank, const uint64_t* partition,
+                mpress_exchange_fn exchange, void* exchange_user,
+                mpress_ctx_t** out);
+
+/*
+ * mpress_init_local -- single-process variant: peer p's pool lives on
+ * devices[p] and holds only this source's partition (partition[source*world+p]
+ * bytes).  With every devices[p] equal it is the 1-GPU "loopback" mode: the
+ * peers are disjoint VMM pools of the same GPU, so the whole data path
+ * (planner, mapping, kernels, scheduler) runs with HBM standing in for NVLink.
+ */
+MPRESS_API int mpress_init_local(int world, int source, const int* devices,
+                      const uint64_t* partition, mpress_ctx_t** out);
+
+/* Collective for contexts made by mpress_init (barrier, unmap, release).
+ * Outstanding handles are freed.  NULL is a no-op. */
+MPRESS_API int mpress_finalize(mpress_ctx_t* ctx);
+
+/* Largest contiguous free extent of this source's partition on each peer
+ * [world] -> the spare_bytes argument of mpress_plan for the next batch. */
+MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
+
+/* Tunables.  MPRESS_OPT_PATH: 0 = SM kernel, direct 16-B loads/stores
+ * (default); 1 = SM kernel, bulk-async (TMA engine) staged through shared
+ * memory; 2 = copy engines (cudaMemcpyAsync per stripe on per-peer streams,
+ * the measured comparator).  MPRESS_OPT_MAX_CTAS: cap on the kernel grid
+ * (0 = one wave of resident CTAs over all SMs); each CTA occupies one SM slot,
+ * so this is the SM-count cap that protects a concurrent GEMM.            */
+#define MPRESS_OPT_PATH      1
+#define MPRESS_OPT_MAX_CTAS  2
+#define MPRESS_PATH_DIRECT   0
+#define MPRESS_PATH_BULK     1
+#define MPRESS_PATH_CE       2
+MPRESS_API int mpress_set_option(mpress_ctx_t* ctx, int key, int64_t value);
+MPRESS_API int mpress_get_option(const mpress_ctx_t* ctx, int key, int64_t* value);
+
+/* ---- the swap --------------------------------------------------------------- */
+
+/* Handle states (R13; "record ... before the execution of the swap-out
+ * operator ... updated when it completes"). */
+#define MPRESS_STATE_OUT_PENDING 1  /* swap-out enqueued                      */
+#define MPRESS_STATE_OUT         2  /* swap-out complete: sources reusable     */
+#define MPRESS_STATE_IN_PENDING  3  /* swap-in enqueued                       */
+#define MPRESS_STATE_IN          4  /* swap-in complete: stash slice released  */
+
+/*
+ * mpress_swap_out -- enqueue the move of every stripe of `plan` from the
+ * caller's tensors into this source's stash slices on the peers.
+ *   tensors  [plan n_tensors] device pointers, 16-byte aligned, each at least
+ *            tensor_bytes long; must stay valid until the handle reaches
+ *            MPRESS_STATE_OUT (mpress_wait / mpress_query)
+ *   stream   cudaStream_t the kernel runs on (the "swap-out stream")
+ *   after    cudaEvent_t the stream waits on first (e.g. recorded on the
+ *            compute stream after the producing op), or NULL
+ *   out      receives a handle holding one contiguous slice per used peer
+ *            (first fit, lowest address, inside this source's partition)
+ * Bytes are copied bit-exactly; nothing interprets them (R18).
+ * Errors: MPRESS_ERR_ARG, MPRESS_ERR_ALIGN, MPRESS_ERR_NO_SPACE (partition
+ * full), MPRESS_ERR_PEER (plan uses a peer this context has not mapped, or
+ * plan.source != the context's source), MPRESS_ERR_CUDA.
+ */
+MPRESS_API int mpress_swap_out(mpress_ctx_t* ctx, const mpress_plan_t* plan,
+                    void* const* tensors, void* stream, void* after,
+                    mpress_handle_t** out);
+
+/*
+ * mpress_swap_in -- enqueue the move of every stripe back into `dst`
+ * ([n_tensors] device pointers, 16-byte aligned; may differ from the
+ * swap-out tensors, R14).  The stream first waits for the swap-out.  The
+ * handle's slices are released for reuse once this copy completes (later
+ * swap-outs into the same bytes are ordered after it by an event).
+ * Errors: MPRESS_ERR_STATE unless the handle is OUT_PENDING or OUT;
+ * MPRESS_ERR_ARG, MPRESS_ERR_ALIGN, MPRESS_ERR_CUDA.
+ */
+MPRESS_API int mpress_swap_in(mpress_ctx_t* ctx, mpress_handle_t* handle, void* const* dst,
+                   void* stream);
+
+/* Make `consumer` wait (cudaStreamWaitEvent, enqueue-only) for the handle's
+ * latest operation: the swap-out if no swap-in was issued, else the swap-in. */
+MPRESS_API int mpress_wait(mpress_ctx_t* ctx, mpress_handle_t* handle, void* consumer);
+
+/* Non-blocking: 1 = latest operation complete, 0 = pending, < 0 = error.
+ * Advances the handle state (OUT_PENDING->OUT, IN_PENDING->IN). */
+MPRESS_API int mpress_query(mpress_ctx_t* ctx, mpress_handle_t* handle);
+
+/* Current state (MPRESS_STATE_*) without querying the device. */
+MPRESS_API int mpress_handle_state(const mpress_handle_t* handle);
+
+/* Slice base of the handle inside this source's partition of each peer's
+ * pool [world]; UINT64_MAX for peers the plan does not use (tests). */
+MPRESS_API int mpress_handle_slices(const mpress_handle_t* handle, uint64_t* slice_off);
+
+/* Release a handle.  A handle still OUT_PENDING or OUT (data only in the
+ * stash) is an error (MPRESS_ERR_STATE) unless `force` is nonzero.  An
+ * IN_PENDING handle may be freed: its slices stay fenced by the swap-in event. */
+MPRESS_API int mpress_handle_free(mpress_ctx_t* ctx, mpress_handle_t* handle, int force);
+
+/* Debug / test: synchronous copy of `len` bytes at byte `offset` of this
+ * source's partition on `peer` into host memory `host_dst`. */
+MPRESS_API int mpress_peer_read(mpress_ctx_t* ctx, int peer, uint64_t offset, uint64_t len,
+                     void* host_dst);
+
+/* Kernel launches the last swap_out / swap_in call enqueued (for accounting). */
+MPRESS_API int mpress_last_launches(const mpress_ctx_t* ctx);
+
+/* ---- utilities ---------------------------------------------------------------- */
+
+/*
+ * mpress_share_fds -- the fd-passing step of mpress_init, exposed for tests:
+ * rank r offers `my_fd`; for every p with want[p] != 0 it receives a duplicate
+ * of rank p's fd in fds_out[p] (else -1).  Collective; uses `exchange` for the
+ * rendezvous and Unix-domain sockets with SCM_RIGHTS for the descriptors.
+ * The caller closes the received descriptors.
+ */
+MPRESS_API int mpress_share_fds(int world, int rank, int my_fd, const int32_t* want,
+                     mpress_exchange_fn exchange, void* exchange_user,
+                     int32_t* fds_out);
+
+MPRESS_API const char* mpress_last_error(void);
+MPRESS_API int mpress_version(void);
+
+#ifdef __cplusplus
+}  /* extern "C" */
+#endif
+#endif  /* MPRESS_H_ */

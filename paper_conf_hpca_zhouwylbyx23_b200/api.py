@@ -1,0 +1,329 @@
+"""Thin ctypes binding of libmpress (include/mpress.h).  Marshalling only.
+
+Every step of the swap path -- planning, peer mapping, the copy kernels,
+events -- runs inside libmpress.so; this module turns Python lists into C
+arrays, torch tensors into device pointers (``data_ptr()``) and torch
+streams / events into ``cudaStream_t`` / ``cudaEvent_t``.  There is no
+fallback: if the library is missing the import fails loudly.
+"""
+import ctypes
+import os
+from ctypes import (CFUNCTYPE, POINTER, byref, c_char_p, c_int, c_int32, c_int64,
+                    c_size_t, c_uint32, c_uint64, c_void_p)
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libmpress.so")
+
+OK = 0
+ERR_ARG, ERR_NO_SPACE, ERR_ALIGN, ERR_STATE, ERR_PEER, ERR_CUDA, ERR_SYS = -1, -2, -3, -4, -5, -6, -7
+ALIGN = 256
+DEFAULT_GRANULE = 65536
+OPT_PATH, OPT_MAX_CTAS = 1, 2
+PATH_DIRECT, PATH_BULK, PATH_CE = 0, 1, 2
+STATE_OUT_PENDING, STATE_OUT, STATE_IN_PENDING, STATE_IN = 1, 2, 3, 4
+
+_ERR_NAMES = {ERR_ARG: "ERR_ARG", ERR_NO_SPACE: "ERR_NO_SPACE", ERR_ALIGN: "ERR_ALIGN",
+              ERR_STATE: "ERR_STATE", ERR_PEER: "ERR_PEER", ERR_CUDA: "ERR_CUDA",
+              ERR_SYS: "ERR_SYS"}
+
+EXPORTED = [
+    "mpress_plan", "mpress_plan_stripes", "mpress_plan_units", "mpress_plan_get_info",
+    "mpress_plan_free", "mpress_partition_sequential", "mpress_init", "mpress_init_local",
+    "mpress_finalize", "mpress_stash_free", "mpress_set_option", "mpress_get_option",
+    "mpress_swap_out", "mpress_swap_in", "mpress_wait", "mpress_query", "mpress_handle_state",
+    "mpress_handle_slices", "mpress_handle_free", "mpress_peer_read", "mpress_last_launches",
+    "mpress_share_fds", "mpress_last_error", "mpress_version",
+]
+
+
+class MPressError(RuntimeError):
+    def __init__(self, code, msg):
+        super().__init__("%s (%d): %s" % (_ERR_NAMES.get(code, "?"), code, msg))
+        self.code = code
+
+
+class Stripe(ctypes.Structure):
+    _fields_ = [("tensor", c_uint32), ("peer", c_uint32), ("src_off", c_uint64),
+                ("dst_off", c_uint64), ("len", c_uint64)]
+
+
+class PlanInfo(ctypes.Structure):
+    _fields_ = [("world", c_int32), ("source", c_int32), ("n_tensors", c_uint32),
+                ("n_stripes", c_uint32), ("granule", c_uint64), ("virtual_bytes", c_uint64),
+                ("units", c_uint64)]
+
+
+EXCHANGE_FN = CFUNCTYPE(c_int, c_void_p, c_void_p, c_size_t, c_void_p)
+
+
+def _load():
+    if not os.path.exists(LIB_PATH):
+        raise ImportError("libmpress.so not built at %s: run "
+                          "`python -c 'import __graft_entry__ as g; g.build()'`" % LIB_PATH)
+    lib = ctypes.CDLL(LIB_PATH)
+    P = c_void_p
+    sig = {
+        "mpress_plan": (c_int, [c_int, c_int, P, P, c_uint32, P, c_uint64, POINTER(P)]),
+        "mpress_plan_stripes": (c_int, [P, POINTER(POINTER(Stripe)), POINTER(c_uint32), POINTER(POINTER(c_uint64))]),
+        "mpress_plan_units": (c_int, [P, POINTER(POINTER(c_uint64))]),
+        "mpress_plan_get_info": (c_int, [P, POINTER(PlanInfo)]),
+        "mpress_plan_free": (None, [P]),
+        "mpress_partition_sequential": (c_int, [c_int, P, P, c_uint32, P, P, P, P, c_uint64, P]),
+        "mpress_init": (c_int, [c_int, c_int, c_int, P, EXCHANGE_FN, P, POINTER(P)]),
+        "mpress_init_local": (c_int, [c_int, c_int, P, P, POINTER(P)]),
+        "mpress_finalize": (c_int, [P]),
+        "mpress_stash_free": (c_int, [P, P]),
+        "mpress_set_option": (c_int, [P, c_int, c_int64]),
+        "mpress_get_option": (c_int, [P, c_int, POINTER(c_int64)]),
+        "mpress_swap_out": (c_int, [P, P, P, P, P, POINTER(P)]),
+        "mpress_swap_in": (c_int, [P, P, P, P]),
+        "mpress_wait": (c_int, [P, P, P]),
+        "mpress_query": (c_int, [P, P]),
+        "mpress_handle_state": (c_int, [P]),
+        "mpress_handle_slices": (c_int, [P, P]),
+        "mpress_handle_free": (c_int, [P, P, c_int]),
+        "mpress_peer_read": (c_int, [P, c_int, c_uint64, c_uint64, P]),
+        "mpress_last_launches": (c_int, [P]),
+        "mpress_share_fds": (c_int, [c_int, c_int, c_int, P, EXCHANGE_FN, P, P]),
+        "mpress_last_error": (c_char_p, []),
+        "mpress_version": (c_int, []),
+    }
+    for name, (res, args) in sig.items():
+        f = getattr(lib, name)
+        f.restype = res
+        f.argtypes = args
+    return lib
+
+
+lib = _load()
+
+
+def _check(rc):
+    if rc < 0:
+        raise MPressError(rc, lib.mpress_last_error().decode(errors="replace"))
+    return rc
+
+
+def _u64(values):
+    return (c_uint64 * len(values))(*[int(v) for v in values])
+
+
+def _ptr(x):
+    """Device pointer of a torch tensor, or an int address."""
+    if hasattr(x, "data_ptr"):
+        return int(x.data_ptr())
+    return int(x)
+
+
+def _stream(s, device=None):
+    if s is None:
+        import torch
+        return c_void_p(torch.cuda.current_stream(device).cuda_stream)
+    if hasattr(s, "cuda_stream"):
+        return c_void_p(s.cuda_stream)
+    return c_void_p(int(s))
+
+
+def _event(e):
+    if e is None:
+        return None
+    if hasattr(e, "cuda_event"):
+        return c_void_p(e.cuda_event)
+    return c_void_p(int(e))
+
+
+# ------------------------------------------------------------------------- plans
+
+class Plan:
+    """Owner of an mpress_plan_t (the metadata table of one batch)."""
+
+    def __init__(self, world, source, spare, bw, sizes, granule=0):
+        if len(spare) != world or len(bw) != world:
+            raise MPressError(ERR_ARG, "spare/bw must have `world` entries")
+        h = c_void_p()
+        _check(lib.mpress_plan(world, source, _u64(spare), _u64(bw), len(sizes), _u64(sizes),
+                               granule, byref(h)))
+        self._h = h
+        self.world = world
+        self.sizes = [int(s) for s in sizes]
+
+    def __del__(self):
+        h = getattr(self, "_h", None)
+        if h is not None and h.value:
+            lib.mpress_plan_free(h)
+            self._h = None
+
+    @property
+    def handle(self):
+        return self._h
+
+    @property
+    def info(self):
+        i = PlanInfo()
+        _check(lib.mpress_plan_get_info(self._h, byref(i)))
+        return i
+
+    @property
+    def stripes(self):
+        p = POINTER(Stripe)()
+        n = c_uint32()
+        _check(lib.mpress_plan_stripes(self._h, byref(p), byref(n), None))
+        return [(p[i].tensor, p[i].peer, p[i].src_off, p[i].dst_off, p[i].len) for i in range(n.value)]
+
+    @property
+    def peer_bytes(self):
+        pb = POINTER(c_uint64)()
+        _check(lib.mpress_plan_stripes(self._h, None, None, byref(pb)))
+        return [pb[i] for i in range(self.world)]
+
+    @property
+    def units(self):
+        u = POINTER(c_uint64)()
+        _check(lib.mpress_plan_units(self._h, byref(u)))
+        return [u[i] for i in range(self.world)]
+
+
+def plan(world, source, spare, bw, sizes, granule=0):
+    return Plan(world, source, spare, bw, sizes, granule)
+
+
+def partition_sequential(world, spare, bw_matrix, requests, granule=0):
+    """requests: [(source, sizes, copies)] -> partition[s][p] (bytes)."""
+    srcs = (c_int32 * len(requests))(*[r[0] for r in requests])
+    ns = (c_uint32 * len(requests))(*[len(r[1]) for r in requests])
+    cp = (c_uint32 * len(requests))(*[r[2] for r in requests])
+    flat = _u64([s for r in requests for s in r[1]] or [0])
+    bwm = _u64([b for row in bw_matrix for b in row])
+    out = (c_uint64 * (world * world))()
+    _check(lib.mpress_partition_sequential(world, _u64(spare), bwm, len(requests), srcs, ns, flat,
+                                           cp, granule, out))
+    return [[out[s * world + p] for p in range(world)] for s in range(world)]
+
+
+# ------------------------------------------------------------------- exchange
+
+def torch_exchange(group=None):
+    """An all-gather callback over a torch.distributed process group (gloo for
+    CPU bytes; an NCCL default group gets a gloo side group)."""
+    import torch.distributed as dist
+    if group is None and dist.get_backend() != "gloo":
+        group = dist.new_group(backend="gloo")
+    world = dist.get_world_size(group)
+
+    def cb(user, mine, ln, out):
+        try:
+            import torch
+            t = torch.frombuffer(bytearray(ctypes.string_at(mine, ln)), dtype=torch.uint8)
+            outs = [torch.empty(ln, dtype=torch.uint8) for _ in range(world)]
+            dist.all_gather(outs, t, group=group)
+            buf = b"".join(bytes(o.numpy().tobytes()) for o in outs)
+            ctypes.memmove(out, buf, len(buf))
+            return 0
+        except Exception as e:  # pragma: no cover - reported through the C status
+            print("mpress exchange failed:", e)
+            return -1
+    return EXCHANGE_FN(cb)
+
+
+def share_fds(world, rank, my_fd, want, exchange_cb):
+    w = (c_int32 * world)(*[1 if x else 0 for x in want])
+    out = (c_int32 * world)()
+    _check(lib.mpress_share_fds(world, rank, my_fd, w, exchange_cb, None, out))
+    return list(out)
+
+
+# --------------------------------------------------------------- context / swap
+
+class Handle:
+    def __init__(self, ctx, h, plan):
+        self._ctx = ctx
+        self._h = h
+        self.plan = plan  # keeps the Plan alive while the handle exists
+
+    @property
+    def state(self):
+        return _check(lib.mpress_handle_state(self._h))
+
+    def slices(self):
+        out = (c_uint64 * self._ctx.world)()
+        _check(lib.mpress_handle_slices(self._h, out))
+        return list(out)
+
+    def free(self, force=False):
+        if self._h is not None and self._h.value:
+            _check(lib.mpress_handle_free(self._ctx._h, self._h, 1 if force else 0))
+        self._h = None
+
+
+class Context:
+    """An mpress_ctx_t: this source's view of the peers' stash pools."""
+
+    def __init__(self, h, world, source, device, exchange_cb=None):
+        self._h = h
+        self.world = world
+        self.source = source
+        self.device = device
+        self._exchange = exchange_cb  # keep the ctypes callback alive
+
+    @classmethod
+    def local(cls, world, source, devices, partition):
+        """Single process; every devices[p] equal = 1-GPU loopback."""
+        h = c_void_p()
+        devs = (c_int * world)(*devices)
+        flat = _u64([partition[s][p] for s in range(world) for p in range(world)])
+        _check(lib.mpress_init_local(world, source, devs, flat, byref(h)))
+        return cls(h, world, source, devices[source])
+
+    @classmethod
+    def distributed(cls, device, world, rank, partition, exchange_cb=None):
+        """Collective over torch.distributed (one process per GPU)."""
+        if exchange_cb is None:
+            exchange_cb = torch_exchange()
+        h = c_void_p()
+        flat = _u64([partition[s][p] for s in range(world) for p in range(world)])
+        _check(lib.mpress_init(device, world, rank, flat, exchange_cb, None, byref(h)))
+        return cls(h, world, rank, device, exchange_cb)
+
+    def finalize(self):
+        if self._h is not None:
+            _check(lib.mpress_finalize(self._h))
+            self._h = None
+
+    def set_option(self, key, value):
+        _check(lib.mpress_set_option(self._h, key, int(value)))
+
+    def get_option(self, key):
+        v = c_int64()
+        _check(lib.mpress_get_option(self._h, key, byref(v)))
+        return v.value
+
+    def stash_free(self):
+        out = (c_uint64 * self.world)()
+        _check(lib.mpress_stash_free(self._h, out))
+        return list(out)
+
+    def swap_out(self, plan_, tensors, stream=None, after=None):
+        ptrs = (c_void_p * len(tensors))(*[_ptr(t) for t in tensors])
+        h = c_void_p()
+        _check(lib.mpress_swap_out(self._h, plan_.handle, ptrs, _stream(stream, self.device),
+                                   _event(after), byref(h)))
+        return Handle(self, h, plan_)
+
+    def swap_in(self, handle, dst, stream=None):
+        ptrs = (c_void_p * len(dst))(*[_ptr(t) for t in dst])
+        _check(lib.mpress_swap_in(self._h, handle._h, ptrs, _stream(stream, self.device)))
+
+    def wait(self, handle, stream=None):
+        _check(lib.mpress_wait(self._h, handle._h, _stream(stream, self.device)))
+
+    def query(self, handle):
+        return _check(lib.mpress_query(self._h, handle._h)) == 1
+
+    def peer_read(self, peer, offset, length):
+        buf = ctypes.create_string_buffer(max(1, length))
+        _check(lib.mpress_peer_read(self._h, peer, offset, length, buf))
+        return buf.raw[:length]
+
+    @property
+    def last_launches(self):
+        return lib.mpress_last_launches(self._h)

@@ -1,0 +1,105 @@
+// Internal state of a libmpress context and its handles (not part of the ABI).
+#pragma once
+
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <map>
+#include <mutex>
+#include <set>
+#include <vector>
+
+#include "common.h"
+
+namespace mpress {
+
+// CUDA driver entry points, fetched through cudart (cudaGetDriverEntryPoint)
+// so libmpress.so has no link-time dependency on libcuda.so: it loads and
+// plans on a host without a GPU driver.
+struct Driver {
+  CUresult (*mem_create)(CUmemGenericAllocationHandle*, size_t, const CUmemAllocationProp*, unsigned long long);
+  CUresult (*mem_release)(CUmemGenericAllocationHandle);
+  CUresult (*mem_address_reserve)(CUdeviceptr*, size_t, size_t, CUdeviceptr, unsigned long long);
+  CUresult (*mem_address_free)(CUdeviceptr, size_t);
+  CUresult (*mem_map)(CUdeviceptr, size_t, size_t, CUmemGenericAllocationHandle, unsigned long long);
+  CUresult (*mem_unmap)(CUdeviceptr, size_t);
+  CUresult (*mem_set_access)(CUdeviceptr, size_t, const CUmemAccessDesc*, size_t);
+  CUresult (*mem_export)(void*, CUmemGenericAllocationHandle, CUmemAllocationHandleType, unsigned long long);
+  CUresult (*mem_import)(CUmemGenericAllocationHandle*, void*, CUmemAllocationHandleType);
+  CUresult (*mem_granularity)(size_t*, const CUmemAllocationProp*, CUmemAllocationGranularity_flags);
+  CUresult (*get_error_string)(CUresult, const char**);
+};
+int driver(const Driver** out);
+int cu_fail(const Driver* d, CUresult r, const char* what);
+
+// RAII: make `dev` current, restore the caller's device afterwards.
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    cudaGetDevice(&prev);
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+// A VMM mapping: physical allocation (created or imported) mapped at `va`.
+struct Mapping {
+  CUmemGenericAllocationHandle handle = 0;
+  CUdeviceptr va = 0;
+  size_t size = 0;
+  bool reserved = false, mapped = false, has_handle = false;
+};
+
+// A released slice whose bytes a pending swap-in may still be reading.
+struct Fence {
+  uint64_t off, len;
+  cudaEvent_t ev;
+};
+
+// This source's partition of one peer's stash pool (R21).
+struct Partition {
+  uint8_t* base = nullptr;            // local VA of the partition start
+  uint64_t size = 0;
+  std::map<uint64_t, uint64_t> free;  // first-fit free list: offset -> length
+  std::vector<Fence> fences;
+};
+
+}  // namespace mpress
+
+struct mpress_handle_s;
+
+struct mpress_ctx_s {
+  int device = -1;
+  int world = 0;
+  int source = 0;                     // this context's rank = the exporter it serves
+  bool local = false;                 // mpress_init_local
+  mpress_exchange_fn exchange = nullptr;
+  void* exchange_user = nullptr;
+  std::vector<uint64_t> partition;    // [world*world]
+  mpress::Mapping own;                // multi-process: this rank's exported pool
+  std::vector<mpress::Mapping> maps;  // [world] pool mappings used by this source
+  std::vector<mpress::Partition> parts;  // [world]
+  int path = MPRESS_PATH_DIRECT;
+  int max_ctas = 0;
+  int last_launches = 0;
+  std::vector<cudaStream_t> ce_streams;  // copy-engine comparator, one per peer
+  std::vector<cudaEvent_t> ev_pool;
+  std::set<mpress_handle_s*> handles;
+  std::mutex mu;
+};
+
+struct mpress_handle_s {
+  mpress_ctx_s* ctx = nullptr;
+  int state = 0;
+  std::vector<mpress_stripe> stripes;
+  std::vector<uint64_t> sizes;
+  std::vector<uint64_t> slice_off;    // [world], UINT64_MAX if unused
+  std::vector<uint64_t> slice_len;    // [world]
+  cudaEvent_t out_done = nullptr;
+  cudaEvent_t in_done = nullptr;
+  bool slices_held = false;
+};

@@ -1,0 +1,330 @@
+// Event-driven swap scheduler: handles = the
+// paper's D2D metadata table ("number of sub-blocks, the sizes of each
+// sub-block, and the indices of target GPU devices ... recorded before the
+// execution of the swap-out operator ... used to guide the execution of the
+// latter swap-in operator and updated when it completes"), stash-slice
+// allocation inside the source's partition (R21), and completion events.
+//
+// The paper runs swap-out and swap-in on two executor threads with their own
+// CUDA streams so launches and status checks never block the main thread
+// (P:236).  Here the caller's side streams carry the kernels and CUDA
+// events carry completion: every call only enqueues work, and
+// mpress_wait / mpress_query are enqueue-only / non-blocking, so no helper
+// thread is needed.
+#include <algorithm>
+#include <cstring>
+
+#include "ctx.h"
+#include "swap_kernels.h"
+
+namespace mpress {
+namespace {
+
+cudaEvent_t take_event(mpress_ctx_s* c) {
+  if (!c->ev_pool.empty()) {
+    cudaEvent_t e = c->ev_pool.back();
+    c->ev_pool.pop_back();
+    return e;
+  }
+  cudaEvent_t e = nullptr;
+  if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) return nullptr;
+  return e;
+}
+
+void give_event(mpress_ctx_s* c, cudaEvent_t e) {
+  if (e) c->ev_pool.push_back(e);
+}
+
+// Drop fences whose swap-in has completed.
+void reap_fences(mpress_ctx_s* c, Partition* part) {
+  auto& f = part->fences;
+  size_t w = 0;
+  for (size_t r = 0; r < f.size(); ++r) {
+    if (cudaEventQuery(f[r].ev) == cudaSuccess) give_event(c, f[r].ev);
+    else f[w++] = f[r];
+  }
+  f.resize(w);
+  cudaGetLastError();  // cudaEventQuery's cudaErrorNotReady is not sticky; clear it
+}
+
+// First fit, lowest address.
+bool alloc_slice(Partition* part, uint64_t len, uint64_t* off) {
+  for (auto it = part->free.begin(); it != part->free.end(); ++it) {
+    if (it->second >= len) {
+      *off = it->first;
+      const uint64_t rest = it->second - len, roff = it->first + len;
+      part->free.erase(it);
+      if (rest) part->free[roff] = rest;
+      return true;
+    }
+  }
+  return false;
+}
+
+void free_slice(Partition* part, uint64_t off, uint64_t len) {
+  auto next = part->free.lower_bound(off);
+  if (next != part->free.end() && off + len == next->first) {  // merge right
+    len += next->second;
+    next = part->free.erase(next);
+  }
+  if (next != part->free.begin()) {  // merge left
+    auto prev = std::prev(next);
+    if (prev->first + prev->second == off) {
+      prev->second += len;
+      return;
+    }
+  }
+  part->free[off] = len;
+}
+
+int check_ptrs(void* const* p, size_t n, const char* what) {
+  if (!p) return fail(MPRESS_ERR_ARG, "%s: null pointer array", what);
+  for (size_t i = 0; i < n; ++i) {
+    if (!p[i]) return fail(MPRESS_ERR_ARG, "%s: pointer %zu is null", what, i);
+    if (reinterpret_cast<uintptr_t>(p[i]) & 15)
+      return fail(MPRESS_ERR_ALIGN, "%s: pointer %zu (%p) is not 16-byte aligned", what, i, p[i]);
+  }
+  return MPRESS_OK;
+}
+
+int cuda_fail(cudaError_t e, const char* what) {
+  return fail(MPRESS_ERR_CUDA, "%s: %s", what, cudaGetErrorString(e));
+}
+
+// Move every descriptor on `stream` with the context's path.
+int run_copy(mpress_ctx_s* c, int dir, const std::vector<CopyDesc>& d,
+             const std::vector<int>& desc_peer, cudaStream_t stream) {
+  c->last_launches = 0;
+  if (c->path != MPRESS_PATH_CE)
+    return launch_copy(c->path, dir, d.data(), d.size(), c->max_ctas, stream, &c->last_launches);
+
+  // Copy-engine comparator: cudaMemcpyAsync per stripe, one side stream per
+  // peer so the engines of different peers overlap; fork/join by events.
+  if (c->ce_streams.empty()) {
+    c->ce_streams.assign(c->world, nullptr);
+    for (int p = 0; p < c->world; ++p) {
+      cudaError_t e = cudaStreamCreateWithFlags(&c->ce_streams[p], cudaStreamNonBlocking);
+      if (e != cudaSuccess) return cuda_fail(e, "cudaStreamCreate (copy-engine path)");
+    }
+  }
+  cudaEvent_t fork = take_event(c);
+  if (!fork) return fail(MPRESS_ERR_CUDA, "cudaEventCreate failed");
+  cudaEventRecord(fork, stream);
+  std::vector<char> used(c->world, 0);
+  for (int p : desc_peer) used[p] = 1;
+  int rc = MPRESS_OK;
+  std::vector<cudaEvent_t> joins;
+  for (int p = 0; p < c->world && rc == MPRESS_OK; ++p) {
+    if (!used[p]) continue;
+    cudaStream_t s = c->ce_streams[p];
+    cudaStreamWaitEvent(s, fork, 0);
+    for (size_t i = 0; i < d.size(); ++i) {
+      if (desc_peer[i] != p) continue;
+      cudaError_t e = cudaMemcpyAsync(d[i].dst, d[i].src, d[i].len, cudaMemcpyDefault, s);
+      if (e != cudaSuccess) { rc = cuda_fail(e, "cudaMemcpyAsync (copy-engine path)"); break; }
+    }
+    cudaEvent_t j = take_event(c);
+    cudaEventRecord(j, s);
+    cudaStreamWaitEvent(stream, j, 0);
+    joins.push_back(j);
+  }
+  // Events may be re-recorded once the waits above are enqueued.
+  give_event(c, fork);
+  for (auto j : joins) give_event(c, j);
+  return rc;
+}
+
+}  // namespace
+}  // namespace mpress
+
+using namespace mpress;
+
+extern "C" int mpress_swap_out(mpress_ctx_t* c, const mpress_plan_t* plan_, void* const* tensors,
+                               void* stream_, void* after, mpress_handle_t** out) {
+  if (!c || !plan_ || !out) return fail(MPRESS_ERR_ARG, "mpress_swap_out: null argument");
+  *out = nullptr;
+  std::lock_guard<std::mutex> lk(c->mu);
+  const uint64_t *units, *peer_bytes;
+  const mpress_stripe* st;
+  uint32_t n_st;
+  mpress_plan_info info;
+  MP_TRY(mpress_plan_get_info(plan_, &info));
+  MP_TRY(mpress_plan_units(plan_, &units));
+  MP_TRY(mpress_plan_stripes(plan_, &st, &n_st, &peer_bytes));
+  if (info.world != c->world || info.source != c->source)
+    return fail(MPRESS_ERR_PEER, "mpress_swap_out: plan is for source %d of %d, context serves %d of %d",
+                info.source, info.world, c->source, c->world);
+  MP_TRY(check_ptrs(tensors, info.n_tensors, "mpress_swap_out(tensors)"));
+  DeviceGuard g(c->device);
+  cudaStream_t stream = static_cast<cudaStream_t>(stream_);
+
+  auto* h = new mpress_handle_s();
+  h->ctx = c;
+  h->slice_off.assign(c->world, UINT64_MAX);
+  h->slice_len.assign(c->world, 0);
+  std::vector<cudaEvent_t> waits;
+  int rc = MPRESS_OK;
+  for (int p = 0; p < c->world && rc == MPRESS_OK; ++p) {
+    if (units[p] == 0) continue;
+    Partition& part = c->parts[p];
+    if (!part.base) {
+      rc = fail(MPRESS_ERR_PEER, "mpress_swap_out: peer %d is not mapped (partition 0)", p);
+      break;
+    }
+    reap_fences(c, &part);
+    const uint64_t len = units[p] * info.granule;
+    uint64_t off;
+    if (!alloc_slice(&part, len, &off)) {
+      rc = fail(MPRESS_ERR_NO_SPACE, "mpress_swap_out: no %llu-byte slice left in the partition on peer %d",
+                (unsigned long long)len, p);
+      break;
+    }
+    h->slice_off[p] = off;
+    h->slice_len[p] = len;
+    for (auto& f : part.fences)  // earlier swap-ins still reading these bytes
+      if (f.off < off + len && off < f.off + f.len) waits.push_back(f.ev);
+  }
+  if (rc != MPRESS_OK) {
+    for (int p = 0; p < c->world; ++p)
+      if (h->slice_off[p] != UINT64_MAX) free_slice(&c->parts[p], h->slice_off[p], h->slice_len[p]);
+    delete h;
+    return rc;
+  }
+  h->slices_held = true;
+  h->stripes.assign(st, st + n_st);
+  h->sizes.resize(info.n_tensors);
+
+  std::vector<CopyDesc> d(n_st);
+  std::vector<int> dp(n_st);
+  for (uint32_t i = 0; i < n_st; ++i) {
+    const mpress_stripe& s = st[i];
+    d[i].src = static_cast<const uint8_t*>(tensors[s.tensor]) + s.src_off;
+    d[i].dst = c->parts[s.peer].base + h->slice_off[s.peer] + s.dst_off;
+    d[i].len = s.len;
+    dp[i] = (int)s.peer;
+  }
+  for (auto e : waits) cudaStreamWaitEvent(stream, e, 0);
+  if (after) cudaStreamWaitEvent(stream, static_cast<cudaEvent_t>(after), 0);
+  h->out_done = take_event(c);
+  rc = h->out_done ? run_copy(c, kDirOut, d, dp, stream) : fail(MPRESS_ERR_CUDA, "cudaEventCreate failed");
+  if (rc == MPRESS_OK) {
+    cudaError_t e = cudaEventRecord(h->out_done, stream);
+    if (e != cudaSuccess) rc = cuda_fail(e, "cudaEventRecord(out_done)");
+  }
+  if (rc != MPRESS_OK) {
+    // Kernels may already be queued: keep the slices fenced by a sync.
+    cudaStreamSynchronize(stream);
+    for (int p = 0; p < c->world; ++p)
+      if (h->slice_off[p] != UINT64_MAX) free_slice(&c->parts[p], h->slice_off[p], h->slice_len[p]);
+    give_event(c, h->out_done);
+    delete h;
+    return rc;
+  }
+  h->state = MPRESS_STATE_OUT_PENDING;
+  c->handles.insert(h);
+  *out = h;
+  return MPRESS_OK;
+}
+
+extern "C" int mpress_swap_in(mpress_ctx_t* c, mpress_handle_t* h, void* const* dst, void* stream_) {
+  if (!c || !h) return fail(MPRESS_ERR_ARG, "mpress_swap_in: null argument");
+  std::lock_guard<std::mutex> lk(c->mu);
+  if (h->ctx != c || !c->handles.count(h)) return fail(MPRESS_ERR_ARG, "mpress_swap_in: handle not of this context");
+  if (h->state != MPRESS_STATE_OUT_PENDING && h->state != MPRESS_STATE_OUT)
+    return fail(MPRESS_ERR_STATE, "mpress_swap_in: handle is in state %d, not swapped out", h->state);
+  MP_TRY(check_ptrs(dst, h->sizes.size(), "mpress_swap_in(dst)"));
+  DeviceGuard g(c->device);
+  cudaStream_t stream = static_cast<cudaStream_t>(stream_);
+
+  std::vector<CopyDesc> d(h->stripes.size());
+  std::vector<int> dp(h->stripes.size());
+  for (size_t i = 0; i < h->stripes.size(); ++i) {
+    const mpress_stripe& s = h->stripes[i];
+    d[i].src = c->parts[s.peer].base + h->slice_off[s.peer] + s.dst_off;
+    d[i].dst = static_cast<uint8_t*>(dst[s.tensor]) + s.src_off;
+    d[i].len = s.len;
+    dp[i] = (int)s.peer;
+  }
+  cudaStreamWaitEvent(stream, h->out_done, 0);
+  if (!h->in_done) h->in_done = take_event(c);
+  if (!h->in_done) return fail(MPRESS_ERR_CUDA, "cudaEventCreate failed");
+  int rc = run_copy(c, kDirIn, d, dp, stream);
+  if (rc != MPRESS_OK) return rc;
+  cudaError_t e = cudaEventRecord(h->in_done, stream);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaEventRecord(in_done)");
+  h->state = MPRESS_STATE_IN_PENDING;
+
+  // Release the slices now; bytes stay fenced until this swap-in completes
+  // (the table entry is "updated when it completes").
+  for (int p = 0; p < c->world; ++p) {
+    if (h->slice_off[p] == UINT64_MAX) continue;
+    cudaEvent_t f = take_event(c);
+    if (!f || cudaEventRecord(f, stream) != cudaSuccess) {
+      cudaStreamSynchronize(stream);  // cannot fence: wait instead
+      give_event(c, f);
+    } else {
+      c->parts[p].fences.push_back({h->slice_off[p], h->slice_len[p], f});
+    }
+    free_slice(&c->parts[p], h->slice_off[p], h->slice_len[p]);
+  }
+  h->slices_held = false;
+  return MPRESS_OK;
+}
+
+extern "C" int mpress_wait(mpress_ctx_t* c, mpress_handle_t* h, void* consumer) {
+  if (!c || !h || h->ctx != c) return fail(MPRESS_ERR_ARG, "mpress_wait: bad argument");
+  DeviceGuard g(c->device);
+  cudaEvent_t e = (h->state == MPRESS_STATE_IN_PENDING || h->state == MPRESS_STATE_IN) ? h->in_done : h->out_done;
+  if (!e) return fail(MPRESS_ERR_STATE, "mpress_wait: nothing enqueued");
+  cudaError_t r = cudaStreamWaitEvent(static_cast<cudaStream_t>(consumer), e, 0);
+  if (r != cudaSuccess) return cuda_fail(r, "mpress_wait: cudaStreamWaitEvent");
+  return MPRESS_OK;
+}
+
+extern "C" int mpress_query(mpress_ctx_t* c, mpress_handle_t* h) {
+  if (!c || !h || h->ctx != c) return fail(MPRESS_ERR_ARG, "mpress_query: bad argument");
+  DeviceGuard g(c->device);
+  cudaEvent_t e;
+  int next;
+  switch (h->state) {
+    case MPRESS_STATE_OUT: case MPRESS_STATE_IN: return 1;
+    case MPRESS_STATE_OUT_PENDING: e = h->out_done; next = MPRESS_STATE_OUT; break;
+    case MPRESS_STATE_IN_PENDING: e = h->in_done; next = MPRESS_STATE_IN; break;
+    default: return fail(MPRESS_ERR_STATE, "mpress_query: bad state %d", h->state);
+  }
+  cudaError_t r = cudaEventQuery(e);
+  if (r == cudaSuccess) { h->state = next; return 1; }
+  if (r == cudaErrorNotReady) { cudaGetLastError(); return 0; }
+  return cuda_fail(r, "mpress_query: cudaEventQuery");
+}
+
+extern "C" int mpress_handle_state(const mpress_handle_t* h) { return h ? h->state : MPRESS_ERR_ARG; }
+
+extern "C" int mpress_handle_slices(const mpress_handle_t* h, uint64_t* slice_off) {
+  if (!h || !slice_off) return fail(MPRESS_ERR_ARG, "mpress_handle_slices: null argument");
+  std::copy(h->slice_off.begin(), h->slice_off.end(), slice_off);
+  return MPRESS_OK;
+}
+
+extern "C" int mpress_handle_free(mpress_ctx_t* c, mpress_handle_t* h, int force) {
+  if (!c || !h) return fail(MPRESS_ERR_ARG, "mpress_handle_free: null argument");
+  std::lock_guard<std::mutex> lk(c->mu);
+  if (h->ctx != c || !c->handles.count(h)) return fail(MPRESS_ERR_ARG, "mpress_handle_free: handle not of this context");
+  DeviceGuard g(c->device);
+  if (h->slices_held) {
+    if (!force)
+      return fail(MPRESS_ERR_STATE, "mpress_handle_free: data still only in the stash (state %d); swap in or force", h->state);
+    cudaEventSynchronize(h->out_done);  // swap-out kernels may still write the slices
+    for (int p = 0; p < c->world; ++p)
+      if (h->slice_off[p] != UINT64_MAX) free_slice(&c->parts[p], h->slice_off[p], h->slice_len[p]);
+  }
+  // An IN_PENDING handle's slices are covered by fences with their own events;
+  // its events go back to the pool only once they can no longer be waited on
+  // by this handle (it is being destroyed), and re-recording them later is
+  // ordered after everything already enqueued.
+  give_event(c, h->out_done);
+  give_event(c, h->in_done);
+  c->handles.erase(h);
+  delete h;
+  return MPRESS_OK;
+}

@@ -1,0 +1,65 @@
+"""Multi-process host logic on CPU (gloo, world size 2 and 3): the fd-passing
+rendezvous mpress_init uses for cuMem pool handles (SCM_RIGHTS over Unix
+sockets, csrc/fdpass.cpp), driven through the torch process-group exchange
+callback, and the rank-independence of plans/partitions (§8(b) multi-source:
+every rank computes the same table with no communication)."""
+import os
+import socket
+import tempfile
+
+import pytest
+import torch.multiprocessing as tmp
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    return port
+
+
+def _worker(rank, world, port, want_matrix, outdir):
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import paper_conf_hpca_zhouwylbyx23_b200 as mp
+    from synth import workloads
+
+    fd = os.memfd_create("mpress-test-%d" % rank)
+    os.write(fd, ("payload-of-rank-%d" % rank).encode())
+    cb = mp.torch_exchange()
+    fds = mp.share_fds(world, rank, fd, want_matrix[rank], cb)
+    got = {}
+    for p, f in enumerate(fds):
+        if f >= 0:
+            os.lseek(f, 0, os.SEEK_SET)
+            got[p] = os.read(f, 64).decode()
+            os.close(f)
+    os.close(fd)
+
+    # every rank computes the same partition table (no communication)
+    c = workloads.CONFIGS[5]
+    spare = workloads.spare_vector(8, 0, c["peers"], spare=c["spare"])
+    bwm = [workloads.bw_vector(8, s, c["peers"]) for s in range(8)]
+    reqs = [(s, workloads.cfg5_source_sizes(s), 2) for s in c["sources"]]
+    part = mp.partition_sequential(8, spare, bwm, reqs)
+    with open(os.path.join(outdir, "r%d.txt" % rank), "w") as f:
+        f.write(repr((got, part)))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,want", [
+    (2, [[0, 1], [1, 0]]),
+    (3, [[0, 1, 1], [0, 0, 0], [1, 1, 0]]),
+])
+def test_share_fds_gloo(world, want):
+    with tempfile.TemporaryDirectory() as d:
+        tmp.spawn(_worker, args=(world, _free_port(), want, d), nprocs=world, join=True)
+        results = [eval(open(os.path.join(d, "r%d.txt" % r)).read()) for r in range(world)]
+    for r, (got, part) in enumerate(results):
+        expect = {p: "payload-of-rank-%d" % p for p in range(world) if want[r][p] and p != r}
+        assert got == expect
+        assert part == results[0][1]
