@@ -1,0 +1,162 @@
+#!/usr/bin/env python
+"""Tuning sweeps on one B200 (loopback peers): swap GB/s per path x grid cap x
+size, and the slowdown of a concurrent bf16 GEMM (the second half of the
+BASELINE metric).  Prints one JSON object per row.  Not the bench: bench.py
+keeps the driver's contract; this explains it.
+
+  python tools/sweep.py paths        # cfg2 micro-batch, every path x cap
+  python tools/sweep.py sizes        # cfg4 sizes 4 KiB .. 4 GiB, 1/3/7 peers
+  python tools/sweep.py gemm         # GEMM slowdown vs swap path x cap
+"""
+import json
+import os
+import statistics
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import torch  # noqa: E402
+
+import paper_conf_hpca_zhouwylbyx23_b200 as mp  # noqa: E402
+from synth import device as synth_dev  # noqa: E402
+from synth import workloads  # noqa: E402
+
+PATHS = {"direct": mp.PATH_DIRECT, "bulk": mp.PATH_BULK, "ce": mp.PATH_CE}
+
+
+def setup(sizes, peers_n, copies=1):
+    world = peers_n + 1
+    peers = list(range(1, world))
+    spare = workloads.spare_vector(world, 0, peers, spare=64 << 30)
+    bw = workloads.bw_vector(world, 0, peers)
+    pl = mp.plan(world, 0, spare, bw, sizes)
+    part = [[0] * world for _ in range(world)]
+    part[0] = [copies * u * mp.DEFAULT_GRANULE for u in pl.units]
+    ctx = mp.Context.local(world, 0, [0] * world, part)
+    src = [torch.empty(s, dtype=torch.uint8, device="cuda") for s in sizes]
+    for i, t in enumerate(src):
+        synth_dev.fill(t, 77, i)
+    dst = [torch.empty(s, dtype=torch.uint8, device="cuda") for s in sizes]
+    return ctx, pl, src, dst
+
+
+def time_swaps(ctx, pl, src, dst, reps, stream):
+    outs, ins = [], []
+    for r in range(reps + 2):
+        e = [torch.cuda.Event(enable_timing=True) for _ in range(3)]
+        e[0].record(stream)
+        h = ctx.swap_out(pl, src, stream=stream)
+        e[1].record(stream)
+        ctx.swap_in(h, dst, stream=stream)
+        e[2].record(stream)
+        h.free()
+        if r >= 2:
+            outs.append(e)
+    torch.cuda.synchronize()
+    to = [a.elapsed_time(b) for a, b, c in outs]
+    ti = [b.elapsed_time(c) for a, b, c in outs]
+    return statistics.median(to), statistics.median(ti)
+
+
+def paths():
+    sizes = workloads.cfg2_sizes(1)
+    nbytes = sum(sizes)
+    ctx, pl, src, dst = setup(sizes, 3)
+    s = torch.cuda.Stream()
+    for name, path in PATHS.items():
+        caps = [0] if name == "ce" else [0, 4, 8, 16, 32, 64, 148, 296, 592]
+        for cap in caps:
+            ctx.set_option(mp.OPT_PATH, path)
+            ctx.set_option(mp.OPT_MAX_CTAS, cap)
+            to, ti = time_swaps(ctx, pl, src, dst, 10, s)
+            print(json.dumps({"sweep": "paths", "path": name, "max_ctas": cap,
+                              "out_gbs": nbytes / to / 1e6, "in_gbs": nbytes / ti / 1e6,
+                              "hbm_gbs_out": 2 * nbytes / to / 1e6}), flush=True)
+    ctx.finalize()
+
+
+def sizes_sweep():
+    s = torch.cuda.Stream()
+    for peers_n in (1, 3, 7):
+        for size in workloads.cfg4_sizes():
+            ctx, pl, src, dst = setup([size], peers_n)
+            for name in ("direct", "bulk", "ce"):
+                ctx.set_option(mp.OPT_PATH, PATHS[name])
+                reps = 20 if size < (256 << 20) else 5
+                to, ti = time_swaps(ctx, pl, src, dst, reps, s)
+                print(json.dumps({"sweep": "sizes", "peers": peers_n, "bytes": size, "path": name,
+                                  "out_gbs": size / to / 1e6, "in_gbs": size / ti / 1e6,
+                                  "out_us": to * 1e3, "in_us": ti * 1e3}), flush=True)
+            ctx.finalize()
+            del src, dst
+            torch.cuda.empty_cache()
+
+
+def gemm():
+    sizes = workloads.cfg2_sizes(1)
+    nbytes = sum(sizes)
+    ctx, pl, src, dst = setup(sizes, 3)
+    shapes = {"8192^3": (8192, 8192, 8192), "gpt_fc1": (4096, 5120, 20480)}
+    comp = torch.cuda.current_stream()
+    swap = torch.cuda.Stream()
+    for sname, (M, K, N) in shapes.items():
+        a = torch.randn(M, K, dtype=torch.bfloat16, device="cuda")
+        b = torch.randn(K, N, dtype=torch.bfloat16, device="cuda")
+        c = torch.empty(M, N, dtype=torch.bfloat16, device="cuda")
+
+        def gemms(n):
+            evs = []
+            for _ in range(n):
+                e0 = torch.cuda.Event(enable_timing=True)
+                e1 = torch.cuda.Event(enable_timing=True)
+                e0.record(comp)
+                torch.matmul(a, b, out=c)
+                e1.record(comp)
+                evs.append((e0, e1))
+            return evs
+
+        gemms(20)
+        torch.cuda.synchronize()
+        alone = statistics.median(x.elapsed_time(y) for x, y in gemms(60))
+        torch.cuda.synchronize()
+        print(json.dumps({"sweep": "gemm", "shape": sname, "mode": "alone", "gemm_ms": alone,
+                          "tflops": 2 * M * N * K / alone / 1e9}), flush=True)
+        for name in ("direct", "bulk", "ce"):
+            caps = [0] if name == "ce" else [4, 8, 16, 32, 0]
+            for cap in caps:
+                ctx.set_option(mp.OPT_PATH, PATHS[name])
+                ctx.set_option(mp.OPT_MAX_CTAS, cap)
+                # swaps looped on the side stream to cover the GEMM window
+                n_gemm = 60
+                window_ms = alone * n_gemm
+                to, ti = time_swaps(ctx, pl, src, dst, 3, swap)
+                n_swap = int(window_ms / (to + ti)) + 2
+                torch.cuda.synchronize()
+                sw0 = torch.cuda.Event(enable_timing=True)
+                sw1 = torch.cuda.Event(enable_timing=True)
+                sw0.record(swap)
+                for _ in range(n_swap):
+                    h = ctx.swap_out(pl, src, stream=swap)
+                    ctx.swap_in(h, dst, stream=swap)
+                    h.free()
+                sw1.record(swap)
+                evs = gemms(n_gemm)
+                torch.cuda.synchronize()
+                swap_ms = sw0.elapsed_time(sw1)
+                # only GEMMs that ran entirely inside the swap window
+                inside = [x.elapsed_time(y) for x, y in evs
+                          if sw0.elapsed_time(x) >= 0 and sw0.elapsed_time(y) <= swap_ms]
+                if not inside:
+                    inside = [float("nan")]
+                during = statistics.median(inside)
+                print(json.dumps({"sweep": "gemm", "shape": sname, "mode": "with_swap", "path": name,
+                                  "max_ctas": cap, "gemm_ms": during,
+                                  "slowdown": during / alone - 1,
+                                  "swap_gbs_under_gemm": 2 * n_swap * nbytes / swap_ms / 1e6}), flush=True)
+    ctx.finalize()
+
+
+if __name__ == "__main__":
+    what = sys.argv[1] if len(sys.argv) > 1 else "paths"
+    {"paths": paths, "sizes": sizes_sweep, "gemm": gemm}[what]()
