@@ -203,13 +203,20 @@ MPRESS_API int mpress_finalize(mpress_ctx_t* ctx);
 MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
 
 /* Tunables.  MPRESS_OPT_PATH: 0 = SM kernel, direct 16-B loads/stores
- * (default); 1 = SM kernel, bulk-async (TMA engine) staged through shared
- * memory; 2 = copy engines (cudaMemcpyAsync per stripe on per-peer streams,
- * the measured comparator).  MPRESS_OPT_MAX_CTAS: cap on the kernel grid
- * (0 = one wave of resident CTAs over all SMs); each CTA occupies one SM slot,
- * so this is the SM-count cap that protects a concurrent GEMM.            */
+ * (default); 1 = SM kernel, bulk-async copies (the SM's TMA engine,
+ * cp.async.bulk) staged through shared memory; 2 = copy engines
+ * (cudaMemcpyAsync per stripe on per-peer streams, the measured comparator).
+ * Setting the path resets the variant to 0.
+ * MPRESS_OPT_MAX_CTAS: cap on the kernel grid (0 = the variant's default
+ * grid, a multiple of the SM count); CTAs spread one per SM first, so this is
+ * the SM-count cap that protects a concurrent GEMM.
+ * MPRESS_OPT_VARIANT: kernel shape within the path -- direct: 0 = 256
+ * threads x 8 vectors (2 CTAs/SM by default), 1 = 512x8, 2 = 256x16,
+ * 3 = 1024x4; bulk: 0 = 6 slots x 32 KiB, 1 = 12 x 16 KiB, 2 = 3 x 64 KiB.
+ * Invalid values -> MPRESS_ERR_ARG. */
 #define MPRESS_OPT_PATH      1
 #define MPRESS_OPT_MAX_CTAS  2
+#define MPRESS_OPT_VARIANT   3
 #define MPRESS_PATH_DIRECT   0
 #define MPRESS_PATH_BULK     1
 #define MPRESS_PATH_CE       2

@@ -16,6 +16,7 @@
 #include <mutex>
 
 #include "ctx.h"
+#include "swap_kernels.h"
 
 namespace mpress {
 
@@ -327,11 +328,19 @@ extern "C" int mpress_set_option(mpress_ctx_t* c, int key, int64_t value) {
       if (value != MPRESS_PATH_DIRECT && value != MPRESS_PATH_BULK && value != MPRESS_PATH_CE)
         return fail(MPRESS_ERR_ARG, "unknown path %lld", (long long)value);
       c->path = (int)value;
+      c->variant = 0;  // variants are per path
       return MPRESS_OK;
     case MPRESS_OPT_MAX_CTAS:
       if (value < 0 || value > (1 << 20)) return fail(MPRESS_ERR_ARG, "bad max_ctas %lld", (long long)value);
       c->max_ctas = (int)value;
       return MPRESS_OK;
+    case MPRESS_OPT_VARIANT: {
+      const int nvar = c->path == MPRESS_PATH_BULK ? kBulkVariants : kDirectVariants;
+      if (value < 0 || value >= nvar)
+        return fail(MPRESS_ERR_ARG, "variant %lld out of range for path %d", (long long)value, c->path);
+      c->variant = (int)value;
+      return MPRESS_OK;
+    }
   }
   return fail(MPRESS_ERR_ARG, "unknown option %d", key);
 }
@@ -341,6 +350,7 @@ extern "C" int mpress_get_option(const mpress_ctx_t* c, int key, int64_t* value)
   switch (key) {
     case MPRESS_OPT_PATH: *value = c->path; return MPRESS_OK;
     case MPRESS_OPT_MAX_CTAS: *value = c->max_ctas; return MPRESS_OK;
+    case MPRESS_OPT_VARIANT: *value = c->variant; return MPRESS_OK;
   }
   return fail(MPRESS_ERR_ARG, "unknown option %d", key);
 }

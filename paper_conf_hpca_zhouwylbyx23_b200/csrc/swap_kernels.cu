@@ -26,6 +26,8 @@
 
 #include <algorithm>
 #include <mutex>
+#include <set>
+#include <utility>
 
 #include "common.h"
 #include "swap_kernels.h"
@@ -33,27 +35,19 @@
 namespace mpress {
 namespace {
 
-constexpr int kThreads = 256;                 // direct path CTA size
-constexpr int kUnroll = 8;                    // 16-B vectors in flight per thread
-constexpr uint32_t kChunk = kThreads * kUnroll * 16;  // 32 KiB per chunk
-constexpr uint32_t kChunkShift = 15;
-static_assert((1u << kChunkShift) == kChunk, "chunk must be a power of two");
-
-constexpr int kBulkThreads = 32;
-constexpr uint32_t kSlot = 32768;             // bytes per bulk piece / smem slot
-constexpr int kStages = 6;                    // 192 KiB of shared memory per CTA
-constexpr uint32_t kSlotShift = 15;
-static_assert((1u << kSlotShift) == kSlot, "slot must be a power of two");
-
+// Descriptor tables come in three capacities so a small swap does not ship a
+// 28 KB parameter block with its launch (launch latency grows with it).
+template <int CAP>
 struct CopyTable {
-  uint32_t n;                                  // descriptors
-  uint32_t total_chunks;                       // chunks over all descriptors
-  uint32_t first_chunk[kMaxDescPerLaunch + 1]; // prefix sum of chunks
-  CopyDesc d[kMaxDescPerLaunch];
+  uint32_t n;                   // descriptors
+  uint32_t total_chunks;        // chunks over all descriptors
+  uint32_t first_chunk[CAP + 1];  // prefix sum of chunks per descriptor
+  CopyDesc d[CAP];
 };
-static_assert(sizeof(CopyTable) <= 32764, "kernel parameter space is 32764 bytes");
+static_assert(sizeof(CopyTable<kMaxDescPerLaunch>) <= 32764, "kernel parameter space is 32764 bytes");
 
-__device__ __forceinline__ uint32_t find_desc(const CopyTable& t, uint32_t c) {
+template <int CAP>
+__device__ __forceinline__ uint32_t find_desc(const CopyTable<CAP>& t, uint32_t c) {
   // largest s with first_chunk[s] <= c (first_chunk[0] == 0)
   uint32_t lo = 0, hi = t.n;
   while (hi - lo > 1) {
@@ -75,36 +69,39 @@ __device__ __forceinline__ void st_stream(int4* p, const int4& v) {
                :: "l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
 }
 
-// Bytes [off, off+len) of one descriptor, len <= kChunk, by all kThreads threads.
-__device__ __forceinline__ void copy_partial(const uint8_t* src, uint8_t* dst, uint32_t len) {
-  const uint32_t n16 = len >> 4;
-  const int4* s = reinterpret_cast<const int4*>(src);
-  int4* o = reinterpret_cast<int4*>(dst);
-  for (uint32_t v = threadIdx.x; v < n16; v += kThreads) st_stream(o + v, ld_stream(s + v));
-  const uint32_t tail = len & 15u;
-  if (threadIdx.x < tail) dst[(n16 << 4) + threadIdx.x] = src[(n16 << 4) + threadIdx.x];
-}
-
-template <int DIR>
-__global__ void __launch_bounds__(kThreads)
-mp_swap_direct(const __grid_constant__ CopyTable t) {
+// ---------------------------------------------------------------- direct path
+// THREADS threads each keep UNROLL independent 16-B loads in flight, then
+// store them: one chunk = THREADS*UNROLL*16 bytes per CTA iteration.
+template <int DIR, int THREADS, int UNROLL, int CAP>
+__global__ void __launch_bounds__(THREADS)
+mp_swap_direct(const __grid_constant__ CopyTable<CAP> t) {
+  constexpr uint32_t kChunk = THREADS * UNROLL * 16;
+  static_assert((kChunk & (kChunk - 1)) == 0, "chunk must be a power of two");
+  constexpr uint32_t kShift = __builtin_ctz(kChunk);
   for (uint32_t c = blockIdx.x; c < t.total_chunks; c += gridDim.x) {
     const uint32_t s = find_desc(t, c);
     const CopyDesc& d = t.d[s];
-    const uint64_t off = (uint64_t)(c - t.first_chunk[s]) << kChunkShift;
+    const uint64_t off = (uint64_t)(c - t.first_chunk[s]) << kShift;
     const uint8_t* src = static_cast<const uint8_t*>(d.src) + off;
     uint8_t* dst = static_cast<uint8_t*>(d.dst) + off;
     const uint64_t rem = d.len - off;
     if (rem >= kChunk) {
       const int4* sv = reinterpret_cast<const int4*>(src) + threadIdx.x;
       int4* dv = reinterpret_cast<int4*>(dst) + threadIdx.x;
-      int4 v[kUnroll];
+      int4 v[UNROLL];
 #pragma unroll
-      for (int j = 0; j < kUnroll; ++j) v[j] = ld_stream(sv + j * kThreads);
+      for (int j = 0; j < UNROLL; ++j) v[j] = ld_stream(sv + j * THREADS);
 #pragma unroll
-      for (int j = 0; j < kUnroll; ++j) st_stream(dv + j * kThreads, v[j]);
+      for (int j = 0; j < UNROLL; ++j) st_stream(dv + j * THREADS, v[j]);
     } else {
-      copy_partial(src, dst, (uint32_t)rem);
+      // ragged last chunk of a stripe: 16-B body, then the <16-byte tail
+      const uint32_t len = (uint32_t)rem;
+      const uint32_t n16 = len >> 4;
+      const int4* sv = reinterpret_cast<const int4*>(src);
+      int4* dv = reinterpret_cast<int4*>(dst);
+      for (uint32_t v = threadIdx.x; v < n16; v += THREADS) st_stream(dv + v, ld_stream(sv + v));
+      const uint32_t tail = len & 15u;
+      if (threadIdx.x < tail) dst[(n16 << 4) + threadIdx.x] = src[(n16 << 4) + threadIdx.x];
     }
   }
 }
@@ -146,10 +143,7 @@ __device__ __forceinline__ void bulk_store(void* gdst, const void* smem, uint32_
 }
 
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void bulk_wait_read() {
-  asm volatile("cp.async.bulk.wait_group.read %0;" :: "n"(N) : "memory");
-}
+__device__ __forceinline__ void bulk_wait_read1() { asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 
 struct Piece {
@@ -158,29 +152,33 @@ struct Piece {
   uint32_t bytes;  // multiple of 16
 };
 
-__device__ __forceinline__ Piece bulk_piece(const CopyTable& t, uint32_t c) {
+template <int SHIFT, int CAP>
+__device__ __forceinline__ Piece bulk_piece(const CopyTable<CAP>& t, uint32_t c) {
   const uint32_t s = find_desc(t, c);
   const CopyDesc& d = t.d[s];
-  const uint64_t off = (uint64_t)(c - t.first_chunk[s]) << kSlotShift;
+  const uint64_t off = (uint64_t)(c - t.first_chunk[s]) << SHIFT;
   const uint64_t rem = d.len - off;
   Piece p;
   p.src = static_cast<const uint8_t*>(d.src) + off;
   p.dst = static_cast<uint8_t*>(d.dst) + off;
-  p.bytes = (uint32_t)(rem >= kSlot ? kSlot : (rem & ~15ull));
+  p.bytes = (uint32_t)(rem >= (1ull << SHIFT) ? (1ull << SHIFT) : (rem & ~15ull));
   return p;
 }
 
-template <int DIR>
-__global__ void __launch_bounds__(kBulkThreads)
-mp_swap_bulk(const __grid_constant__ CopyTable t) {
+// One warp per CTA: lane 0 streams pieces of 2^SHIFT bytes through STAGES
+// shared-memory slots with the SM's bulk-copy engine (cp.async.bulk G->S with
+// mbarrier completion, then S->G bulk stores); the warp first copies the
+// <16-byte tails the bulk engine cannot move.
+template <int DIR, int SHIFT, int STAGES, int CAP>
+__global__ void __launch_bounds__(32)
+mp_swap_bulk(const __grid_constant__ CopyTable<CAP> t) {
+  constexpr uint32_t kSlot = 1u << SHIFT;
   extern __shared__ __align__(128) uint8_t smem[];
-  __shared__ __align__(8) uint64_t bars[kStages];
+  __shared__ __align__(8) uint64_t bars[STAGES];
 
   const uint32_t first = blockIdx.x;
   const uint32_t mine = first < t.total_chunks ? (t.total_chunks - first + gridDim.x - 1) / gridDim.x : 0;
 
-  // Sub-16-byte tails (last chunk of a descriptor whose length % 16 != 0):
-  // plain byte copies by the warp, disjoint from every bulk piece.
   for (uint32_t i = 0; i < mine; ++i) {
     const uint32_t c = first + i * gridDim.x;
     const uint32_t s = find_desc(t, c);
@@ -194,29 +192,29 @@ mp_swap_bulk(const __grid_constant__ CopyTable t) {
   }
   if (threadIdx.x != 0 || mine == 0) return;
 
-  for (int k = 0; k < kStages; ++k) mbar_init(&bars[k], 1);
+  for (int k = 0; k < STAGES; ++k) mbar_init(&bars[k], 1);
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
 
   auto issue_load = [&](uint32_t i) {
-    const Piece p = bulk_piece(t, first + i * gridDim.x);
-    uint64_t* bar = &bars[i % kStages];
+    const Piece p = bulk_piece<SHIFT>(t, first + i * gridDim.x);
+    uint64_t* bar = &bars[i % STAGES];
     mbar_expect_tx(bar, p.bytes);
-    if (p.bytes) bulk_load(smem + (size_t)(i % kStages) * kSlot, p.src, p.bytes, bar);
+    if (p.bytes) bulk_load(smem + (size_t)(i % STAGES) * kSlot, p.src, p.bytes, bar);
   };
 
-  const uint32_t prologue = mine < (uint32_t)kStages ? mine : (uint32_t)kStages;
+  const uint32_t prologue = mine < (uint32_t)STAGES ? mine : (uint32_t)STAGES;
   for (uint32_t i = 0; i < prologue; ++i) issue_load(i);
   for (uint32_t i = 0; i < mine; ++i) {
-    mbar_wait(&bars[i % kStages], (i / kStages) & 1u);
-    const Piece p = bulk_piece(t, first + i * gridDim.x);
-    if (p.bytes) bulk_store(p.dst, smem + (size_t)(i % kStages) * kSlot, p.bytes);
+    mbar_wait(&bars[i % STAGES], (i / STAGES) & 1u);
+    const Piece p = bulk_piece<SHIFT>(t, first + i * gridDim.x);
+    if (p.bytes) bulk_store(p.dst, smem + (size_t)(i % STAGES) * kSlot, p.bytes);
     bulk_commit();
     // Refill the slot of piece i-1 once its store has finished reading smem
-    // (at most the newest group, piece i's store, may still be reading).
+    // (only the newest group, piece i's store, may still be reading).
     if (i >= 1) {
-      const uint32_t nxt = i - 1 + kStages;
+      const uint32_t nxt = i - 1 + STAGES;
       if (nxt < mine) {
-        bulk_wait_read<1>();
+        bulk_wait_read1();
         issue_load(nxt);
       }
     }
@@ -224,91 +222,140 @@ mp_swap_bulk(const __grid_constant__ CopyTable t) {
   bulk_wait_all();
 }
 
-struct WaveCache {
-  std::mutex mu;
-  int ctas[2][64] = {};
-};
-WaveCache g_wave;
+// ---------------------------------------------------------------- variants
 
-template <typename K>
-int wave_of(K kernel, int threads, size_t smem) {
-  int dev = 0, sms = 0, per_sm = 0;
-  if (cudaGetDevice(&dev) != cudaSuccess) return 0;
-  if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) return 0;
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, threads, smem) != cudaSuccess) return 0;
-  return sms * std::max(per_sm, 1);
+struct Shape {
+  int threads;
+  uint32_t shift;   // log2 bytes per chunk / bulk piece
+  size_t smem;      // dynamic shared memory
+  int per_sm;       // default CTAs per SM when MPRESS_OPT_MAX_CTAS = 0
+};
+
+// direct: (threads, unroll) = (256,8) (512,8) (256,16) (1024,4)
+// bulk:   (piece, stages)   = (32K,6) (16K,12) (64K,3)
+constexpr Shape kDirect[kDirectVariants] = {
+    {256, 15, 0, 2}, {512, 16, 0, 1}, {256, 16, 0, 2}, {1024, 16, 0, 1}};
+constexpr Shape kBulk[kBulkVariants] = {
+    {32, 15, 6u << 15, 1}, {32, 14, 12u << 14, 1}, {32, 16, 3u << 16, 1}};
+
+template <int CAP>
+using KernelFn = void (*)(CopyTable<CAP>);
+
+template <int CAP>
+KernelFn<CAP> kernel_for(int path, int variant, int dir) {
+  const bool o = dir == kDirOut;
+  if (path == MPRESS_PATH_BULK) {
+    switch (variant) {
+      case 1: return o ? mp_swap_bulk<kDirOut, 14, 12, CAP> : mp_swap_bulk<kDirIn, 14, 12, CAP>;
+      case 2: return o ? mp_swap_bulk<kDirOut, 16, 3, CAP> : mp_swap_bulk<kDirIn, 16, 3, CAP>;
+      default: return o ? mp_swap_bulk<kDirOut, 15, 6, CAP> : mp_swap_bulk<kDirIn, 15, 6, CAP>;
+    }
+  }
+  switch (variant) {
+    case 1: return o ? mp_swap_direct<kDirOut, 512, 8, CAP> : mp_swap_direct<kDirIn, 512, 8, CAP>;
+    case 2: return o ? mp_swap_direct<kDirOut, 256, 16, CAP> : mp_swap_direct<kDirIn, 256, 16, CAP>;
+    case 3: return o ? mp_swap_direct<kDirOut, 1024, 4, CAP> : mp_swap_direct<kDirIn, 1024, 4, CAP>;
+    default: return o ? mp_swap_direct<kDirOut, 256, 8, CAP> : mp_swap_direct<kDirIn, 256, 8, CAP>;
+  }
 }
 
-constexpr size_t kBulkSmem = (size_t)kStages * kSlot;
+const Shape& shape_of(int path, int variant) {
+  return path == MPRESS_PATH_BULK ? kBulk[variant] : kDirect[variant];
+}
 
-int configure_bulk_once() {
-  // The dynamic-smem opt-in is a per-device function attribute.
+// Per-device cache of "CTAs resident in one wave" and of the smem opt-in.
+struct DevCache {
+  std::mutex mu;
+  int wave[2][8][64] = {};
+};
+DevCache g_cache;
+
+// Opt a kernel into > 48 KB of dynamic shared memory, once per device.
+template <int CAP>
+int prepare(KernelFn<CAP> k, const Shape& sh) {
+  if (sh.smem <= 48 * 1024) return MPRESS_OK;
   static std::mutex mu;
-  static bool done[64] = {};
+  static std::set<std::pair<int, const void*>> done;
   int dev = 0;
-  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64)
-    return fail(MPRESS_ERR_CUDA, "cudaGetDevice failed");
+  if (cudaGetDevice(&dev) != cudaSuccess) return fail(MPRESS_ERR_CUDA, "cudaGetDevice failed");
   std::lock_guard<std::mutex> lk(mu);
-  if (done[dev]) return MPRESS_OK;
-  cudaError_t err = cudaFuncSetAttribute(mp_swap_bulk<kDirOut>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBulkSmem);
-  if (err == cudaSuccess)
-    err = cudaFuncSetAttribute(mp_swap_bulk<kDirIn>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBulkSmem);
-  if (err != cudaSuccess)
-    return fail(MPRESS_ERR_CUDA, "cudaFuncSetAttribute(bulk smem): %s", cudaGetErrorString(err));
-  done[dev] = true;
+  if (done.count({dev, (const void*)k})) return MPRESS_OK;
+  cudaError_t e = cudaFuncSetAttribute((const void*)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sh.smem);
+  if (e != cudaSuccess) return fail(MPRESS_ERR_CUDA, "cudaFuncSetAttribute(smem): %s", cudaGetErrorString(e));
+  done.insert({dev, (const void*)k});
+  return MPRESS_OK;
+}
+
+template <int CAP>
+int launch_table(int path, int variant, int dir, const CopyTable<CAP>& t, unsigned grid,
+                 cudaStream_t stream) {
+  const Shape& sh = shape_of(path, variant);
+  KernelFn<CAP> k = kernel_for<CAP>(path, variant, dir);
+  MP_TRY(prepare<CAP>(k, sh));
+  k<<<grid, sh.threads, sh.smem, stream>>>(t);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return fail(MPRESS_ERR_CUDA, "swap kernel launch: %s", cudaGetErrorString(e));
+  return MPRESS_OK;
+}
+
+template <int CAP>
+int launch_batch(int path, int variant, int dir, const CopyDesc* d, uint32_t n, uint32_t shift,
+                 int cap, cudaStream_t stream, bool* launched) {
+  CopyTable<CAP> t;
+  t.n = n;
+  uint64_t chunks = 0;
+  for (uint32_t i = 0; i < n; ++i) {
+    t.d[i] = d[i];
+    t.first_chunk[i] = (uint32_t)chunks;
+    chunks += (d[i].len + (1ull << shift) - 1) >> shift;
+    if (chunks > 0xFFFFFFFFull) return fail(MPRESS_ERR_ARG, "swap batch exceeds 2^32 chunks");
+  }
+  t.first_chunk[n] = (uint32_t)chunks;
+  t.total_chunks = (uint32_t)chunks;
+  *launched = false;
+  if (chunks == 0) return MPRESS_OK;
+  const unsigned grid = (unsigned)std::min<uint64_t>(chunks, (uint64_t)cap);
+  MP_TRY(launch_table<CAP>(path, variant, dir, t, grid, stream));
+  *launched = true;
   return MPRESS_OK;
 }
 
 }  // namespace
 
-int copy_wave_ctas(int path) {
+int copy_wave_ctas(int path, int variant) {
   int dev = 0;
   if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return 0;
-  const int slot = path == MPRESS_PATH_BULK ? 1 : 0;
-  std::lock_guard<std::mutex> lk(g_wave.mu);
-  if (g_wave.ctas[slot][dev] == 0) {
-    if (slot == 1) {
-      if (configure_bulk_once() != MPRESS_OK) return 0;
-      g_wave.ctas[slot][dev] = wave_of(mp_swap_bulk<kDirOut>, kBulkThreads, kBulkSmem);
-    } else {
-      g_wave.ctas[slot][dev] = wave_of(mp_swap_direct<kDirOut>, kThreads, 0);
-    }
+  const int pi = path == MPRESS_PATH_BULK ? 1 : 0;
+  std::lock_guard<std::mutex> lk(g_cache.mu);
+  int& w = g_cache.wave[pi][variant][dev];
+  if (w == 0) {
+    const Shape& sh = shape_of(path, variant);
+    KernelFn<kMaxDescPerLaunch> k = kernel_for<kMaxDescPerLaunch>(path, variant, kDirOut);
+    if (prepare<kMaxDescPerLaunch>(k, sh) != MPRESS_OK) return 0;
+    int sms = 0, per_sm = 0;
+    if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) return 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, (const void*)k, sh.threads, sh.smem) != cudaSuccess)
+      return 0;
+    w = sms * std::max(1, std::min(per_sm, sh.per_sm));
   }
-  return g_wave.ctas[slot][dev];
+  return w;
 }
 
-int launch_copy(int path, int dir, const CopyDesc* d, size_t n, int max_ctas,
+int launch_copy(int path, int variant, int dir, const CopyDesc* d, size_t n, int max_ctas,
                 cudaStream_t stream, int* launches) {
-  const bool bulk = path == MPRESS_PATH_BULK;
-  if (bulk) MP_TRY(configure_bulk_once());
-  const int wave = copy_wave_ctas(path);
+  const int nvar = path == MPRESS_PATH_BULK ? kBulkVariants : kDirectVariants;
+  if (variant < 0 || variant >= nvar) return fail(MPRESS_ERR_ARG, "kernel variant %d out of range", variant);
+  const int wave = copy_wave_ctas(path, variant);
   if (wave <= 0) return fail(MPRESS_ERR_CUDA, "occupancy query failed");
-  const int cap = max_ctas > 0 ? std::min(max_ctas, wave) : wave;
-  const uint32_t shift = bulk ? kSlotShift : kChunkShift;
+  const int cap = max_ctas > 0 ? max_ctas : wave;
+  const uint32_t shift = shape_of(path, variant).shift;
   for (size_t base = 0; base < n; base += kMaxDescPerLaunch) {
-    CopyTable t;
-    t.n = (uint32_t)std::min<size_t>(kMaxDescPerLaunch, n - base);
-    uint64_t chunks = 0;
-    for (uint32_t i = 0; i < t.n; ++i) {
-      t.d[i] = d[base + i];
-      t.first_chunk[i] = (uint32_t)chunks;
-      chunks += (d[base + i].len + (1ull << shift) - 1) >> shift;
-      if (chunks > 0xFFFFFFFFull) return fail(MPRESS_ERR_ARG, "swap batch exceeds 2^32 chunks");
-    }
-    t.first_chunk[t.n] = (uint32_t)chunks;
-    t.total_chunks = (uint32_t)chunks;
-    if (chunks == 0) continue;
-    const unsigned grid = (unsigned)std::min<uint64_t>(chunks, (uint64_t)cap);
-    if (bulk) {
-      if (dir == kDirOut) mp_swap_bulk<kDirOut><<<grid, kBulkThreads, kBulkSmem, stream>>>(t);
-      else mp_swap_bulk<kDirIn><<<grid, kBulkThreads, kBulkSmem, stream>>>(t);
-    } else {
-      if (dir == kDirOut) mp_swap_direct<kDirOut><<<grid, kThreads, 0, stream>>>(t);
-      else mp_swap_direct<kDirIn><<<grid, kThreads, 0, stream>>>(t);
-    }
-    cudaError_t e = cudaGetLastError();
-    if (e != cudaSuccess) return fail(MPRESS_ERR_CUDA, "swap kernel launch: %s", cudaGetErrorString(e));
-    if (launches) ++*launches;
+    const uint32_t m = (uint32_t)std::min<size_t>(kMaxDescPerLaunch, n - base);
+    bool launched = false;
+    if (m <= 16) MP_TRY(launch_batch<16>(path, variant, dir, d + base, m, shift, cap, stream, &launched));
+    else if (m <= 128) MP_TRY(launch_batch<128>(path, variant, dir, d + base, m, shift, cap, stream, &launched));
+    else MP_TRY(launch_batch<kMaxDescPerLaunch>(path, variant, dir, d + base, m, shift, cap, stream, &launched));
+    if (launched && launches) ++*launches;
   }
   return MPRESS_OK;
 }

@@ -18,17 +18,19 @@ struct CopyDesc {
 };
 
 constexpr int kMaxDescPerLaunch = 1024;  // fits the 32 KB kernel-parameter space
+constexpr int kDirectVariants = 4;       // MPRESS_OPT_VARIANT range, direct path
+constexpr int kBulkVariants = 3;         // MPRESS_OPT_VARIANT range, bulk path
 
 enum CopyDir { kDirOut = 0, kDirIn = 1 };
 
 // Enqueue kernels moving every descriptor on `stream`; `path` is
-// MPRESS_PATH_DIRECT or MPRESS_PATH_BULK; `max_ctas` caps the grid (0 = one
-// full wave).  Adds the number of kernel launches to *launches.
-// Returns MPRESS_OK or MPRESS_ERR_CUDA (message set).
-int launch_copy(int path, int dir, const CopyDesc* d, size_t n, int max_ctas,
+// MPRESS_PATH_DIRECT or MPRESS_PATH_BULK, `variant` its kernel shape;
+// `max_ctas` caps the grid (0 = the variant's default grid).  Adds the number
+// of kernel launches to *launches.  Returns MPRESS_OK or MPRESS_ERR_*.
+int launch_copy(int path, int variant, int dir, const CopyDesc* d, size_t n, int max_ctas,
                 cudaStream_t stream, int* launches);
 
-// CTAs of the given path that fit on one wave of the current device.
-int copy_wave_ctas(int path);
+// Default grid of a path/variant on the current device (SMs x CTAs per SM).
+int copy_wave_ctas(int path, int variant);
 
 }  // namespace mpress

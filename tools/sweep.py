@@ -64,15 +64,19 @@ def paths():
     nbytes = sum(sizes)
     ctx, pl, src, dst = setup(sizes, 3)
     s = torch.cuda.Stream()
+    nvar = {"direct": 4, "bulk": 3, "ce": 1}
     for name, path in PATHS.items():
-        caps = [0] if name == "ce" else [0, 4, 8, 16, 32, 64, 148, 296, 592]
-        for cap in caps:
-            ctx.set_option(mp.OPT_PATH, path)
-            ctx.set_option(mp.OPT_MAX_CTAS, cap)
-            to, ti = time_swaps(ctx, pl, src, dst, 10, s)
-            print(json.dumps({"sweep": "paths", "path": name, "max_ctas": cap,
-                              "out_gbs": nbytes / to / 1e6, "in_gbs": nbytes / ti / 1e6,
-                              "hbm_gbs_out": 2 * nbytes / to / 1e6}), flush=True)
+        caps = [0] if name == "ce" else [0, 8, 16, 32, 64, 148, 296, 444, 592]
+        for var in range(nvar[name]):
+            for cap in caps:
+                ctx.set_option(mp.OPT_PATH, path)
+                if name != "ce":
+                    ctx.set_option(mp.OPT_VARIANT, var)
+                ctx.set_option(mp.OPT_MAX_CTAS, cap)
+                to, ti = time_swaps(ctx, pl, src, dst, 10, s)
+                print(json.dumps({"sweep": "paths", "path": name, "variant": var, "max_ctas": cap,
+                                  "out_gbs": nbytes / to / 1e6, "in_gbs": nbytes / ti / 1e6,
+                                  "hbm_gbs_out": 2 * nbytes / to / 1e6}), flush=True)
     ctx.finalize()
 
 
@@ -118,7 +122,9 @@ def gemm():
 
         gemms(20)
         torch.cuda.synchronize()
-        alone = statistics.median(x.elapsed_time(y) for x, y in gemms(60))
+        evs = gemms(60)
+        torch.cuda.synchronize()
+        alone = statistics.median(x.elapsed_time(y) for x, y in evs)
         torch.cuda.synchronize()
         print(json.dumps({"sweep": "gemm", "shape": sname, "mode": "alone", "gemm_ms": alone,
                           "tflops": 2 * M * N * K / alone / 1e9}), flush=True)
