@@ -55,6 +55,9 @@ def parse():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
+    ap.add_argument("--gemm-cap", type=int, default=32,
+                    help="swap grid cap (CTAs = SMs touched) while the concurrent GEMM runs")
+    ap.add_argument("--no-gemm", action="store_true")
     return ap.parse_args()
 
 
@@ -382,6 +385,8 @@ def main():
     per_dir = {k: bytes_per_mb / (statistics.mean(v) / 1e3) / 1e9 for k, v in dur.items()}
 
     e2e = run_e2e(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap_stream, n, dist)
+    gemm = None if args.no_gemm else gemm_interference(args, ctx, mp, world, source, per_copy, bw,
+                                                        sizes, src, dst, swap_stream, n, dist)
 
     cpu = None
     if rank == 0 and n == 1 and not args.no_cpu_baseline:
@@ -396,7 +401,7 @@ def main():
             "config": workload_config(args, n),
             "per_direction_gbs": per_dir,
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
-            "gpu_launches": launches[0], "clocks": clk,
+            "gpu_launches": launches[0], "clocks": clk, "gemm_slowdown": gemm,
             "parity": "round trip bit-exact vs generator (all %d tensors x %d ranks)" % (47 * mb, n),
         }
         print(json.dumps(line))
@@ -417,6 +422,81 @@ def traffic_from_profile():
         except Exception:
             return None
     return None
+
+
+def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap, n, dist):
+    """Second half of the metric: slowdown of a bf16 GEMM (8192^3, the shape
+    MEASURED_PEAKS.json is quoted on) on the compute stream while swaps loop on
+    the side stream with the grid capped at --gemm-cap CTAs.  Alone and
+    with-swap rounds alternate (so power-cap drift hits both), and only GEMMs
+    that ran entirely inside the swap window count."""
+    import torch
+    comp = torch.cuda.current_stream()
+    M = K = N = 8192
+    a = torch.randn(M, K, dtype=torch.bfloat16, device="cuda")
+    b = torch.randn(K, N, dtype=torch.bfloat16, device="cuda")
+    c = torch.empty(M, N, dtype=torch.bfloat16, device="cuda")
+    G = 24
+
+    def gemms():
+        evs = []
+        for _ in range(G):
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(comp)
+            torch.matmul(a, b, out=c)
+            e1.record(comp)
+            evs.append((e0, e1))
+        return evs
+
+    pl = mp.plan(world, source, per_copy, bw, sizes)
+    old_cap = ctx.get_option(mp.OPT_MAX_CTAS)
+    ctx.set_option(mp.OPT_MAX_CTAS, args.gemm_cap)
+    # swap time at this cap, to size the loop that must cover the GEMM window
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    e0.record(swap)
+    h = ctx.swap_out(pl, src[0], stream=swap)
+    ctx.swap_in(h, dst[0], stream=swap)
+    e1.record(swap)
+    h.free()
+    gemms()
+    torch.cuda.synchronize()
+    per_swap_ms = e0.elapsed_time(e1)
+    alone, during, swap_gbs = [], [], []
+    for _ in range(3):
+        evs = gemms()
+        torch.cuda.synchronize()
+        alone += [x.elapsed_time(y) for x, y in evs[4:]]
+        gemm_ms = statistics.median(alone)
+        n_swap = int(2.0 * G * gemm_ms / per_swap_ms) + 2
+        s0 = torch.cuda.Event(enable_timing=True)
+        s1 = torch.cuda.Event(enable_timing=True)
+        s0.record(swap)
+        for _ in range(n_swap):
+            h = ctx.swap_out(pl, src[0], stream=swap)
+            ctx.swap_in(h, dst[0], stream=swap)
+            h.free()
+        s1.record(swap)
+        evs = gemms()
+        torch.cuda.synchronize()
+        win = s0.elapsed_time(s1)
+        during += [x.elapsed_time(y) for x, y in evs[4:]
+                   if s0.elapsed_time(x) >= 0 and s0.elapsed_time(y) <= win]
+        swap_gbs.append(2 * n_swap * sum(sizes) / win / 1e6)
+    ctx.set_option(mp.OPT_MAX_CTAS, old_cap)
+    t = torch.tensor([statistics.median(alone), statistics.median(during) if during else float("nan")],
+                     dtype=torch.float64, device="cuda")
+    if n > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    a_ms, d_ms = float(t[0]), float(t[1])
+    return {"gemm": "bf16 8192x8192x8192 torch.matmul (cuBLAS) on the compute stream",
+            "alone_ms": a_ms, "with_swap_ms": d_ms, "slowdown": d_ms / a_ms - 1,
+            "swap_path": args.path, "swap_max_ctas": args.gemm_cap,
+            "swap_gbs_during": statistics.median(swap_gbs),
+            "gemms_counted": len(during),
+            "note": "N=1 loopback: the swap's bytes also load the GEMM's HBM (2 B per swapped "
+                    "byte), a harsher case than NVLink (1 B of source HBM per byte)"}
 
 
 def run_e2e(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, stream, n, dist):
