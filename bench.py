@@ -237,9 +237,16 @@ def main():
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
     n = world_env
-    torch.cuda.set_device(local_rank)
+    # One rank per GPU.  Ranks sharing a GPU (only in the 1-GPU test of this
+    # code path) use gloo alone; the reductions below are on CPU tensors, so
+    # nothing on the swap path depends on the collective backend.
+    ngpu = torch.cuda.device_count()
+    device = local_rank % ngpu
+    torch.cuda.set_device(device)
     if n > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        shared = int(os.environ.get("LOCAL_WORLD_SIZE", n)) > ngpu
+        dist.init_process_group("gloo" if shared else "cpu:gloo,cuda:nccl")
+    local_rank = device
 
     import paper_conf_hpca_zhouwylbyx23_b200 as mp
     from synth import device as synth_dev
@@ -338,7 +345,7 @@ def main():
     torch.cuda.synchronize()
     clk = clocks.stop()
     ms = t_start.elapsed_time(t_end)
-    ms_t = torch.tensor([ms], dtype=torch.float64, device="cuda")
+    ms_t = torch.tensor([ms], dtype=torch.float64)
     if n > 1:
         dist.all_reduce(ms_t, op=dist.ReduceOp.MAX)
     ms_max = float(ms_t.item())
@@ -351,7 +358,7 @@ def main():
     for m in range(mb):
         for i, t in enumerate(dst[m]):
             bad += synth_dev.check(t, seed0 + m, i)
-    bad_t = torch.tensor([bad], dtype=torch.int64, device="cuda")
+    bad_t = torch.tensor([bad], dtype=torch.int64)
     if n > 1:
         dist.all_reduce(bad_t)
     if int(bad_t.item()) != 0:
@@ -486,7 +493,7 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
         swap_gbs.append(2 * n_swap * sum(sizes) / win / 1e6)
     ctx.set_option(mp.OPT_MAX_CTAS, old_cap)
     t = torch.tensor([statistics.median(alone), statistics.median(during) if during else float("nan")],
-                     dtype=torch.float64, device="cuda")
+                     dtype=torch.float64)
     if n > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     a_ms, d_ms = float(t[0]), float(t[1])
@@ -541,7 +548,7 @@ def run_e2e(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, stream,
     e1.record(stream)
     torch.cuda.synchronize()
     ms = e0.elapsed_time(e1)
-    t = torch.tensor([ms], dtype=torch.float64, device="cuda")
+    t = torch.tensor([ms], dtype=torch.float64)
     if n > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     ms = float(t.item()) / steps

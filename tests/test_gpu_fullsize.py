@@ -1,0 +1,106 @@
+"""Full-size parity at BASELINE.json's sizes, in the launch configuration
+bench.py times (default path and grid): sampled stash windows against the
+oracle's plan + the generator (the oracle computes each window one by one),
+and the round trip checked on the device against the generator for every
+byte.  Plus compute-sanitizer memcheck of the smoke path."""
+import os
+import random
+import shutil
+import subprocess
+import sys
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import paper_conf_hpca_zhouwylbyx23_b200 as mp
+from synth import device as synth_dev
+from synth import splitmix64_bytes, workloads
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _sampled_roundtrip(world, source, spare, bw, sizes, seed, samples=64):
+    o = oracle.plan(world, source, spare, bw, sizes)
+    pl = mp.plan(world, source, spare, bw, sizes)
+    assert pl.stripes == [tuple(s) for s in o["stripes"]]
+    assert pl.units == o["units"] and pl.peer_bytes == o["peer_bytes"]
+    part = [[0] * world for _ in range(world)]
+    part[source] = [u * o["G"] for u in pl.units]
+    ctx = mp.Context.local(world, source, [0] * world, part)
+    try:
+        src = []
+        for i, n in enumerate(sizes):
+            t = torch.empty(n, dtype=torch.uint8, device="cuda")
+            synth_dev.fill(t, seed, i)
+            src.append(t)
+        s = torch.cuda.Stream()
+        h = ctx.swap_out(pl, src, stream=s)
+        s.synchronize()
+        sl = h.slices()
+        rng = random.Random(seed)
+        picks = list(o["stripes"])
+        rng.shuffle(picks)
+        # first/last bytes of every stripe + random interior windows
+        for (i, p, so, do, ln) in o["stripes"]:
+            for x in (0, max(0, ln - 4096)):
+                n = min(4096, ln - x)
+                got = np.frombuffer(ctx.peer_read(p, sl[p] + do + x, n), dtype=np.uint8)
+                assert np.array_equal(got, splitmix64_bytes(seed, i, so + x, n)), (i, p, x)
+        for (i, p, so, do, ln) in picks[:samples]:
+            x = rng.randrange(0, ln)
+            n = min(1 << 16, ln - x)
+            got = np.frombuffer(ctx.peer_read(p, sl[p] + do + x, n), dtype=np.uint8)
+            assert np.array_equal(got, splitmix64_bytes(seed, i, so + x, n)), (i, p, x)
+        del src
+        torch.cuda.empty_cache()
+        dst = [torch.empty(n, dtype=torch.uint8, device="cuda") for n in sizes]
+        ctx.swap_in(h, dst, stream=s)
+        s.synchronize()
+        for i, d in enumerate(dst):
+            assert synth_dev.check(d, seed, i) == 0, i
+        h.free()
+    finally:
+        ctx.finalize()
+    return o
+
+
+def test_config3_gpt_adam_states_full_size():
+    """BJ:9: 100 fp32 Adam m/v tensors (12.21 GB) -> peers 5,6,7 with 8/8/2 GiB
+    spare: the cap binds on peer 7 (water-fill)."""
+    c = workloads.CONFIGS[3]
+    spare = workloads.spare_vector(8, 0, c["peers"], spare_by_peer=c["spare_by_peer"])
+    bw = workloads.bw_vector(8, 0, c["peers"])
+    o = _sampled_roundtrip(8, 0, spare, bw, workloads.cfg3_sizes(), seed=3000)
+    assert o["units"][7] * o["G"] == 2 << 30
+
+
+def test_config4_largest_size_seven_peers():
+    """BJ:10: one 4 GiB uint8 tensor striped over 7 peers."""
+    peers = list(range(1, 8))
+    spare = workloads.spare_vector(8, 0, peers, spare=8 << 30)
+    bw = workloads.bw_vector(8, 0, peers)
+    _sampled_roundtrip(8, 0, spare, bw, [4 << 30], seed=4000)
+
+
+def test_config2_x8_single_batch_full_size():
+    """BJ:8: the 8 in-flight micro-batches (376 tensors, 7.03 GiB) as one plan
+    over 3 peers."""
+    peers = [1, 2, 3]
+    spare = workloads.spare_vector(4, 0, peers, spare=24 << 30)
+    bw = workloads.bw_vector(4, 0, peers)
+    _sampled_roundtrip(4, 0, spare, bw, workloads.cfg2_sizes(8), seed=2000)
+
+
+@pytest.mark.skipif(shutil.which("compute-sanitizer") is None and
+                    not os.path.exists("/usr/local/cuda/bin/compute-sanitizer"),
+                    reason="compute-sanitizer not installed")
+def test_memcheck_smoke():
+    cs = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitizer"
+    r = subprocess.run([cs, "--tool", "memcheck", "--error-exitcode", "9", sys.executable, "-c",
+                        "import __graft_entry__ as g; g.smoke()"],
+                       cwd=ROOT, capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0, (r.stdout[-3000:], r.stderr[-3000:])
+    assert "ERROR SUMMARY: 0 errors" in r.stdout + r.stderr

@@ -86,3 +86,94 @@ def test_two_processes_one_gpu(path):
         tmp.spawn(_worker, args=(2, _free_port(), d, path), nprocs=2, join=True)
         for r in range(2):
             assert open(os.path.join(d, "r%d.txt" % r)).read() == "ok"
+
+
+def _cfg5_worker(rank, world, port, outdir):
+    """Config 5 topology (Table IV): sources 0-3 swap (4-s) scaled
+    Bert micro-batch sets into importers 4-7 concurrently; sequential partition
+    (R12) computed identically on every rank."""
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    torch.cuda.set_device(0)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import oracle
+    import paper_conf_hpca_zhouwylbyx23_b200 as mp
+    from synth import device as synth_dev
+    from synth import splitmix64_bytes, workloads
+
+    def sizes_of(s):  # 1/64-scale Bert sets, ragged tails
+        return [max(1, b // 64 + 7 * s) for b in workloads.cfg5_source_sizes(s)]
+
+    sources, peers = [0, 1, 2, 3], [4, 5, 6, 7]
+    spare = [0] * 4 + [400 << 20] * 4
+    bwm = [[1 if (s in sources and p in peers) else 0 for p in range(world)] for s in range(world)]
+    reqs = [(s, sizes_of(s), 1) for s in sources]
+    part = mp.partition_sequential(world, spare, bwm, reqs)
+    opart, oplans = oracle.sequential_partition(world, spare, bwm, reqs)
+    err = "" if part == opart else "partition differs from the oracle"
+    ctx = mp.Context.distributed(0, world, rank, part)
+    try:
+        if rank in sources and not err:
+            sizes = sizes_of(rank)
+            rem = list(spare)
+            for s in sources:   # the spare each source planned against
+                if s == rank:
+                    break
+                rem = [r - part[s][p] for p, r in enumerate(rem)]
+            pl = mp.plan(world, rank, rem, bwm[rank], sizes)
+            o = oplans[rank]
+            assert pl.stripes == [tuple(x) for x in o["stripes"]]
+            src = []
+            for i, n in enumerate(sizes):
+                t = torch.empty(n, dtype=torch.uint8, device="cuda")
+                synth_dev.fill(t, 5000 + rank, i)
+                src.append(t)
+            torch.cuda.synchronize()
+            h = ctx.swap_out(pl, src)
+            torch.cuda.synchronize()
+            host = [splitmix64_bytes(5000 + rank, i, 0, n) for i, n in enumerate(sizes)]
+            sl = h.slices()
+            for p, (buf, defined) in oracle.swap_out(o, host).items():
+                got = np.frombuffer(ctx.peer_read(p, sl[p], len(buf)), dtype=np.uint8)
+                assert not np.any((got != buf) & defined), "stash differs on peer %d" % p
+            dst = [torch.empty(n, dtype=torch.uint8, device="cuda") for n in sizes]
+            ctx.swap_in(h, dst)
+            torch.cuda.synchronize()
+            for i, d in enumerate(dst):
+                assert synth_dev.check(d, 5000 + rank, i) == 0
+            h.free()
+        dist.barrier()
+    except Exception as e:
+        err = repr(e)
+    finally:
+        ctx.finalize()
+    with open(os.path.join(outdir, "r%d.txt" % rank), "w") as f:
+        f.write(err or "ok")
+    dist.destroy_process_group()
+
+
+def test_config5_eight_processes_one_gpu():
+    with tempfile.TemporaryDirectory() as d:
+        tmp.spawn(_cfg5_worker, args=(8, _free_port(), d), nprocs=8, join=True)
+        for r in range(8):
+            assert open(os.path.join(d, "r%d.txt" % r)).read() == "ok", r
+
+
+def test_bench_torchrun_two_ranks_one_gpu():
+    """bench.py's N>1 path (every rank a source and an importer, mpress_init
+    over the process group) under torchrun, both ranks on the one GPU."""
+    import json
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
+           "--master-addr=127.0.0.1", "--master-port=%d" % _free_port(), "bench.py", "--gpus", "2",
+           "--steps", "3", "--warmup", "1", "--micro-batches", "2", "--e2e-steps", "1", "--no-gemm"]
+    r = subprocess.run(cmd, cwd=root, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stderr[-3000:]
+    line = json.loads([l for l in r.stdout.splitlines() if l.startswith("{")][-1])
+    assert line["n_gpus"] == 2 and line["value"] > 0 and line["roofline"]["bound"] == "nvlink"
+    assert "bit-exact" in line["parity"]
