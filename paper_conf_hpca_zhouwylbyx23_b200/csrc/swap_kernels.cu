@@ -1,27 +1,36 @@
 // sm_100a swap kernels: the byte movers of swap-out and swap-in
-// (SURVEY.md §8(a) rows a3 / a5; P:121, P:151, P:236).
+// (SURVEY.md §8(a) rows a3 / a5; P:121, P:151, P:153, P:209, P:236).
 //
 // The D2D swap moves bytes and computes nothing (tensor cores unused), so the
 // kernels are shaped by the memory system alone:
 //   * one launch per plan (the whole batch, "we also batch tensors"),
 //     descriptors passed as a __grid_constant__ parameter (no upload);
-//   * the batch is cut into fixed-size chunks that a grid of CTAs walks with a
-//     grid stride, so adjacent chunks are in flight on different SMs at once;
+//   * the descriptors are grouped by peer (the plan's stripes are sorted by
+//     peer) and the CTAs are split between the groups in proportion to the
+//     group's bytes, so every peer link carries its share concurrently for the
+//     whole swap -- the paper's "transmit them in parallel through disjoint
+//     links" with sub-blocks sized to the links, done at CTA
+//     granularity.  With several sources swapping at once (config 5, or every
+//     rank in the N-GPU bench) each peer's NVLink ingress is then shared by
+//     all sources all the time instead of every source converging on its
+//     first peer;
+//   * inside a group, fixed-size chunks are walked with a stride, so adjacent
+//     chunks are in flight on different SMs at once;
 //   * the grid is capped (MPRESS_OPT_MAX_CTAS) so a concurrent GEMM keeps
 //     most SMs;
 //   * every address is 16-B aligned (tensor pointers are checked; stripe
 //     offsets are multiples of 256, R6), so bodies move int4 / bulk pieces and
 //     only the last <16 bytes of a tensor take a byte loop.
 //
-// PATH_DIRECT: 256 threads, each issuing 8 independent 16-B loads before its
-//   8 stores (32 KiB per CTA in flight per chunk), L1 bypassed on both sides.
-//   Peer addresses route over NVLink by their VA; loads of peer memory bypass
-//   the local L2 (B300_MICROARCH.md "NVLink"), so depth of outstanding loads
-//   sets swap-in bandwidth (Little's law).
-// PATH_BULK: one warp per CTA drives the bulk-async copy engine of the SM
+// PATH_DIRECT: THREADS threads, each issuing UNROLL independent 16-B loads
+//   before its UNROLL stores, L1 bypassed on both sides.  Peer addresses
+//   route over NVLink by their VA; loads of peer memory bypass the local L2
+//   (B300_MICROARCH.md "NVLink"), so the depth of outstanding loads sets
+//   swap-in bandwidth (Little's law).
+// PATH_BULK: one warp per CTA drives the SM's bulk-async copy engine
 //   (cp.async.bulk, SASS UBLKCP): chunk loads land in a ring of shared-memory
 //   slots (mbarrier completion), then bulk stores drain them, so one SM keeps
-//   kStages*32 KiB in flight with a single issuing thread.
+//   STAGES x piece bytes in flight with a single issuing thread.
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -35,26 +44,48 @@
 namespace mpress {
 namespace {
 
+constexpr int kMaxGroups = 64;  // peers per launch (NVSwitch domains up to 64 GPUs)
+
 // Descriptor tables come in three capacities so a small swap does not ship a
 // 28 KB parameter block with its launch (launch latency grows with it).
 template <int CAP>
 struct CopyTable {
-  uint32_t n;                   // descriptors
-  uint32_t total_chunks;        // chunks over all descriptors
-  uint32_t first_chunk[CAP + 1];  // prefix sum of chunks per descriptor
+  uint32_t n;                        // descriptors
+  uint32_t n_groups;                 // runs of descriptors with the same peer
+  uint32_t n_workers;                // virtual workers over all groups
+  uint32_t pad;
+  uint32_t g_chunk[kMaxGroups + 1];  // first chunk of each group (prefix)
+  uint32_t g_worker[kMaxGroups + 1]; // first virtual worker of each group (prefix)
+  uint32_t first_chunk[CAP + 1];     // first chunk of each descriptor (prefix)
   CopyDesc d[CAP];
 };
 static_assert(sizeof(CopyTable<kMaxDescPerLaunch>) <= 32764, "kernel parameter space is 32764 bytes");
 
-template <int CAP>
-__device__ __forceinline__ uint32_t find_desc(const CopyTable<CAP>& t, uint32_t c) {
-  // largest s with first_chunk[s] <= c (first_chunk[0] == 0)
-  uint32_t lo = 0, hi = t.n;
+// largest i in [0, n) with a[i] <= x  (a[0] == 0 <= x)
+__device__ __forceinline__ uint32_t upper_idx(const uint32_t* a, uint32_t n, uint32_t x) {
+  uint32_t lo = 0, hi = n;
   while (hi - lo > 1) {
     uint32_t mid = (lo + hi) >> 1;
-    if (t.first_chunk[mid] <= c) lo = mid; else hi = mid;
+    if (a[mid] <= x) lo = mid; else hi = mid;
   }
   return lo;
+}
+
+// Virtual worker v of the table: its group, its rank in the group, the
+// group's worker count and chunk range.
+struct Worker {
+  uint32_t chunk0, nchunks, rank, count;
+};
+
+template <int CAP>
+__device__ __forceinline__ Worker worker_of(const CopyTable<CAP>& t, uint32_t v) {
+  const uint32_t g = upper_idx(t.g_worker, t.n_groups, v);
+  Worker w;
+  w.chunk0 = t.g_chunk[g];
+  w.nchunks = t.g_chunk[g + 1] - t.g_chunk[g];
+  w.rank = v - t.g_worker[g];
+  w.count = t.g_worker[g + 1] - t.g_worker[g];
+  return w;
 }
 
 __device__ __forceinline__ int4 ld_stream(const int4* p) {
@@ -78,30 +109,34 @@ mp_swap_direct(const __grid_constant__ CopyTable<CAP> t) {
   constexpr uint32_t kChunk = THREADS * UNROLL * 16;
   static_assert((kChunk & (kChunk - 1)) == 0, "chunk must be a power of two");
   constexpr uint32_t kShift = __builtin_ctz(kChunk);
-  for (uint32_t c = blockIdx.x; c < t.total_chunks; c += gridDim.x) {
-    const uint32_t s = find_desc(t, c);
-    const CopyDesc& d = t.d[s];
-    const uint64_t off = (uint64_t)(c - t.first_chunk[s]) << kShift;
-    const uint8_t* src = static_cast<const uint8_t*>(d.src) + off;
-    uint8_t* dst = static_cast<uint8_t*>(d.dst) + off;
-    const uint64_t rem = d.len - off;
-    if (rem >= kChunk) {
-      const int4* sv = reinterpret_cast<const int4*>(src) + threadIdx.x;
-      int4* dv = reinterpret_cast<int4*>(dst) + threadIdx.x;
-      int4 v[UNROLL];
+  for (uint32_t v = blockIdx.x; v < t.n_workers; v += gridDim.x) {
+    const Worker w = worker_of(t, v);
+    for (uint32_t k = w.rank; k < w.nchunks; k += w.count) {
+      const uint32_t c = w.chunk0 + k;
+      const uint32_t s = upper_idx(t.first_chunk, t.n, c);
+      const CopyDesc& d = t.d[s];
+      const uint64_t off = (uint64_t)(c - t.first_chunk[s]) << kShift;
+      const uint8_t* src = static_cast<const uint8_t*>(d.src) + off;
+      uint8_t* dst = static_cast<uint8_t*>(d.dst) + off;
+      const uint64_t rem = d.len - off;
+      if (rem >= kChunk) {
+        const int4* sv = reinterpret_cast<const int4*>(src) + threadIdx.x;
+        int4* dv = reinterpret_cast<int4*>(dst) + threadIdx.x;
+        int4 r[UNROLL];
 #pragma unroll
-      for (int j = 0; j < UNROLL; ++j) v[j] = ld_stream(sv + j * THREADS);
+        for (int j = 0; j < UNROLL; ++j) r[j] = ld_stream(sv + j * THREADS);
 #pragma unroll
-      for (int j = 0; j < UNROLL; ++j) st_stream(dv + j * THREADS, v[j]);
-    } else {
-      // ragged last chunk of a stripe: 16-B body, then the <16-byte tail
-      const uint32_t len = (uint32_t)rem;
-      const uint32_t n16 = len >> 4;
-      const int4* sv = reinterpret_cast<const int4*>(src);
-      int4* dv = reinterpret_cast<int4*>(dst);
-      for (uint32_t v = threadIdx.x; v < n16; v += THREADS) st_stream(dv + v, ld_stream(sv + v));
-      const uint32_t tail = len & 15u;
-      if (threadIdx.x < tail) dst[(n16 << 4) + threadIdx.x] = src[(n16 << 4) + threadIdx.x];
+        for (int j = 0; j < UNROLL; ++j) st_stream(dv + j * THREADS, r[j]);
+      } else {
+        // ragged last chunk of a stripe: 16-B body, then the <16-byte tail
+        const uint32_t len = (uint32_t)rem;
+        const uint32_t n16 = len >> 4;
+        const int4* sv = reinterpret_cast<const int4*>(src);
+        int4* dv = reinterpret_cast<int4*>(dst);
+        for (uint32_t x = threadIdx.x; x < n16; x += THREADS) st_stream(dv + x, ld_stream(sv + x));
+        const uint32_t tail = len & 15u;
+        if (threadIdx.x < tail) dst[(n16 << 4) + threadIdx.x] = src[(n16 << 4) + threadIdx.x];
+      }
     }
   }
 }
@@ -154,7 +189,7 @@ struct Piece {
 
 template <int SHIFT, int CAP>
 __device__ __forceinline__ Piece bulk_piece(const CopyTable<CAP>& t, uint32_t c) {
-  const uint32_t s = find_desc(t, c);
+  const uint32_t s = upper_idx(t.first_chunk, t.n, c);
   const CopyDesc& d = t.d[s];
   const uint64_t off = (uint64_t)(c - t.first_chunk[s]) << SHIFT;
   const uint64_t rem = d.len - off;
@@ -164,6 +199,29 @@ __device__ __forceinline__ Piece bulk_piece(const CopyTable<CAP>& t, uint32_t c)
   p.bytes = (uint32_t)(rem >= (1ull << SHIFT) ? (1ull << SHIFT) : (rem & ~15ull));
   return p;
 }
+
+// The chunks of this CTA, in order: for each of its virtual workers
+// (blockIdx.x, + gridDim.x, ...), that worker's chunks rank, rank+count, ...
+template <int CAP>
+struct MyChunks {
+  const CopyTable<CAP>& t;
+  uint32_t total = 0;
+  __device__ explicit MyChunks(const CopyTable<CAP>& tt) : t(tt) {
+    for (uint32_t v = blockIdx.x; v < t.n_workers; v += gridDim.x) total += count_of(worker_of(t, v));
+  }
+  __device__ static uint32_t count_of(const Worker& w) {
+    return w.rank < w.nchunks ? (w.nchunks - w.rank + w.count - 1) / w.count : 0;
+  }
+  __device__ uint32_t chunk(uint32_t i) const {
+    for (uint32_t v = blockIdx.x; v < t.n_workers; v += gridDim.x) {
+      const Worker w = worker_of(t, v);
+      const uint32_t n = count_of(w);
+      if (i < n) return w.chunk0 + w.rank + i * w.count;
+      i -= n;
+    }
+    return 0;  // unreachable for i < total
+  }
+};
 
 // One warp per CTA: lane 0 streams pieces of 2^SHIFT bytes through STAGES
 // shared-memory slots with the SM's bulk-copy engine (cp.async.bulk G->S with
@@ -176,12 +234,12 @@ mp_swap_bulk(const __grid_constant__ CopyTable<CAP> t) {
   extern __shared__ __align__(128) uint8_t smem[];
   __shared__ __align__(8) uint64_t bars[STAGES];
 
-  const uint32_t first = blockIdx.x;
-  const uint32_t mine = first < t.total_chunks ? (t.total_chunks - first + gridDim.x - 1) / gridDim.x : 0;
+  const MyChunks<CAP> my(t);
+  const uint32_t mine = my.total;
 
   for (uint32_t i = 0; i < mine; ++i) {
-    const uint32_t c = first + i * gridDim.x;
-    const uint32_t s = find_desc(t, c);
+    const uint32_t c = my.chunk(i);
+    const uint32_t s = upper_idx(t.first_chunk, t.n, c);
     if (c + 1 != t.first_chunk[s + 1]) continue;  // not the last chunk of desc s
     const CopyDesc& d = t.d[s];
     const uint32_t tail = (uint32_t)(d.len & 15u);
@@ -196,7 +254,7 @@ mp_swap_bulk(const __grid_constant__ CopyTable<CAP> t) {
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
 
   auto issue_load = [&](uint32_t i) {
-    const Piece p = bulk_piece<SHIFT>(t, first + i * gridDim.x);
+    const Piece p = bulk_piece<SHIFT>(t, my.chunk(i));
     uint64_t* bar = &bars[i % STAGES];
     mbar_expect_tx(bar, p.bytes);
     if (p.bytes) bulk_load(smem + (size_t)(i % STAGES) * kSlot, p.src, p.bytes, bar);
@@ -206,7 +264,7 @@ mp_swap_bulk(const __grid_constant__ CopyTable<CAP> t) {
   for (uint32_t i = 0; i < prologue; ++i) issue_load(i);
   for (uint32_t i = 0; i < mine; ++i) {
     mbar_wait(&bars[i % STAGES], (i / STAGES) & 1u);
-    const Piece p = bulk_piece<SHIFT>(t, first + i * gridDim.x);
+    const Piece p = bulk_piece<SHIFT>(t, my.chunk(i));
     if (p.bytes) bulk_store(p.dst, smem + (size_t)(i % STAGES) * kSlot, p.bytes);
     bulk_commit();
     // Refill the slot of piece i-1 once its store has finished reading smem
@@ -263,7 +321,7 @@ const Shape& shape_of(int path, int variant) {
   return path == MPRESS_PATH_BULK ? kBulk[variant] : kDirect[variant];
 }
 
-// Per-device cache of "CTAs resident in one wave" and of the smem opt-in.
+// Per-device cache of the default grid.
 struct DevCache {
   std::mutex mu;
   int wave[2][8][64] = {};
@@ -286,36 +344,49 @@ int prepare(KernelFn<CAP> k, const Shape& sh) {
   return MPRESS_OK;
 }
 
+// Build the table for descriptors d[0..n) (group ids gid[]), split `cap`
+// CTAs between the groups in proportion to their chunks, launch.
 template <int CAP>
-int launch_table(int path, int variant, int dir, const CopyTable<CAP>& t, unsigned grid,
-                 cudaStream_t stream) {
-  const Shape& sh = shape_of(path, variant);
-  KernelFn<CAP> k = kernel_for<CAP>(path, variant, dir);
-  MP_TRY(prepare<CAP>(k, sh));
-  k<<<grid, sh.threads, sh.smem, stream>>>(t);
-  cudaError_t e = cudaGetLastError();
-  if (e != cudaSuccess) return fail(MPRESS_ERR_CUDA, "swap kernel launch: %s", cudaGetErrorString(e));
-  return MPRESS_OK;
-}
-
-template <int CAP>
-int launch_batch(int path, int variant, int dir, const CopyDesc* d, uint32_t n, uint32_t shift,
-                 int cap, cudaStream_t stream, bool* launched) {
+int launch_batch(int path, int variant, int dir, const CopyDesc* d, const int* gid, uint32_t n,
+                 uint32_t shift, int cap, cudaStream_t stream, bool* launched) {
   CopyTable<CAP> t;
   t.n = n;
+  t.pad = 0;
   uint64_t chunks = 0;
+  uint32_t ng = 0;
   for (uint32_t i = 0; i < n; ++i) {
+    if (i == 0 || gid[i] != gid[i - 1]) {
+      if (ng == (uint32_t)kMaxGroups) return fail(MPRESS_ERR_ARG, "more than %d peers in one swap", kMaxGroups);
+      t.g_chunk[ng++] = (uint32_t)chunks;
+    }
     t.d[i] = d[i];
     t.first_chunk[i] = (uint32_t)chunks;
     chunks += (d[i].len + (1ull << shift) - 1) >> shift;
     if (chunks > 0xFFFFFFFFull) return fail(MPRESS_ERR_ARG, "swap batch exceeds 2^32 chunks");
   }
   t.first_chunk[n] = (uint32_t)chunks;
-  t.total_chunks = (uint32_t)chunks;
+  t.g_chunk[ng] = (uint32_t)chunks;
+  t.n_groups = ng;
   *launched = false;
   if (chunks == 0) return MPRESS_OK;
-  const unsigned grid = (unsigned)std::min<uint64_t>(chunks, (uint64_t)cap);
-  MP_TRY(launch_table<CAP>(path, variant, dir, t, grid, stream));
+  // workers per group ~ cap * share of chunks, at least 1, at most its chunks
+  uint32_t workers = 0;
+  for (uint32_t g = 0; g < ng; ++g) {
+    const uint64_t gc = t.g_chunk[g + 1] - t.g_chunk[g];
+    uint64_t w = (gc * (uint64_t)cap + chunks / 2) / chunks;
+    w = std::max<uint64_t>(1, std::min<uint64_t>(w, gc));
+    t.g_worker[g] = workers;
+    workers += (uint32_t)w;
+  }
+  t.g_worker[ng] = workers;
+  t.n_workers = workers;
+  const unsigned grid = (unsigned)std::min<uint64_t>(workers, (uint64_t)cap);
+  const Shape& sh = shape_of(path, variant);
+  KernelFn<CAP> k = kernel_for<CAP>(path, variant, dir);
+  MP_TRY(prepare<CAP>(k, sh));
+  k<<<grid, sh.threads, sh.smem, stream>>>(t);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return fail(MPRESS_ERR_CUDA, "swap kernel launch: %s", cudaGetErrorString(e));
   *launched = true;
   return MPRESS_OK;
 }
@@ -341,8 +412,8 @@ int copy_wave_ctas(int path, int variant) {
   return w;
 }
 
-int launch_copy(int path, int variant, int dir, const CopyDesc* d, size_t n, int max_ctas,
-                cudaStream_t stream, int* launches) {
+int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* group, size_t n,
+                int max_ctas, cudaStream_t stream, int* launches) {
   const int nvar = path == MPRESS_PATH_BULK ? kBulkVariants : kDirectVariants;
   if (variant < 0 || variant >= nvar) return fail(MPRESS_ERR_ARG, "kernel variant %d out of range", variant);
   const int wave = copy_wave_ctas(path, variant);
@@ -352,9 +423,13 @@ int launch_copy(int path, int variant, int dir, const CopyDesc* d, size_t n, int
   for (size_t base = 0; base < n; base += kMaxDescPerLaunch) {
     const uint32_t m = (uint32_t)std::min<size_t>(kMaxDescPerLaunch, n - base);
     bool launched = false;
-    if (m <= 16) MP_TRY(launch_batch<16>(path, variant, dir, d + base, m, shift, cap, stream, &launched));
-    else if (m <= 128) MP_TRY(launch_batch<128>(path, variant, dir, d + base, m, shift, cap, stream, &launched));
-    else MP_TRY(launch_batch<kMaxDescPerLaunch>(path, variant, dir, d + base, m, shift, cap, stream, &launched));
+    if (m <= 16)
+      MP_TRY(launch_batch<16>(path, variant, dir, d + base, group + base, m, shift, cap, stream, &launched));
+    else if (m <= 128)
+      MP_TRY(launch_batch<128>(path, variant, dir, d + base, group + base, m, shift, cap, stream, &launched));
+    else
+      MP_TRY(launch_batch<kMaxDescPerLaunch>(path, variant, dir, d + base, group + base, m, shift, cap, stream,
+                                             &launched));
     if (launched && launches) ++*launches;
   }
   return MPRESS_OK;

@@ -27,7 +27,8 @@ enum CopyDir { kDirOut = 0, kDirIn = 1 };
 // MPRESS_PATH_DIRECT or MPRESS_PATH_BULK, `variant` its kernel shape;
 // `max_ctas` caps the grid (0 = the variant's default grid).  Adds the number
 // of kernel launches to *launches.  Returns MPRESS_OK or MPRESS_ERR_*.
-int launch_copy(int path, int variant, int dir, const CopyDesc* d, size_t n, int max_ctas,
+int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* group, size_t n,
+                int max_ctas,
                 cudaStream_t stream, int* launches);
 
 // Default grid of a path/variant on the current device (SMs x CTAs per SM).
