@@ -213,10 +213,17 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
  * MPRESS_OPT_VARIANT: kernel shape within the path -- direct: 0 = 256
  * threads x 8 vectors (2 CTAs/SM by default), 1 = 512x8, 2 = 256x16,
  * 3 = 1024x4; bulk: 0 = 6 slots x 32 KiB, 1 = 12 x 16 KiB, 2 = 3 x 64 KiB.
+ * MPRESS_OPT_ORDER: chunk order inside one launch -- 0 = interleave the
+ * peers by a weighted round robin, so every peer link carries its share of
+ * the swap at every moment (default; needed when several sources share
+ * peers); 1 = plan order (peer by peer).
  * Invalid values -> MPRESS_ERR_ARG. */
 #define MPRESS_OPT_PATH      1
 #define MPRESS_OPT_MAX_CTAS  2
 #define MPRESS_OPT_VARIANT   3
+#define MPRESS_OPT_ORDER     4
+#define MPRESS_ORDER_INTERLEAVE 0
+#define MPRESS_ORDER_PLAN       1
 #define MPRESS_PATH_DIRECT   0
 #define MPRESS_PATH_BULK     1
 #define MPRESS_PATH_CE       2

@@ -86,6 +86,7 @@ struct mpress_ctx_s {
   int path = MPRESS_PATH_DIRECT;
   int max_ctas = 0;
   int variant = 0;
+  int order = MPRESS_ORDER_INTERLEAVE;
   int last_launches = 0;
   std::vector<cudaStream_t> ce_streams;  // copy-engine comparator, one per peer
   std::vector<cudaEvent_t> ev_pool;

@@ -334,6 +334,11 @@ extern "C" int mpress_set_option(mpress_ctx_t* c, int key, int64_t value) {
       if (value < 0 || value > (1 << 20)) return fail(MPRESS_ERR_ARG, "bad max_ctas %lld", (long long)value);
       c->max_ctas = (int)value;
       return MPRESS_OK;
+    case MPRESS_OPT_ORDER:
+      if (value != MPRESS_ORDER_INTERLEAVE && value != MPRESS_ORDER_PLAN)
+        return fail(MPRESS_ERR_ARG, "unknown chunk order %lld", (long long)value);
+      c->order = (int)value;
+      return MPRESS_OK;
     case MPRESS_OPT_VARIANT: {
       const int nvar = c->path == MPRESS_PATH_BULK ? kBulkVariants : kDirectVariants;
       if (value < 0 || value >= nvar)
@@ -351,6 +356,7 @@ extern "C" int mpress_get_option(const mpress_ctx_t* c, int key, int64_t* value)
     case MPRESS_OPT_PATH: *value = c->path; return MPRESS_OK;
     case MPRESS_OPT_MAX_CTAS: *value = c->max_ctas; return MPRESS_OK;
     case MPRESS_OPT_VARIANT: *value = c->variant; return MPRESS_OK;
+    case MPRESS_OPT_ORDER: *value = c->order; return MPRESS_OK;
   }
   return fail(MPRESS_ERR_ARG, "unknown option %d", key);
 }

@@ -96,7 +96,8 @@ int run_copy(mpress_ctx_s* c, int dir, const std::vector<CopyDesc>& d,
              const std::vector<int>& desc_peer, cudaStream_t stream) {
   c->last_launches = 0;
   if (c->path != MPRESS_PATH_CE)
-    return launch_copy(c->path, c->variant, dir, d.data(), desc_peer.data(), d.size(), c->max_ctas, stream,
+    return launch_copy(c->path, c->variant, dir, d.data(),
+                       c->order == MPRESS_ORDER_INTERLEAVE ? desc_peer.data() : nullptr, d.size(), c->max_ctas, stream,
                        &c->last_launches);
 
   // Copy-engine comparator: cudaMemcpyAsync per stripe, one side stream per

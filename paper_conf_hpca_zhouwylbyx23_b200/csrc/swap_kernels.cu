@@ -6,16 +6,18 @@
 //   * one launch per plan (the whole batch, "we also batch tensors"),
 //     descriptors passed as a __grid_constant__ parameter (no upload);
 //   * the descriptors are grouped by peer (the plan's stripes are sorted by
-//     peer) and the CTAs are split between the groups in proportion to the
-//     group's bytes, so every peer link carries its share concurrently for the
-//     whole swap -- the paper's "transmit them in parallel through disjoint
-//     links" with sub-blocks sized to the links, done at CTA
-//     granularity.  With several sources swapping at once (config 5, or every
-//     rank in the N-GPU bench) each peer's NVLink ingress is then shared by
-//     all sources all the time instead of every source converging on its
-//     first peer;
-//   * inside a group, fixed-size chunks are walked with a stride, so adjacent
-//     chunks are in flight on different SMs at once;
+//     peer) and the chunks of the groups are interleaved by a weighted round
+//     robin (round r takes chunk floor(r*n_g/R) of group g, R = the largest
+//     group's chunk count rounded up to a power of two, so the division is a
+//     shift), so at every moment each peer link carries its proportional
+//     share of the swap -- the paper's "transmit them in parallel through
+//     disjoint links" with sub-blocks sized to the links.
+//     With several sources swapping at once (config 5, or every rank of the
+//     N-GPU bench) each peer's NVLink ingress is then shared by all sources
+//     all the time instead of every source converging on its first peer;
+//   * the CTAs walk that interleaved sequence with a grid stride, so any grid
+//     size is load-balanced and adjacent chunks are in flight on different
+//     SMs at once;
 //   * the grid is capped (MPRESS_OPT_MAX_CTAS) so a concurrent GEMM keeps
 //     most SMs;
 //   * every address is 16-B aligned (tensor pointers are checked; stripe
@@ -37,6 +39,7 @@
 #include <mutex>
 #include <set>
 #include <utility>
+#include <vector>
 
 #include "common.h"
 #include "swap_kernels.h"
@@ -52,10 +55,10 @@ template <int CAP>
 struct CopyTable {
   uint32_t n;                        // descriptors
   uint32_t n_groups;                 // runs of descriptors with the same peer
-  uint32_t n_workers;                // virtual workers over all groups
+  uint32_t rounds_log2;              // R = 2^rounds_log2 >= chunks of the largest group
   uint32_t pad;
   uint32_t g_chunk[kMaxGroups + 1];  // first chunk of each group (prefix)
-  uint32_t g_worker[kMaxGroups + 1]; // first virtual worker of each group (prefix)
+  uint32_t g_desc[kMaxGroups + 1];   // first descriptor of each group (prefix)
   uint32_t first_chunk[CAP + 1];     // first chunk of each descriptor (prefix)
   CopyDesc d[CAP];
 };
@@ -71,22 +74,44 @@ __device__ __forceinline__ uint32_t upper_idx(const uint32_t* a, uint32_t n, uin
   return lo;
 }
 
-// Virtual worker v of the table: its group, its rank in the group, the
-// group's worker count and chunk range.
-struct Worker {
-  uint32_t chunk0, nchunks, rank, count;
-};
-
+// The interleaved sequence has R rounds of n_groups positions; position
+// (r, g) holds chunk k = floor(r * n_g / R) of group g.  k is non-decreasing
+// in r with steps of 0 or 1 and reaches n_g - 1 by r = R - 1, so taking only
+// the first round that reaches each k visits every chunk exactly once; the
+// other positions are skipped.  A CTA walks positions blockIdx.x,
+// + gridDim.x, ... with (r, g) advanced incrementally (no division per step).
 template <int CAP>
-__device__ __forceinline__ Worker worker_of(const CopyTable<CAP>& t, uint32_t v) {
-  const uint32_t g = upper_idx(t.g_worker, t.n_groups, v);
-  Worker w;
-  w.chunk0 = t.g_chunk[g];
-  w.nchunks = t.g_chunk[g + 1] - t.g_chunk[g];
-  w.rank = v - t.g_worker[g];
-  w.count = t.g_worker[g + 1] - t.g_worker[g];
-  return w;
-}
+struct Cursor {
+  const CopyTable<CAP>& t;
+  uint32_t g, gm, gd;
+  uint64_t r;
+  __device__ explicit Cursor(const CopyTable<CAP>& tt) : t(tt) {
+    g = blockIdx.x % t.n_groups;
+    r = blockIdx.x / t.n_groups;
+    gm = gridDim.x % t.n_groups;
+    gd = gridDim.x / t.n_groups;
+  }
+  // Next chunk of this CTA: its index *c and its descriptor *s.
+  __device__ bool next(uint32_t* c, uint32_t* s) {
+    const uint64_t R = 1ull << t.rounds_log2;
+    while (r < R) {
+      const uint32_t gg = g;
+      const uint64_t rr = r;
+      g += gm;
+      r += gd;
+      if (g >= t.n_groups) { g -= t.n_groups; ++r; }
+      const uint64_t gc = t.g_chunk[gg + 1] - t.g_chunk[gg];
+      const uint64_t k = (rr * gc) >> t.rounds_log2;
+      if (rr > 0 && (((rr - 1) * gc) >> t.rounds_log2) == k) continue;
+      *c = t.g_chunk[gg] + (uint32_t)k;
+      // descriptor: search only inside the group's descriptors
+      const uint32_t d0 = t.g_desc[gg];
+      *s = d0 + upper_idx(t.first_chunk + d0, t.g_desc[gg + 1] - d0, *c);
+      return true;
+    }
+    return false;
+  }
+};
 
 __device__ __forceinline__ int4 ld_stream(const int4* p) {
   int4 r;
@@ -109,34 +134,31 @@ mp_swap_direct(const __grid_constant__ CopyTable<CAP> t) {
   constexpr uint32_t kChunk = THREADS * UNROLL * 16;
   static_assert((kChunk & (kChunk - 1)) == 0, "chunk must be a power of two");
   constexpr uint32_t kShift = __builtin_ctz(kChunk);
-  for (uint32_t v = blockIdx.x; v < t.n_workers; v += gridDim.x) {
-    const Worker w = worker_of(t, v);
-    for (uint32_t k = w.rank; k < w.nchunks; k += w.count) {
-      const uint32_t c = w.chunk0 + k;
-      const uint32_t s = upper_idx(t.first_chunk, t.n, c);
-      const CopyDesc& d = t.d[s];
-      const uint64_t off = (uint64_t)(c - t.first_chunk[s]) << kShift;
-      const uint8_t* src = static_cast<const uint8_t*>(d.src) + off;
-      uint8_t* dst = static_cast<uint8_t*>(d.dst) + off;
-      const uint64_t rem = d.len - off;
-      if (rem >= kChunk) {
-        const int4* sv = reinterpret_cast<const int4*>(src) + threadIdx.x;
-        int4* dv = reinterpret_cast<int4*>(dst) + threadIdx.x;
-        int4 r[UNROLL];
+  Cursor<CAP> cur(t);
+  uint32_t c, s;
+  while (cur.next(&c, &s)) {
+    const CopyDesc& d = t.d[s];
+    const uint64_t off = (uint64_t)(c - t.first_chunk[s]) << kShift;
+    const uint8_t* src = static_cast<const uint8_t*>(d.src) + off;
+    uint8_t* dst = static_cast<uint8_t*>(d.dst) + off;
+    const uint64_t rem = d.len - off;
+    if (rem >= kChunk) {
+      const int4* sv = reinterpret_cast<const int4*>(src) + threadIdx.x;
+      int4* dv = reinterpret_cast<int4*>(dst) + threadIdx.x;
+      int4 r[UNROLL];
 #pragma unroll
-        for (int j = 0; j < UNROLL; ++j) r[j] = ld_stream(sv + j * THREADS);
+      for (int j = 0; j < UNROLL; ++j) r[j] = ld_stream(sv + j * THREADS);
 #pragma unroll
-        for (int j = 0; j < UNROLL; ++j) st_stream(dv + j * THREADS, r[j]);
-      } else {
-        // ragged last chunk of a stripe: 16-B body, then the <16-byte tail
-        const uint32_t len = (uint32_t)rem;
-        const uint32_t n16 = len >> 4;
-        const int4* sv = reinterpret_cast<const int4*>(src);
-        int4* dv = reinterpret_cast<int4*>(dst);
-        for (uint32_t x = threadIdx.x; x < n16; x += THREADS) st_stream(dv + x, ld_stream(sv + x));
-        const uint32_t tail = len & 15u;
-        if (threadIdx.x < tail) dst[(n16 << 4) + threadIdx.x] = src[(n16 << 4) + threadIdx.x];
-      }
+      for (int j = 0; j < UNROLL; ++j) st_stream(dv + j * THREADS, r[j]);
+    } else {
+      // ragged last chunk of a stripe: 16-B body, then the <16-byte tail
+      const uint32_t len = (uint32_t)rem;
+      const uint32_t n16 = len >> 4;
+      const int4* sv = reinterpret_cast<const int4*>(src);
+      int4* dv = reinterpret_cast<int4*>(dst);
+      for (uint32_t x = threadIdx.x; x < n16; x += THREADS) st_stream(dv + x, ld_stream(sv + x));
+      const uint32_t tail = len & 15u;
+      if (threadIdx.x < tail) dst[(n16 << 4) + threadIdx.x] = src[(n16 << 4) + threadIdx.x];
     }
   }
 }
@@ -188,8 +210,7 @@ struct Piece {
 };
 
 template <int SHIFT, int CAP>
-__device__ __forceinline__ Piece bulk_piece(const CopyTable<CAP>& t, uint32_t c) {
-  const uint32_t s = upper_idx(t.first_chunk, t.n, c);
+__device__ __forceinline__ Piece bulk_piece(const CopyTable<CAP>& t, uint32_t c, uint32_t s) {
   const CopyDesc& d = t.d[s];
   const uint64_t off = (uint64_t)(c - t.first_chunk[s]) << SHIFT;
   const uint64_t rem = d.len - off;
@@ -199,29 +220,6 @@ __device__ __forceinline__ Piece bulk_piece(const CopyTable<CAP>& t, uint32_t c)
   p.bytes = (uint32_t)(rem >= (1ull << SHIFT) ? (1ull << SHIFT) : (rem & ~15ull));
   return p;
 }
-
-// The chunks of this CTA, in order: for each of its virtual workers
-// (blockIdx.x, + gridDim.x, ...), that worker's chunks rank, rank+count, ...
-template <int CAP>
-struct MyChunks {
-  const CopyTable<CAP>& t;
-  uint32_t total = 0;
-  __device__ explicit MyChunks(const CopyTable<CAP>& tt) : t(tt) {
-    for (uint32_t v = blockIdx.x; v < t.n_workers; v += gridDim.x) total += count_of(worker_of(t, v));
-  }
-  __device__ static uint32_t count_of(const Worker& w) {
-    return w.rank < w.nchunks ? (w.nchunks - w.rank + w.count - 1) / w.count : 0;
-  }
-  __device__ uint32_t chunk(uint32_t i) const {
-    for (uint32_t v = blockIdx.x; v < t.n_workers; v += gridDim.x) {
-      const Worker w = worker_of(t, v);
-      const uint32_t n = count_of(w);
-      if (i < n) return w.chunk0 + w.rank + i * w.count;
-      i -= n;
-    }
-    return 0;  // unreachable for i < total
-  }
-};
 
 // One warp per CTA: lane 0 streams pieces of 2^SHIFT bytes through STAGES
 // shared-memory slots with the SM's bulk-copy engine (cp.async.bulk G->S with
@@ -234,47 +232,51 @@ mp_swap_bulk(const __grid_constant__ CopyTable<CAP> t) {
   extern __shared__ __align__(128) uint8_t smem[];
   __shared__ __align__(8) uint64_t bars[STAGES];
 
-  const MyChunks<CAP> my(t);
-  const uint32_t mine = my.total;
-
-  for (uint32_t i = 0; i < mine; ++i) {
-    const uint32_t c = my.chunk(i);
-    const uint32_t s = upper_idx(t.first_chunk, t.n, c);
-    if (c + 1 != t.first_chunk[s + 1]) continue;  // not the last chunk of desc s
-    const CopyDesc& d = t.d[s];
-    const uint32_t tail = (uint32_t)(d.len & 15u);
-    if (threadIdx.x < tail) {
-      const uint64_t b = (d.len & ~15ull) + threadIdx.x;
-      static_cast<uint8_t*>(d.dst)[b] = static_cast<const uint8_t*>(d.src)[b];
+  {  // tails, by the whole warp
+    Cursor<CAP> cur(t);
+    uint32_t c, s;
+    while (cur.next(&c, &s)) {
+      if (c + 1 != t.first_chunk[s + 1]) continue;  // not the last chunk of desc s
+      const CopyDesc& d = t.d[s];
+      const uint32_t tail = (uint32_t)(d.len & 15u);
+      if (threadIdx.x < tail) {
+        const uint64_t b = (d.len & ~15ull) + threadIdx.x;
+        static_cast<uint8_t*>(d.dst)[b] = static_cast<const uint8_t*>(d.src)[b];
+      }
     }
   }
-  if (threadIdx.x != 0 || mine == 0) return;
+  if (threadIdx.x != 0) return;
 
   for (int k = 0; k < STAGES; ++k) mbar_init(&bars[k], 1);
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
 
-  auto issue_load = [&](uint32_t i) {
-    const Piece p = bulk_piece<SHIFT>(t, my.chunk(i));
-    uint64_t* bar = &bars[i % STAGES];
+  // Two cursors over the same chunk sequence: loads run STAGES ahead of stores.
+  Cursor<CAP> ld(t), st(t);
+  uint32_t issued = 0;
+  auto issue_load = [&]() -> bool {
+    uint32_t c, s;
+    if (!ld.next(&c, &s)) return false;
+    const Piece p = bulk_piece<SHIFT>(t, c, s);
+    uint64_t* bar = &bars[issued % STAGES];
     mbar_expect_tx(bar, p.bytes);
-    if (p.bytes) bulk_load(smem + (size_t)(i % STAGES) * kSlot, p.src, p.bytes, bar);
+    if (p.bytes) bulk_load(smem + (size_t)(issued % STAGES) * kSlot, p.src, p.bytes, bar);
+    ++issued;
+    return true;
   };
 
-  const uint32_t prologue = mine < (uint32_t)STAGES ? mine : (uint32_t)STAGES;
-  for (uint32_t i = 0; i < prologue; ++i) issue_load(i);
-  for (uint32_t i = 0; i < mine; ++i) {
+  for (int k = 0; k < STAGES; ++k)
+    if (!issue_load()) break;
+  uint32_t c, s;
+  for (uint32_t i = 0; st.next(&c, &s); ++i) {
     mbar_wait(&bars[i % STAGES], (i / STAGES) & 1u);
-    const Piece p = bulk_piece<SHIFT>(t, my.chunk(i));
+    const Piece p = bulk_piece<SHIFT>(t, c, s);
     if (p.bytes) bulk_store(p.dst, smem + (size_t)(i % STAGES) * kSlot, p.bytes);
     bulk_commit();
     // Refill the slot of piece i-1 once its store has finished reading smem
     // (only the newest group, piece i's store, may still be reading).
-    if (i >= 1) {
-      const uint32_t nxt = i - 1 + STAGES;
-      if (nxt < mine) {
-        bulk_wait_read1();
-        issue_load(nxt);
-      }
+    if (i >= 1 && issued == i - 1 + STAGES) {
+      bulk_wait_read1();
+      issue_load();
     }
   }
   bulk_wait_all();
@@ -355,8 +357,9 @@ int launch_batch(int path, int variant, int dir, const CopyDesc* d, const int* g
   uint64_t chunks = 0;
   uint32_t ng = 0;
   for (uint32_t i = 0; i < n; ++i) {
-    if (i == 0 || gid[i] != gid[i - 1]) {
+    if (i == 0 || (gid && gid[i] != gid[i - 1])) {
       if (ng == (uint32_t)kMaxGroups) return fail(MPRESS_ERR_ARG, "more than %d peers in one swap", kMaxGroups);
+      t.g_desc[ng] = i;
       t.g_chunk[ng++] = (uint32_t)chunks;
     }
     t.d[i] = d[i];
@@ -366,21 +369,15 @@ int launch_batch(int path, int variant, int dir, const CopyDesc* d, const int* g
   }
   t.first_chunk[n] = (uint32_t)chunks;
   t.g_chunk[ng] = (uint32_t)chunks;
+  t.g_desc[ng] = n;
   t.n_groups = ng;
   *launched = false;
   if (chunks == 0) return MPRESS_OK;
-  // workers per group ~ cap * share of chunks, at least 1, at most its chunks
-  uint32_t workers = 0;
-  for (uint32_t g = 0; g < ng; ++g) {
-    const uint64_t gc = t.g_chunk[g + 1] - t.g_chunk[g];
-    uint64_t w = (gc * (uint64_t)cap + chunks / 2) / chunks;
-    w = std::max<uint64_t>(1, std::min<uint64_t>(w, gc));
-    t.g_worker[g] = workers;
-    workers += (uint32_t)w;
-  }
-  t.g_worker[ng] = workers;
-  t.n_workers = workers;
-  const unsigned grid = (unsigned)std::min<uint64_t>(workers, (uint64_t)cap);
+  uint32_t largest = 0;
+  for (uint32_t g = 0; g < ng; ++g) largest = std::max(largest, t.g_chunk[g + 1] - t.g_chunk[g]);
+  t.rounds_log2 = 0;
+  while ((1ull << t.rounds_log2) < largest) ++t.rounds_log2;
+  const unsigned grid = (unsigned)std::min<uint64_t>(chunks, (uint64_t)cap);
   const Shape& sh = shape_of(path, variant);
   KernelFn<CAP> k = kernel_for<CAP>(path, variant, dir);
   MP_TRY(prepare<CAP>(k, sh));
@@ -424,11 +421,11 @@ int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* gr
     const uint32_t m = (uint32_t)std::min<size_t>(kMaxDescPerLaunch, n - base);
     bool launched = false;
     if (m <= 16)
-      MP_TRY(launch_batch<16>(path, variant, dir, d + base, group + base, m, shift, cap, stream, &launched));
+      MP_TRY(launch_batch<16>(path, variant, dir, d + base, group ? group + base : nullptr, m, shift, cap, stream, &launched));
     else if (m <= 128)
-      MP_TRY(launch_batch<128>(path, variant, dir, d + base, group + base, m, shift, cap, stream, &launched));
+      MP_TRY(launch_batch<128>(path, variant, dir, d + base, group ? group + base : nullptr, m, shift, cap, stream, &launched));
     else
-      MP_TRY(launch_batch<kMaxDescPerLaunch>(path, variant, dir, d + base, group + base, m, shift, cap, stream,
+      MP_TRY(launch_batch<kMaxDescPerLaunch>(path, variant, dir, d + base, group ? group + base : nullptr, m, shift, cap, stream,
                                              &launched));
     if (launched && launches) ++*launches;
   }

@@ -73,10 +73,13 @@ def paths():
                 if name != "ce":
                     ctx.set_option(mp.OPT_VARIANT, var)
                 ctx.set_option(mp.OPT_MAX_CTAS, cap)
-                to, ti = time_swaps(ctx, pl, src, dst, 10, s)
-                print(json.dumps({"sweep": "paths", "path": name, "variant": var, "max_ctas": cap,
-                                  "out_gbs": nbytes / to / 1e6, "in_gbs": nbytes / ti / 1e6,
-                                  "hbm_gbs_out": 2 * nbytes / to / 1e6}), flush=True)
+                for order in (mp.ORDER_INTERLEAVE, mp.ORDER_PLAN):
+                    ctx.set_option(mp.OPT_ORDER, order)
+                    to, ti = time_swaps(ctx, pl, src, dst, 10, s)
+                    print(json.dumps({"sweep": "paths", "path": name, "variant": var, "max_ctas": cap,
+                                      "order": order, "out_gbs": nbytes / to / 1e6,
+                                      "in_gbs": nbytes / ti / 1e6,
+                                      "hbm_gbs_out": 2 * nbytes / to / 1e6}), flush=True)
     ctx.finalize()
 
 
