@@ -126,6 +126,19 @@ __device__ __forceinline__ void st_stream(int4* p, const int4& v) {
 }
 
 // ---------------------------------------------------------------- direct path
+
+struct Span {
+  const uint8_t* src;
+  uint8_t* dst;
+  uint64_t rem;  // bytes of the descriptor from this chunk on
+};
+
+template <uint32_t SHIFT, int CAP>
+__device__ __forceinline__ Span span_of(const CopyTable<CAP>& t, uint32_t c, uint32_t s) {
+  const CopyDesc& d = t.d[s];
+  const uint64_t off = (uint64_t)(c - t.first_chunk[s]) << SHIFT;
+  return Span{static_cast<const uint8_t*>(d.src) + off, static_cast<uint8_t*>(d.dst) + off, d.len - off};
+}
 // THREADS threads each keep UNROLL independent 16-B loads in flight, then
 // store them: one chunk = THREADS*UNROLL*16 bytes per CTA iteration.
 template <int DIR, int THREADS, int UNROLL, int CAP>
@@ -134,32 +147,40 @@ mp_swap_direct(const __grid_constant__ CopyTable<CAP> t) {
   constexpr uint32_t kChunk = THREADS * UNROLL * 16;
   static_assert((kChunk & (kChunk - 1)) == 0, "chunk must be a power of two");
   constexpr uint32_t kShift = __builtin_ctz(kChunk);
+  // The next chunk's address is resolved while the current chunk's loads are
+  // in flight, so the table lookups (constant-bank reads) stay off the
+  // critical path of a latency-bound CTA.
   Cursor<CAP> cur(t);
   uint32_t c, s;
-  while (cur.next(&c, &s)) {
-    const CopyDesc& d = t.d[s];
-    const uint64_t off = (uint64_t)(c - t.first_chunk[s]) << kShift;
-    const uint8_t* src = static_cast<const uint8_t*>(d.src) + off;
-    uint8_t* dst = static_cast<uint8_t*>(d.dst) + off;
-    const uint64_t rem = d.len - off;
-    if (rem >= kChunk) {
-      const int4* sv = reinterpret_cast<const int4*>(src) + threadIdx.x;
-      int4* dv = reinterpret_cast<int4*>(dst) + threadIdx.x;
+  if (!cur.next(&c, &s)) return;
+  Span sp = span_of<kShift>(t, c, s);
+  for (;;) {
+    Span nx;
+    bool more;
+    if (sp.rem >= kChunk) {
+      const int4* sv = reinterpret_cast<const int4*>(sp.src) + threadIdx.x;
+      int4* dv = reinterpret_cast<int4*>(sp.dst) + threadIdx.x;
       int4 r[UNROLL];
 #pragma unroll
       for (int j = 0; j < UNROLL; ++j) r[j] = ld_stream(sv + j * THREADS);
+      more = cur.next(&c, &s);
+      if (more) nx = span_of<kShift>(t, c, s);
 #pragma unroll
       for (int j = 0; j < UNROLL; ++j) st_stream(dv + j * THREADS, r[j]);
     } else {
       // ragged last chunk of a stripe: 16-B body, then the <16-byte tail
-      const uint32_t len = (uint32_t)rem;
+      const uint32_t len = (uint32_t)sp.rem;
       const uint32_t n16 = len >> 4;
-      const int4* sv = reinterpret_cast<const int4*>(src);
-      int4* dv = reinterpret_cast<int4*>(dst);
+      const int4* sv = reinterpret_cast<const int4*>(sp.src);
+      int4* dv = reinterpret_cast<int4*>(sp.dst);
       for (uint32_t x = threadIdx.x; x < n16; x += THREADS) st_stream(dv + x, ld_stream(sv + x));
       const uint32_t tail = len & 15u;
-      if (threadIdx.x < tail) dst[(n16 << 4) + threadIdx.x] = src[(n16 << 4) + threadIdx.x];
+      if (threadIdx.x < tail) sp.dst[(n16 << 4) + threadIdx.x] = sp.src[(n16 << 4) + threadIdx.x];
+      more = cur.next(&c, &s);
+      if (more) nx = span_of<kShift>(t, c, s);
     }
+    if (!more) break;
+    sp = nx;
   }
 }
 
