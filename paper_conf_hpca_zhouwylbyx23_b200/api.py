@@ -12,7 +12,8 @@ from ctypes import (CFUNCTYPE, POINTER, byref, c_char_p, c_int, c_int32, c_int64
                     c_size_t, c_uint32, c_uint64, c_void_p)
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libmpress.so")
+# MPRESS_LIB overrides the library path (A/B runs of two builds, tools/ab.py)
+LIB_PATH = os.environ.get("MPRESS_LIB") or os.path.join(_HERE, "libmpress.so")
 
 OK = 0
 ERR_ARG, ERR_NO_SPACE, ERR_ALIGN, ERR_STATE, ERR_PEER, ERR_CUDA, ERR_SYS = -1, -2, -3, -4, -5, -6, -7
