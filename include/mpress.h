@@ -206,13 +206,15 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
  * (default); 1 = SM kernel, bulk-async copies (the SM's TMA engine,
  * cp.async.bulk) staged through shared memory; 2 = copy engines
  * (cudaMemcpyAsync per stripe on per-peer streams, the measured comparator).
- * Setting the path resets the variant to 0.
+ * Setting the path resets the variant to MPRESS_VARIANT_AUTO.
  * MPRESS_OPT_MAX_CTAS: cap on the kernel grid (0 = the variant's default
  * grid, a multiple of the SM count); CTAs spread one per SM first, so this is
  * the SM-count cap that protects a concurrent GEMM.
  * MPRESS_OPT_VARIANT: kernel shape within the path -- direct: 0 = 256
  * threads x 8 vectors (2 CTAs/SM by default), 1 = 512x8, 2 = 256x16,
- * 3 = 1024x4; bulk: 0 = 6 slots x 32 KiB, 1 = 12 x 16 KiB, 2 = 3 x 64 KiB.
+ * 3 = 1024x4; bulk: 0 = 6 slots x 32 KiB, 1 = 12 x 16 KiB, 2 = 3 x 64 KiB;
+ * MPRESS_VARIANT_AUTO (-1, default) = direct 1 when the grid is capped at
+ * <= one CTA per SM, else 0.
  * MPRESS_OPT_ORDER: chunk order inside one launch -- 0 = interleave the
  * peers by a weighted round robin, so every peer link carries its share of
  * the swap at every moment (default; needed when several sources share
@@ -222,6 +224,7 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
 #define MPRESS_OPT_MAX_CTAS  2
 #define MPRESS_OPT_VARIANT   3
 #define MPRESS_OPT_ORDER     4
+#define MPRESS_VARIANT_AUTO  (-1)
 #define MPRESS_ORDER_INTERLEAVE 0
 #define MPRESS_ORDER_PLAN       1
 #define MPRESS_PATH_DIRECT   0

@@ -4,7 +4,7 @@ The product is ``libmpress.so`` (C ABI in ``include/mpress.h``); this package is
 its thin Python binding (``api``).  See DESIGN.md.
 """
 from .api import (  # noqa: F401
-    ALIGN, DEFAULT_GRANULE, EXPORTED, LIB_PATH, OPT_MAX_CTAS, OPT_ORDER, OPT_PATH, OPT_VARIANT, ORDER_INTERLEAVE, ORDER_PLAN, PATH_BULK, PATH_CE,
+    ALIGN, DEFAULT_GRANULE, EXPORTED, LIB_PATH, OPT_MAX_CTAS, OPT_ORDER, OPT_PATH, OPT_VARIANT, ORDER_INTERLEAVE, ORDER_PLAN, VARIANT_AUTO, PATH_BULK, PATH_CE,
     PATH_DIRECT, STATE_IN, STATE_IN_PENDING, STATE_OUT, STATE_OUT_PENDING, Context, Handle,
     MPressError, Plan, lib, partition_sequential, plan, share_fds, torch_exchange,
 )

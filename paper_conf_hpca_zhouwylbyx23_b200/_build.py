@@ -13,15 +13,18 @@ import sys
 PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
-BUILD = os.path.join(ROOT, "build")
-LIB = os.path.join(PKG, "libmpress.so")
+# MPRESS_BUILD_TAG + MPRESS_NVCC_FLAGS: an experimental build (tools/ab.py)
+# into build/<tag>/ and build/ab/libmpress_<tag>.so; the product build is untagged.
+_TAG = os.environ.get("MPRESS_BUILD_TAG", "")
+BUILD = os.path.join(ROOT, "build", _TAG) if _TAG else os.path.join(ROOT, "build")
+LIB = os.path.join(ROOT, "build", "ab", "libmpress_%s.so" % _TAG) if _TAG else os.path.join(PKG, "libmpress.so")
 SYNTH_SRC = os.path.join(ROOT, "synth", "fill.cu")
 SYNTH_LIB = os.path.join(ROOT, "synth", "libsynth.so")
 
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 CFLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-fvisibility=hidden",
-          "-I" + os.path.join(ROOT, "include")]
+          "-I" + os.path.join(ROOT, "include")] + os.environ.get("MPRESS_NVCC_FLAGS", "").split()
 
 
 def _sources():
@@ -52,6 +55,7 @@ def _run(cmd, verbose):
 
 def build_mpress(verbose=False, force=False):
     os.makedirs(BUILD, exist_ok=True)
+    os.makedirs(os.path.dirname(LIB), exist_ok=True)
     hdrs = _headers()
     objs = []
     for src in _sources():

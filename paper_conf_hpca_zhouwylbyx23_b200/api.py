@@ -21,6 +21,7 @@ ALIGN = 256
 DEFAULT_GRANULE = 65536
 OPT_PATH, OPT_MAX_CTAS, OPT_VARIANT, OPT_ORDER = 1, 2, 3, 4
 ORDER_INTERLEAVE, ORDER_PLAN = 0, 1
+VARIANT_AUTO = -1
 PATH_DIRECT, PATH_BULK, PATH_CE = 0, 1, 2
 STATE_OUT_PENDING, STATE_OUT, STATE_IN_PENDING, STATE_IN = 1, 2, 3, 4
 

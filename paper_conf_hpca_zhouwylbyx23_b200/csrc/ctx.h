@@ -85,7 +85,7 @@ struct mpress_ctx_s {
   std::vector<mpress::Partition> parts;  // [world]
   int path = MPRESS_PATH_DIRECT;
   int max_ctas = 0;
-  int variant = 0;
+  int variant = MPRESS_VARIANT_AUTO;
   int order = MPRESS_ORDER_INTERLEAVE;
   int last_launches = 0;
   std::vector<cudaStream_t> ce_streams;  // copy-engine comparator, one per peer

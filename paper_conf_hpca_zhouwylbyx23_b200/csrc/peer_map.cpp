@@ -328,7 +328,7 @@ extern "C" int mpress_set_option(mpress_ctx_t* c, int key, int64_t value) {
       if (value != MPRESS_PATH_DIRECT && value != MPRESS_PATH_BULK && value != MPRESS_PATH_CE)
         return fail(MPRESS_ERR_ARG, "unknown path %lld", (long long)value);
       c->path = (int)value;
-      c->variant = 0;  // variants are per path
+      c->variant = MPRESS_VARIANT_AUTO;  // variants are per path
       return MPRESS_OK;
     case MPRESS_OPT_MAX_CTAS:
       if (value < 0 || value > (1 << 20)) return fail(MPRESS_ERR_ARG, "bad max_ctas %lld", (long long)value);
@@ -341,7 +341,7 @@ extern "C" int mpress_set_option(mpress_ctx_t* c, int key, int64_t value) {
       return MPRESS_OK;
     case MPRESS_OPT_VARIANT: {
       const int nvar = c->path == MPRESS_PATH_BULK ? kBulkVariants : kDirectVariants;
-      if (value < 0 || value >= nvar)
+      if (value != MPRESS_VARIANT_AUTO && (value < 0 || value >= nvar))
         return fail(MPRESS_ERR_ARG, "variant %lld out of range for path %d", (long long)value, c->path);
       c->variant = (int)value;
       return MPRESS_OK;

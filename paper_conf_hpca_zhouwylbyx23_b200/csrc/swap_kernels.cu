@@ -88,6 +88,7 @@ struct Cursor {
   __device__ explicit Cursor(const CopyTable<CAP>& tt) : t(tt) {
     g = blockIdx.x % t.n_groups;
     r = blockIdx.x / t.n_groups;
+
     gm = gridDim.x % t.n_groups;
     gd = gridDim.x / t.n_groups;
   }
@@ -141,15 +142,17 @@ __device__ __forceinline__ Span span_of(const CopyTable<CAP>& t, uint32_t c, uin
 }
 // THREADS threads each keep UNROLL independent 16-B loads in flight, then
 // store them: one chunk = THREADS*UNROLL*16 bytes per CTA iteration.
-template <int DIR, int THREADS, int UNROLL, int CAP>
+template <int DIR, int THREADS, int UNROLL, bool PF, int CAP>
 __global__ void __launch_bounds__(THREADS)
 mp_swap_direct(const __grid_constant__ CopyTable<CAP> t) {
   constexpr uint32_t kChunk = THREADS * UNROLL * 16;
   static_assert((kChunk & (kChunk - 1)) == 0, "chunk must be a power of two");
   constexpr uint32_t kShift = __builtin_ctz(kChunk);
-  // The next chunk's address is resolved while the current chunk's loads are
-  // in flight, so the table lookups (constant-bank reads) stay off the
-  // critical path of a latency-bound CTA.
+  // PF: the next chunk's address is resolved while the current chunk's loads
+  // are in flight, so the table lookups (constant-bank reads) stay off the
+  // critical path of a latency-bound CTA (<= 1 CTA per SM: +50% at 32 CTAs).
+  // With >= 2 CTAs per SM the memory system is saturated anyway and issuing
+  // the stores first measured ~6% faster (tools/ab.py), so PF is off there.
   Cursor<CAP> cur(t);
   uint32_t c, s;
   if (!cur.next(&c, &s)) return;
@@ -163,10 +166,16 @@ mp_swap_direct(const __grid_constant__ CopyTable<CAP> t) {
       int4 r[UNROLL];
 #pragma unroll
       for (int j = 0; j < UNROLL; ++j) r[j] = ld_stream(sv + j * THREADS);
-      more = cur.next(&c, &s);
-      if (more) nx = span_of<kShift>(t, c, s);
+      if (PF) {
+        more = cur.next(&c, &s);
+        if (more) nx = span_of<kShift>(t, c, s);
+      }
 #pragma unroll
       for (int j = 0; j < UNROLL; ++j) st_stream(dv + j * THREADS, r[j]);
+      if (!PF) {
+        more = cur.next(&c, &s);
+        if (more) nx = span_of<kShift>(t, c, s);
+      }
     } else {
       // ragged last chunk of a stripe: 16-B body, then the <16-byte tail
       const uint32_t len = (uint32_t)sp.rem;
@@ -323,7 +332,7 @@ template <int CAP>
 using KernelFn = void (*)(CopyTable<CAP>);
 
 template <int CAP>
-KernelFn<CAP> kernel_for(int path, int variant, int dir) {
+KernelFn<CAP> kernel_for(int path, int variant, int dir, bool pf) {
   const bool o = dir == kDirOut;
   if (path == MPRESS_PATH_BULK) {
     switch (variant) {
@@ -332,12 +341,16 @@ KernelFn<CAP> kernel_for(int path, int variant, int dir) {
       default: return o ? mp_swap_bulk<kDirOut, 15, 6, CAP> : mp_swap_bulk<kDirIn, 15, 6, CAP>;
     }
   }
+#define MP_DIRECT(T, U) \
+  (o ? (pf ? mp_swap_direct<kDirOut, T, U, true, CAP> : mp_swap_direct<kDirOut, T, U, false, CAP>) \
+     : (pf ? mp_swap_direct<kDirIn, T, U, true, CAP> : mp_swap_direct<kDirIn, T, U, false, CAP>))
   switch (variant) {
-    case 1: return o ? mp_swap_direct<kDirOut, 512, 8, CAP> : mp_swap_direct<kDirIn, 512, 8, CAP>;
-    case 2: return o ? mp_swap_direct<kDirOut, 256, 16, CAP> : mp_swap_direct<kDirIn, 256, 16, CAP>;
-    case 3: return o ? mp_swap_direct<kDirOut, 1024, 4, CAP> : mp_swap_direct<kDirIn, 1024, 4, CAP>;
-    default: return o ? mp_swap_direct<kDirOut, 256, 8, CAP> : mp_swap_direct<kDirIn, 256, 8, CAP>;
+    case 1: return MP_DIRECT(512, 8);
+    case 2: return MP_DIRECT(256, 16);
+    case 3: return MP_DIRECT(1024, 4);
+    default: return MP_DIRECT(256, 8);
   }
+#undef MP_DIRECT
 }
 
 const Shape& shape_of(int path, int variant) {
@@ -371,7 +384,7 @@ int prepare(KernelFn<CAP> k, const Shape& sh) {
 // CTAs between the groups in proportion to their chunks, launch.
 template <int CAP>
 int launch_batch(int path, int variant, int dir, const CopyDesc* d, const int* gid, uint32_t n,
-                 uint32_t shift, int cap, cudaStream_t stream, bool* launched) {
+                 uint32_t shift, int cap, int sms, cudaStream_t stream, bool* launched) {
   CopyTable<CAP> t;
   t.n = n;
   t.pad = 0;
@@ -400,7 +413,7 @@ int launch_batch(int path, int variant, int dir, const CopyDesc* d, const int* g
   while ((1ull << t.rounds_log2) < largest) ++t.rounds_log2;
   const unsigned grid = (unsigned)std::min<uint64_t>(chunks, (uint64_t)cap);
   const Shape& sh = shape_of(path, variant);
-  KernelFn<CAP> k = kernel_for<CAP>(path, variant, dir);
+  KernelFn<CAP> k = kernel_for<CAP>(path, variant, dir, (int)grid <= sms);
   MP_TRY(prepare<CAP>(k, sh));
   k<<<grid, sh.threads, sh.smem, stream>>>(t);
   cudaError_t e = cudaGetLastError();
@@ -419,7 +432,7 @@ int copy_wave_ctas(int path, int variant) {
   int& w = g_cache.wave[pi][variant][dev];
   if (w == 0) {
     const Shape& sh = shape_of(path, variant);
-    KernelFn<kMaxDescPerLaunch> k = kernel_for<kMaxDescPerLaunch>(path, variant, kDirOut);
+    KernelFn<kMaxDescPerLaunch> k = kernel_for<kMaxDescPerLaunch>(path, variant, kDirOut, false);
     if (prepare<kMaxDescPerLaunch>(k, sh) != MPRESS_OK) return 0;
     int sms = 0, per_sm = 0;
     if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) return 0;
@@ -432,6 +445,15 @@ int copy_wave_ctas(int path, int variant) {
 
 int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* group, size_t n,
                 int max_ctas, cudaStream_t stream, int* launches) {
+  int dev = 0, sms = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess)
+    return fail(MPRESS_ERR_CUDA, "cannot query the SM count");
+  if (variant == MPRESS_VARIANT_AUTO) {
+    // direct: a capped grid (<= one CTA per SM, e.g. beside a GEMM) moves the
+    // most bytes per SM with 512-thread CTAs; a full grid saturates HBM with
+    // 2 x 256-thread CTAs per SM (profiles/r01 sweeps).  bulk: 6 x 32 KiB.
+    variant = (path == MPRESS_PATH_DIRECT && max_ctas > 0 && max_ctas <= sms) ? 1 : 0;
+  }
   const int nvar = path == MPRESS_PATH_BULK ? kBulkVariants : kDirectVariants;
   if (variant < 0 || variant >= nvar) return fail(MPRESS_ERR_ARG, "kernel variant %d out of range", variant);
   const int wave = copy_wave_ctas(path, variant);
@@ -440,14 +462,14 @@ int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* gr
   const uint32_t shift = shape_of(path, variant).shift;
   for (size_t base = 0; base < n; base += kMaxDescPerLaunch) {
     const uint32_t m = (uint32_t)std::min<size_t>(kMaxDescPerLaunch, n - base);
+    const int* g = group ? group + base : nullptr;
     bool launched = false;
     if (m <= 16)
-      MP_TRY(launch_batch<16>(path, variant, dir, d + base, group ? group + base : nullptr, m, shift, cap, stream, &launched));
+      MP_TRY(launch_batch<16>(path, variant, dir, d + base, g, m, shift, cap, sms, stream, &launched));
     else if (m <= 128)
-      MP_TRY(launch_batch<128>(path, variant, dir, d + base, group ? group + base : nullptr, m, shift, cap, stream, &launched));
+      MP_TRY(launch_batch<128>(path, variant, dir, d + base, g, m, shift, cap, sms, stream, &launched));
     else
-      MP_TRY(launch_batch<kMaxDescPerLaunch>(path, variant, dir, d + base, group ? group + base : nullptr, m, shift, cap, stream,
-                                             &launched));
+      MP_TRY(launch_batch<kMaxDescPerLaunch>(path, variant, dir, d + base, g, m, shift, cap, sms, stream, &launched));
     if (launched && launches) ++*launches;
   }
   return MPRESS_OK;

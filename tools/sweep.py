@@ -64,10 +64,10 @@ def paths():
     nbytes = sum(sizes)
     ctx, pl, src, dst = setup(sizes, 3)
     s = torch.cuda.Stream()
-    nvar = {"direct": 4, "bulk": 3, "ce": 1}
+    nvar = {"direct": 4, "bulk": 3, "ce": 1}  # plus -1 = auto
     for name, path in PATHS.items():
         caps = [0] if name == "ce" else [0, 8, 16, 32, 64, 148, 296, 444, 592]
-        for var in range(nvar[name]):
+        for var in ([-1] if name != "ce" else []) + list(range(nvar[name])):
             for cap in caps:
                 ctx.set_option(mp.OPT_PATH, path)
                 if name != "ce":
