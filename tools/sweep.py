@@ -132,7 +132,7 @@ def gemm():
         print(json.dumps({"sweep": "gemm", "shape": sname, "mode": "alone", "gemm_ms": alone,
                           "tflops": 2 * M * N * K / alone / 1e9}), flush=True)
         for name in ("direct", "bulk", "ce"):
-            caps = [0] if name == "ce" else [4, 8, 16, 32, 0]
+            caps = [0] if name == "ce" else [8, 16, 24, 32, 48, 64, 0]
             for cap in caps:
                 ctx.set_option(mp.OPT_PATH, PATHS[name])
                 ctx.set_option(mp.OPT_MAX_CTAS, cap)
