@@ -321,10 +321,10 @@ struct Shape {
   int per_sm;       // default CTAs per SM when MPRESS_OPT_MAX_CTAS = 0
 };
 
-// direct: (threads, unroll) = (256,8) (512,8) (256,16) (1024,4)
+// direct: (threads, unroll) = (256,8) (512,8) (256,16) (1024,4) (128,8)
 // bulk:   (piece, stages)   = (32K,6) (16K,12) (64K,3)
 constexpr Shape kDirect[kDirectVariants] = {
-    {256, 15, 0, 2}, {512, 16, 0, 1}, {256, 16, 0, 2}, {1024, 16, 0, 1}};
+    {256, 15, 0, 2}, {512, 16, 0, 1}, {256, 16, 0, 2}, {1024, 16, 0, 1}, {128, 14, 0, 4}};
 constexpr Shape kBulk[kBulkVariants] = {
     {32, 15, 6u << 15, 1}, {32, 14, 12u << 14, 1}, {32, 16, 3u << 16, 1}};
 
@@ -348,6 +348,7 @@ KernelFn<CAP> kernel_for(int path, int variant, int dir, bool pf) {
     case 1: return MP_DIRECT(512, 8);
     case 2: return MP_DIRECT(256, 16);
     case 3: return MP_DIRECT(1024, 4);
+    case 4: return MP_DIRECT(128, 8);
     default: return MP_DIRECT(256, 8);
   }
 #undef MP_DIRECT

@@ -131,11 +131,13 @@ def gemm():
         torch.cuda.synchronize()
         print(json.dumps({"sweep": "gemm", "shape": sname, "mode": "alone", "gemm_ms": alone,
                           "tflops": 2 * M * N * K / alone / 1e9}), flush=True)
-        for name in ("direct", "bulk", "ce"):
-            caps = [0] if name == "ce" else [8, 16, 24, 32, 48, 64, 0]
-            for cap in caps:
+        combos = [("direct", v, c) for v in (0, 1, 4) for c in (16, 32, 64, 96, 148)]
+        combos += [("bulk", 0, c) for c in (8, 16, 32)] + [("ce", 0, 0)]
+        for name, var, cap in combos:
+            if True:
                 ctx.set_option(mp.OPT_PATH, PATHS[name])
-                ctx.set_option(mp.OPT_MAX_CTAS, cap)
+                if name != "ce":
+                    ctx.set_option(mp.OPT_VARIANT, var)
                 # swaps looped on the side stream to cover the GEMM window
                 n_gemm = 60
                 window_ms = alone * n_gemm
@@ -160,7 +162,7 @@ def gemm():
                     inside = [float("nan")]
                 during = statistics.median(inside)
                 print(json.dumps({"sweep": "gemm", "shape": sname, "mode": "with_swap", "path": name,
-                                  "max_ctas": cap, "gemm_ms": during,
+                                  "variant": var, "max_ctas": cap, "gemm_ms": during,
                                   "slowdown": during / alone - 1,
                                   "swap_gbs_under_gemm": 2 * n_swap * nbytes / swap_ms / 1e6}), flush=True)
     ctx.finalize()
