@@ -73,6 +73,7 @@ def paths():
                 if name != "ce":
                     ctx.set_option(mp.OPT_VARIANT, var)
                 ctx.set_option(mp.OPT_MAX_CTAS, cap)
+                ctx.set_option(mp.OPT_MAX_CTAS, cap)
                 for order in (mp.ORDER_INTERLEAVE, mp.ORDER_PLAN):
                     ctx.set_option(mp.OPT_ORDER, order)
                     to, ti = time_swaps(ctx, pl, src, dst, 10, s)
