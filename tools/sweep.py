@@ -73,7 +73,6 @@ def paths():
                 if name != "ce":
                     ctx.set_option(mp.OPT_VARIANT, var)
                 ctx.set_option(mp.OPT_MAX_CTAS, cap)
-                ctx.set_option(mp.OPT_MAX_CTAS, cap)
                 for order in (mp.ORDER_INTERLEAVE, mp.ORDER_PLAN):
                     ctx.set_option(mp.OPT_ORDER, order)
                     to, ti = time_swaps(ctx, pl, src, dst, 10, s)
@@ -102,20 +101,24 @@ def sizes_sweep():
 
 
 def gemm():
+    """GEMM slowdown with the bench's protocol: for every (path, variant, cap)
+    an alone round and a with-swap round of 24 GEMMs alternate, and only GEMMs
+    that ran entirely inside the swap window count."""
     sizes = workloads.cfg2_sizes(1)
     nbytes = sum(sizes)
     ctx, pl, src, dst = setup(sizes, 3)
     shapes = {"8192^3": (8192, 8192, 8192), "gpt_fc1": (4096, 5120, 20480)}
     comp = torch.cuda.current_stream()
     swap = torch.cuda.Stream()
+    G = 24
     for sname, (M, K, N) in shapes.items():
         a = torch.randn(M, K, dtype=torch.bfloat16, device="cuda")
         b = torch.randn(K, N, dtype=torch.bfloat16, device="cuda")
         c = torch.empty(M, N, dtype=torch.bfloat16, device="cuda")
 
-        def gemms(n):
+        def gemms():
             evs = []
-            for _ in range(n):
+            for _ in range(G):
                 e0 = torch.cuda.Event(enable_timing=True)
                 e1 = torch.cuda.Event(enable_timing=True)
                 e0.record(comp)
@@ -124,48 +127,42 @@ def gemm():
                 evs.append((e0, e1))
             return evs
 
-        gemms(20)
+        gemms()
         torch.cuda.synchronize()
-        evs = gemms(60)
-        torch.cuda.synchronize()
-        alone = statistics.median(x.elapsed_time(y) for x, y in evs)
-        torch.cuda.synchronize()
-        print(json.dumps({"sweep": "gemm", "shape": sname, "mode": "alone", "gemm_ms": alone,
-                          "tflops": 2 * M * N * K / alone / 1e9}), flush=True)
-        combos = [("direct", v, c) for v in (0, 1, 4) for c in (16, 32, 64, 96, 148)]
-        combos += [("bulk", 0, c) for c in (8, 16, 32)] + [("ce", 0, 0)]
+        combos = [("direct", v, cap) for v in (0, 1, 4) for cap in (16, 32, 64, 96, 148)]
+        combos += [("bulk", 0, cap) for cap in (8, 16, 32)] + [("ce", 0, 0)]
         for name, var, cap in combos:
-            if True:
-                ctx.set_option(mp.OPT_PATH, PATHS[name])
-                if name != "ce":
-                    ctx.set_option(mp.OPT_VARIANT, var)
-                # swaps looped on the side stream to cover the GEMM window
-                n_gemm = 60
-                window_ms = alone * n_gemm
-                to, ti = time_swaps(ctx, pl, src, dst, 3, swap)
-                n_swap = int(window_ms / (to + ti)) + 2
+            ctx.set_option(mp.OPT_PATH, PATHS[name])
+            if name != "ce":
+                ctx.set_option(mp.OPT_VARIANT, var)
+            ctx.set_option(mp.OPT_MAX_CTAS, cap)
+            to, ti = time_swaps(ctx, pl, src, dst, 3, swap)
+            alone, during, gbs = [], [], []
+            for _ in range(2):
+                evs = gemms()
                 torch.cuda.synchronize()
-                sw0 = torch.cuda.Event(enable_timing=True)
-                sw1 = torch.cuda.Event(enable_timing=True)
-                sw0.record(swap)
+                alone += [x.elapsed_time(y) for x, y in evs[4:]]
+                n_swap = int(2.0 * G * statistics.median(alone) / (to + ti)) + 2
+                s0 = torch.cuda.Event(enable_timing=True)
+                s1 = torch.cuda.Event(enable_timing=True)
+                s0.record(swap)
                 for _ in range(n_swap):
                     h = ctx.swap_out(pl, src, stream=swap)
                     ctx.swap_in(h, dst, stream=swap)
                     h.free()
-                sw1.record(swap)
-                evs = gemms(n_gemm)
+                s1.record(swap)
+                evs = gemms()
                 torch.cuda.synchronize()
-                swap_ms = sw0.elapsed_time(sw1)
-                # only GEMMs that ran entirely inside the swap window
-                inside = [x.elapsed_time(y) for x, y in evs
-                          if sw0.elapsed_time(x) >= 0 and sw0.elapsed_time(y) <= swap_ms]
-                if not inside:
-                    inside = [float("nan")]
-                during = statistics.median(inside)
-                print(json.dumps({"sweep": "gemm", "shape": sname, "mode": "with_swap", "path": name,
-                                  "variant": var, "max_ctas": cap, "gemm_ms": during,
-                                  "slowdown": during / alone - 1,
-                                  "swap_gbs_under_gemm": 2 * n_swap * nbytes / swap_ms / 1e6}), flush=True)
+                win = s0.elapsed_time(s1)
+                during += [x.elapsed_time(y) for x, y in evs[4:]
+                           if s0.elapsed_time(x) >= 0 and s0.elapsed_time(y) <= win]
+                gbs.append(2 * n_swap * nbytes / win / 1e6)
+            am = statistics.median(alone)
+            dm = statistics.median(during) if during else float("nan")
+            print(json.dumps({"sweep": "gemm", "shape": sname, "path": name, "variant": var,
+                              "max_ctas": cap, "alone_ms": am, "gemm_ms": dm, "slowdown": dm / am - 1,
+                              "counted": len(during), "swap_alone_gbs": 2 * nbytes / (to + ti) / 1e6,
+                              "swap_gbs_under_gemm": statistics.median(gbs)}), flush=True)
     ctx.finalize()
 
 
