@@ -55,7 +55,7 @@ def parse():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
-    ap.add_argument("--gemm-cap", type=int, default=32,
+    ap.add_argument("--gemm-cap", type=int, default=96,
                     help="swap grid cap (CTAs = SMs touched) while the concurrent GEMM runs")
     ap.add_argument("--no-gemm", action="store_true")
     return ap.parse_args()

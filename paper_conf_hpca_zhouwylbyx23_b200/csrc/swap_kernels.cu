@@ -450,10 +450,12 @@ int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* gr
   if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess)
     return fail(MPRESS_ERR_CUDA, "cannot query the SM count");
   if (variant == MPRESS_VARIANT_AUTO) {
-    // direct: a capped grid (<= one CTA per SM, e.g. beside a GEMM) moves the
-    // most bytes per SM with 512-thread CTAs; a full grid saturates HBM with
-    // 2 x 256-thread CTAs per SM (profiles/r01 sweeps).  bulk: 6 x 32 KiB.
-    variant = (path == MPRESS_PATH_DIRECT && max_ctas > 0 && max_ctas <= sms) ? 1 : 0;
+    // direct, capped grid (<= one CTA per SM, i.e. beside a GEMM): 128-thread
+    // CTAs fit in the registers and shared memory a cuBLAS GEMM CTA leaves
+    // free (168 regs x 256 threads + 214 KB smem, profiles/r01), so they
+    // co-reside instead of taking SMs away from it; full grid: 2 x 256-thread
+    // CTAs per SM saturate HBM (profiles/r01 sweeps).  bulk: 6 x 32 KiB.
+    variant = (path == MPRESS_PATH_DIRECT && max_ctas > 0 && max_ctas <= sms) ? 4 : 0;
   }
   const int nvar = path == MPRESS_PATH_BULK ? kBulkVariants : kDirectVariants;
   if (variant < 0 || variant >= nvar) return fail(MPRESS_ERR_ARG, "kernel variant %d out of range", variant);

@@ -129,8 +129,14 @@ def gemm():
 
         gemms()
         torch.cuda.synchronize()
-        combos = [("direct", v, cap) for v in (0, 1, 4) for cap in (16, 32, 64, 96, 148)]
-        combos += [("bulk", 0, cap) for cap in (8, 16, 32)] + [("ce", 0, 0)]
+        if os.environ.get("GEMM_COMBOS"):  # e.g. "direct:4:64,96,128;ce:0:0"
+            combos = []
+            for part in os.environ["GEMM_COMBOS"].split(";"):
+                nm, v, caps = part.split(":")
+                combos += [(nm, int(v), int(cap)) for cap in caps.split(",")]
+        else:
+            combos = [("direct", v, cap) for v in (0, 1, 4) for cap in (16, 32, 64, 96, 148)]
+            combos += [("bulk", 0, cap) for cap in (8, 16, 32)] + [("ce", 0, 0)]
         for name, var, cap in combos:
             ctx.set_option(mp.OPT_PATH, PATHS[name])
             if name != "ce":
