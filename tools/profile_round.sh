@@ -14,3 +14,7 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:mp_s
     -o $OUT/prof_swap python bench.py --steps 1 --warmup 1 --micro-batches 1 --e2e-steps 1 \
     --no-cpu-baseline --no-gemm "$@" > $OUT/ncu_full.log 2>&1
 cat $OUT/bench.json; tail -3 $OUT/bench.err
+# the capped configuration the GEMM leg uses (auto variant -> 128-thread CTAs)
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:mp_swap -s 2 -c 2 \
+    -o $OUT/prof_swap_capped python bench.py --steps 1 --warmup 1 --micro-batches 1 --e2e-steps 1 \
+    --no-cpu-baseline --no-gemm --max-ctas 64 "$@" > $OUT/ncu_full_capped.log 2>&1
