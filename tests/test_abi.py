@@ -166,3 +166,31 @@ def test_partition_config5_parity():
     reqs = [(s, workloads.cfg5_source_sizes(s), 1) for s in c["sources"]]
     op, _ = oracle.sequential_partition(world, spare, bwm, reqs)
     assert mp.partition_sequential(world, spare, bwm, reqs) == op
+
+
+def test_init_argument_errors_without_gpu():
+    """Partition validation happens before any CUDA call (R21: a source never
+    stashes on itself; partitions are 256-byte multiples)."""
+    import ctypes
+    P = ctypes.c_void_p
+    h = P()
+    devs = (ctypes.c_int * 2)(0, 0)
+    bad_self = (ctypes.c_uint64 * 4)(256, 0, 0, 0)
+    assert mp.lib.mpress_init_local(2, 0, devs, bad_self, ctypes.byref(h)) == mp.ERR_ARG
+    assert "itself" in mp.lib.mpress_last_error().decode()
+    bad_align = (ctypes.c_uint64 * 4)(0, 100, 0, 0)
+    assert mp.lib.mpress_init_local(2, 0, devs, bad_align, ctypes.byref(h)) == mp.ERR_ARG
+    assert mp.lib.mpress_init_local(2, 2, devs, bad_align, ctypes.byref(h)) == mp.ERR_ARG
+    assert mp.lib.mpress_finalize(None) == 0
+    with pytest.raises(mp.MPressError) as ei:
+        mp.plan(3, 0, [0, 1], [0, 1, 1], [10])
+    assert ei.value.code == mp.ERR_ARG
+
+
+def test_plan_overflow_and_zero_size_rejected():
+    with pytest.raises(mp.MPressError) as ei:
+        mp.plan(2, 0, [0, 1 << 40], [0, 1], [1 << 63, 1 << 63])
+    assert ei.value.code == mp.ERR_ARG
+    with pytest.raises(mp.MPressError) as ei:
+        mp.plan(2, 0, [0, 1 << 40], [0, 1], [5, 0])
+    assert ei.value.code == mp.ERR_ARG
