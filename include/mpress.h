@@ -158,6 +158,42 @@ MPRESS_API int mpress_partition_sequential(int world, const uint64_t* spare_byte
                                 const uint64_t* sizes_flat, const uint32_t* copies,
                                 uint64_t granule, uint64_t* partition);
 
+/*
+ * mpress_plan_global -- NEXT-1: joint assignment of several exporters'
+ * batches to the importers' spare memory (Fig. 6: every way to
+ * distribute each importer's spare among its overflowed neighbours, combined
+ * and scored by the reciprocal of the maximal D2D swap time; reading
+ * R23).  All sources swap at once; with x_sp units of source s on importer p
+ *   T = max( x_sp / B_sp  (every used link),
+ *            sum_p x_sp / E_s  (egress port, if egress && egress[s] > 0),
+ *            sum_s x_sp / I_p  (ingress port, if ingress && ingress[p] > 0) )
+ * is minimised exactly over integer units subject to sum_p x_sp = K_s and
+ * sum_s x_sp <= floor(spare_p / G).
+ *   sources [n_sources] distinct exporters; n_tensors [n_sources];
+ *   sizes_flat the exporters' tensor sizes, concatenated in that order;
+ *   bw_matrix [world*world] row s = link weights of s (0 = no link);
+ *   egress / ingress [world] port weights or NULL (no port limit);
+ *   units_out [n_sources*world] out: x (row i = sources[i]);
+ *   makespan_num / makespan_den out (may be NULL): T* = num / den units per
+ *   weight unit.
+ * T* is unique; the assignment is one optimal x, identical on every rank.
+ * Turn a row into a plan with mpress_plan_from_units.
+ * Errors: MPRESS_ERR_ARG, MPRESS_ERR_NO_SPACE.
+ */
+MPRESS_API int mpress_plan_global(int world, uint32_t n_sources, const int32_t* sources,
+                                  const uint32_t* n_tensors, const uint64_t* sizes_flat,
+                                  const uint64_t* spare_bytes, const uint64_t* bw_matrix,
+                                  const uint64_t* egress, const uint64_t* ingress, uint64_t granule,
+                                  uint64_t* units_out, uint64_t* makespan_num,
+                                  uint64_t* makespan_den);
+
+/* mpress_plan_from_units -- the plan (layout and stripes, R6/R7) of one batch
+ * for a given unit split units[world] (e.g. a row of mpress_plan_global).
+ * Errors: MPRESS_ERR_ARG if units[source] != 0 or sum(units) != K. */
+MPRESS_API int mpress_plan_from_units(int world, int source, const uint64_t* units,
+                                      uint32_t n_tensors, const uint64_t* tensor_bytes,
+                                      uint64_t granule, mpress_plan_t** out);
+
 /* ---- peer-memory layer ----------------------------------------------------- */
 
 /* All-gather callback, implemented by the caller over its process group:

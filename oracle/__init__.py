@@ -15,6 +15,7 @@ Modules
   bytemodel  -- byte-exact model of swap-out / swap-in
   brute      -- exhaustive minimum-makespan search for tiny inputs
   partition  -- sequential multi-source stash reservation (reading R12)
+  global_plan -- NEXT-1: joint multi-exporter assignment (Fig. 6, R23)
 
 Pins (tests/test_oracle.py): the paper's worked 1:2 ratio (golden G2),
 equal striping on symmetric links, brute-force optimality of the score
@@ -23,8 +24,9 @@ bandwidth-proportionality bound, round-trip identity, and a
 hand-checked golden plan (G1).  No function here is "parity unpinned".
 """
 from .plan import (  # noqa: F401
-    ALIGN, DEFAULT_GRANULE, PlanError, ERR_ARG, ERR_NO_SPACE, plan, virtual_layout,
+    ALIGN, DEFAULT_GRANULE, PlanError, ERR_ARG, ERR_NO_SPACE, plan, plan_from_units, virtual_layout,
 )
 from .bytemodel import swap_out, swap_in, stash_sizes  # noqa: F401
 from .brute import brute_force_makespan, makespan  # noqa: F401
 from .partition import sequential_partition  # noqa: F401
+from .global_plan import brute_force_global, scan_global, assignment_time  # noqa: F401

@@ -31,7 +31,8 @@ _ERR_NAMES = {ERR_ARG: "ERR_ARG", ERR_NO_SPACE: "ERR_NO_SPACE", ERR_ALIGN: "ERR_
 
 EXPORTED = [
     "mpress_plan", "mpress_plan_stripes", "mpress_plan_units", "mpress_plan_get_info",
-    "mpress_plan_free", "mpress_partition_sequential", "mpress_init", "mpress_init_local",
+    "mpress_plan_free", "mpress_partition_sequential", "mpress_plan_global",
+    "mpress_plan_from_units", "mpress_init", "mpress_init_local",
     "mpress_finalize", "mpress_stash_free", "mpress_set_option", "mpress_get_option",
     "mpress_swap_out", "mpress_swap_in", "mpress_wait", "mpress_query", "mpress_handle_state",
     "mpress_handle_slices", "mpress_handle_free", "mpress_peer_read", "mpress_last_launches",
@@ -72,6 +73,9 @@ def _load():
         "mpress_plan_get_info": (c_int, [P, POINTER(PlanInfo)]),
         "mpress_plan_free": (None, [P]),
         "mpress_partition_sequential": (c_int, [c_int, P, P, c_uint32, P, P, P, P, c_uint64, P]),
+        "mpress_plan_global": (c_int, [c_int, c_uint32, P, P, P, P, P, P, P, c_uint64, P,
+                                       POINTER(c_uint64), POINTER(c_uint64)]),
+        "mpress_plan_from_units": (c_int, [c_int, c_int, P, c_uint32, P, c_uint64, POINTER(P)]),
         "mpress_init": (c_int, [c_int, c_int, c_int, P, EXCHANGE_FN, P, POINTER(P)]),
         "mpress_init_local": (c_int, [c_int, c_int, P, P, POINTER(P)]),
         "mpress_finalize": (c_int, [P]),
@@ -188,6 +192,34 @@ class Plan:
 
 def plan(world, source, spare, bw, sizes, granule=0):
     return Plan(world, source, spare, bw, sizes, granule)
+
+
+def plan_from_units(world, source, units, sizes, granule=0):
+    """The plan of a batch for a given per-peer unit split (mpress_plan_from_units)."""
+    p = Plan.__new__(Plan)
+    h = c_void_p()
+    _check(lib.mpress_plan_from_units(world, source, _u64(units), len(sizes), _u64(sizes),
+                                      granule, byref(h)))
+    p._h = h
+    p.world = world
+    p.sizes = [int(s) for s in sizes]
+    return p
+
+
+def plan_global(world, requests, spare, bw_matrix, egress=None, ingress=None, granule=0):
+    """NEXT-1 (mpress_plan_global).  requests: [(source, sizes)].
+    Returns (units {source: [world]}, (num, den)) with T* = num / den."""
+    srcs = (c_int32 * len(requests))(*[r[0] for r in requests])
+    ns = (c_uint32 * len(requests))(*[len(r[1]) for r in requests])
+    flat = _u64([s for r in requests for s in r[1]])
+    out = (c_uint64 * (len(requests) * world))()
+    num, den = c_uint64(), c_uint64()
+    _check(lib.mpress_plan_global(world, len(requests), srcs, ns, flat, _u64(spare),
+                                  _u64([b for row in bw_matrix for b in row]),
+                                  _u64(egress) if egress else None, _u64(ingress) if ingress else None,
+                                  granule, out, byref(num), byref(den)))
+    units = {r[0]: [out[i * world + p] for p in range(world)] for i, r in enumerate(requests)}
+    return units, (num.value, den.value)
 
 
 def partition_sequential(world, spare, bw_matrix, requests, granule=0):

@@ -129,6 +129,9 @@ void exact_fixup(std::vector<Peer>& peers, uint64_t K) {
   }
 }
 
+int layout_batch(uint32_t n, const uint64_t* sizes, uint64_t G, mpress_plan_s* pl);
+void build_layout(mpress_plan_s* pl);
+
 int build_plan(int world, int source, const uint64_t* spare, const uint64_t* bw, uint32_t n,
                const uint64_t* sizes, uint64_t granule, mpress_plan_s* pl) {
   if (world < 1 || source < 0 || source >= world)
@@ -143,20 +146,7 @@ int build_plan(int world, int source, const uint64_t* spare, const uint64_t* bw,
 
   pl->world = world;
   pl->source = source;
-  pl->G = G;
-  pl->sizes.assign(sizes, sizes + n);
-  pl->offsets.resize(n);
-  uint64_t V = 0;
-  for (uint32_t i = 0; i < n; ++i) {
-    if (sizes[i] == 0) return fail(MPRESS_ERR_ARG, "mpress_plan: tensor %u has 0 bytes", i);
-    pl->offsets[i] = V;
-    uint64_t padded;
-    if (sizes[i] > UINT64_MAX - (MPRESS_ALIGN - 1) || !add_ok(V, roundup(sizes[i], MPRESS_ALIGN), &padded))
-      return fail(MPRESS_ERR_ARG, "mpress_plan: batch size overflows 64 bits");
-    V = padded;
-  }
-  pl->V = V;
-  pl->K = V / G + (V % G != 0);
+  MP_TRY(layout_batch(n, sizes, G, pl));
 
   std::vector<Peer> peers;
   u128 capsum = 0;
@@ -177,9 +167,37 @@ int build_plan(int world, int source, const uint64_t* spare, const uint64_t* bw,
 
   pl->units.assign(world, 0);
   for (auto& q : peers) pl->units[q.p] = q.k;
+  build_layout(pl);
+  return MPRESS_OK;
+}
 
-  // Contiguous ranges per peer (ascending), intersected with the tensors by a
-  // single forward walk over the batch.
+// Virtual layout of the batch (offsets, V, K) from the tensor sizes.
+int layout_batch(uint32_t n, const uint64_t* sizes, uint64_t G, mpress_plan_s* pl) {
+  pl->G = G;
+  pl->sizes.assign(sizes, sizes + n);
+  pl->offsets.resize(n);
+  uint64_t V = 0;
+  for (uint32_t i = 0; i < n; ++i) {
+    if (sizes[i] == 0) return fail(MPRESS_ERR_ARG, "tensor %u has 0 bytes", i);
+    pl->offsets[i] = V;
+    uint64_t padded;
+    if (sizes[i] > UINT64_MAX - (MPRESS_ALIGN - 1) || !add_ok(V, roundup(sizes[i], MPRESS_ALIGN), &padded))
+      return fail(MPRESS_ERR_ARG, "batch size overflows 64 bits");
+    V = padded;
+  }
+  pl->V = V;
+  pl->K = V / G + (V % G != 0);
+  return MPRESS_OK;
+}
+
+// Contiguous ranges per peer (ascending), intersected with the tensors by a
+// single forward walk over the batch; pl->units must be set.
+void build_layout(mpress_plan_s* pl) {
+  const int world = pl->world;
+  const uint64_t G = pl->G, V = pl->V;
+  const uint32_t n = (uint32_t)pl->sizes.size();
+  const uint64_t* sizes = pl->sizes.data();
+  pl->stripes.clear();
   pl->peer_bytes.assign(world, 0);
   uint64_t a = 0;
   uint32_t i = 0;
@@ -198,7 +216,6 @@ int build_plan(int world, int source, const uint64_t* spare, const uint64_t* bw,
     }
     a = b;
   }
-  return MPRESS_OK;
 }
 
 }  // namespace
@@ -256,6 +273,36 @@ extern "C" int mpress_plan_get_info(const mpress_plan_t* plan, mpress_plan_info*
 }
 
 extern "C" void mpress_plan_free(mpress_plan_t* plan) { delete plan; }
+
+extern "C" int mpress_plan_from_units(int world, int source, const uint64_t* units, uint32_t n_tensors,
+                                      const uint64_t* tensor_bytes, uint64_t granule, mpress_plan_t** out) {
+  if (!out) return fail(MPRESS_ERR_ARG, "mpress_plan_from_units: out is null");
+  *out = nullptr;
+  if (world < 1 || source < 0 || source >= world || !units || !tensor_bytes || n_tensors == 0)
+    return fail(MPRESS_ERR_ARG, "mpress_plan_from_units: bad argument");
+  const uint64_t G = granule ? granule : MPRESS_DEFAULT_GRANULE;
+  if (G % MPRESS_ALIGN != 0) return fail(MPRESS_ERR_ARG, "mpress_plan_from_units: granule not a multiple of 256");
+  auto* pl = new (std::nothrow) mpress_plan_s();
+  if (!pl) return fail(MPRESS_ERR_ARG, "mpress_plan_from_units: out of host memory");
+  pl->world = world;
+  pl->source = source;
+  int rc = layout_batch(n_tensors, tensor_bytes, G, pl);
+  u128 sum = 0;
+  for (int p = 0; p < world && rc == MPRESS_OK; ++p) sum += units[p];
+  if (rc == MPRESS_OK && units[source] != 0)
+    rc = fail(MPRESS_ERR_ARG, "mpress_plan_from_units: units on the source itself");
+  if (rc == MPRESS_OK && sum != pl->K)
+    rc = fail(MPRESS_ERR_ARG, "mpress_plan_from_units: units sum to %llu, the batch has %llu",
+              (unsigned long long)sum, (unsigned long long)pl->K);
+  if (rc != MPRESS_OK) {
+    delete pl;
+    return rc;
+  }
+  pl->units.assign(units, units + world);
+  build_layout(pl);
+  *out = pl;
+  return MPRESS_OK;
+}
 
 extern "C" int mpress_partition_sequential(int world, const uint64_t* spare_bytes,
                                            const uint64_t* bw_matrix, uint32_t n_sources,
