@@ -396,8 +396,10 @@ def main():
                                                         sizes, src, dst, swap_stream, n, dist)
 
     cpu = None
+    planner = None
     if rank == 0 and n == 1 and not args.no_cpu_baseline:
         cpu = oracle_sample(args.cpu_seconds)
+        planner = planner_timing(mp, world, source, per_copy, bw, sizes)
 
     if rank == 0:
         line = {
@@ -409,6 +411,7 @@ def main():
             "per_direction_gbs": per_dir,
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": launches[0], "clocks": clk, "gemm_slowdown": gemm,
+            "planner": planner,
             "parity": "round trip bit-exact vs generator (all %d tensors x %d ranks)" % (47 * mb, n),
         }
         print(json.dumps(line))
@@ -416,6 +419,23 @@ def main():
     if n > 1:
         dist.destroy_process_group()
     return 0
+
+
+def planner_timing(mp, world, source, spare, bw, sizes):
+    """a1 PLAN on the host: the C++ planner (mpress_plan) against the oracle's
+    Python planner on the bench's micro-batch (SURVEY §8(d) "planner timing")."""
+    import oracle
+    reps = 2000
+    t0 = time.perf_counter()
+    for _ in range(reps):
+        mp.plan(world, source, spare, bw, sizes)
+    cpp_us = (time.perf_counter() - t0) / reps * 1e6
+    t0 = time.perf_counter()
+    o = oracle.plan(world, source, spare, bw, sizes)
+    py_us = (time.perf_counter() - t0) * 1e6
+    assert mp.plan(world, source, spare, bw, sizes).stripes == [tuple(s) for s in o["stripes"]]
+    return {"cpp_us_per_plan": cpp_us, "oracle_us_per_plan": py_us, "units": o["K"],
+            "stripes": len(o["stripes"]), "note": "cpp includes the ctypes call; identical plans"}
 
 
 def traffic_from_profile():
