@@ -194,6 +194,59 @@ MPRESS_API int mpress_plan_from_units(int world, int source, const uint64_t* uni
                                       uint32_t n_tensors, const uint64_t* tensor_bytes,
                                       uint64_t granule, mpress_plan_t** out);
 
+/* ---- NEXT-2: 1F1B swap schedule with the live-interval check ------------------ */
+
+/* Inputs (all times in ns, integers).  Computation-balanced stages:
+ * every stage takes t_fwd_ns / t_bwd_ns per micro-batch. */
+typedef struct mpress_1f1b_params {
+  uint32_t stages;         /* S >= 1 pipeline stages (Fig. 1)            */
+  uint32_t stage;          /* the exporter stage e in [0, S) that swaps            */
+  uint32_t micro_batches;  /* M >= 1 per mini-batch                                */
+  uint32_t duplex;         /* 1: swap-outs and swap-ins on two streams     */
+  uint64_t t_fwd_ns;
+  uint64_t t_bwd_ns;
+  uint64_t t_out_ns;       /* swap-out of one micro-batch's activations            */
+  uint64_t t_in_ns;        /* swap-in of them (from the measured GB/s)             */
+} mpress_1f1b_params;
+
+typedef struct mpress_1f1b_slot {  /* one micro-batch at the exporter stage */
+  uint64_t fwd_start, fwd_end, bwd_start, bwd_end;  /* with swapping          */
+  uint64_t live_ns;        /* live interval without swapping: backward start -
+                              forward end (P:226 fn.1)                         */
+  uint64_t out_start, out_end, in_start, in_end;
+  uint32_t in_trigger;     /* the swap-in is enqueued when op #in_trigger of the
+                              stage (1F1B order, 0-based) has ended: the last op
+                              that still leaves t_in before the backward       */
+  uint32_t hidden;         /* 1 if the swap-in ended before the backward could
+                              otherwise start (no extra delay)          */
+  uint64_t exposed_ns;     /* backward start with swapping - without           */
+} mpress_1f1b_slot;
+
+typedef struct mpress_1f1b_summary {
+  uint64_t makespan_ns;            /* whole pipeline, with the exporter swapping */
+  uint64_t makespan_noswap_ns;
+  uint32_t peak_resident;          /* max micro-batch activation sets resident on
+                                      the exporter at once, with swapping       */
+  uint32_t peak_resident_noswap;
+  uint32_t ops;                    /* compute ops of the exporter stage (2M)    */
+  uint32_t pad;
+} mpress_1f1b_summary;
+
+/*
+ * mpress_schedule_1f1b -- the swap schedule of the exporter stage in a 1F1B
+ * pipeline (PipeDream / DAPPLE): every micro-batch's
+ * activations are swapped out after its forward and swapped back in
+ * on the swap-in stream as late as the no-swap timeline allows them to
+ * still arrive before the backward; per micro-batch it reports the live
+ * interval (P:226 fn.1), the swap times, whether the swap is hidden
+ * and the exposed delay (fn.2), plus peak resident activation sets
+ * with and without swapping (the memory the D2D swap saves).  Model: reading
+ * R24.  slots [micro_batches] out; summary may be NULL.
+ * Errors: MPRESS_ERR_ARG.
+ */
+MPRESS_API int mpress_schedule_1f1b(const mpress_1f1b_params* params, mpress_1f1b_slot* slots,
+                                    mpress_1f1b_summary* summary);
+
 /* ---- peer-memory layer ----------------------------------------------------- */
 
 /* All-gather callback, implemented by the caller over its process group:

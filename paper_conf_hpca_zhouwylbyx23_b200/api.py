@@ -32,7 +32,7 @@ _ERR_NAMES = {ERR_ARG: "ERR_ARG", ERR_NO_SPACE: "ERR_NO_SPACE", ERR_ALIGN: "ERR_
 EXPORTED = [
     "mpress_plan", "mpress_plan_stripes", "mpress_plan_units", "mpress_plan_get_info",
     "mpress_plan_free", "mpress_partition_sequential", "mpress_plan_global",
-    "mpress_plan_from_units", "mpress_init", "mpress_init_local",
+    "mpress_plan_from_units", "mpress_schedule_1f1b", "mpress_init", "mpress_init_local",
     "mpress_finalize", "mpress_stash_free", "mpress_set_option", "mpress_get_option",
     "mpress_swap_out", "mpress_swap_in", "mpress_wait", "mpress_query", "mpress_handle_state",
     "mpress_handle_slices", "mpress_handle_free", "mpress_peer_read", "mpress_last_launches",
@@ -57,6 +57,24 @@ class PlanInfo(ctypes.Structure):
                 ("units", c_uint64)]
 
 
+class Params1F1B(ctypes.Structure):
+    _fields_ = [("stages", c_uint32), ("stage", c_uint32), ("micro_batches", c_uint32),
+                ("duplex", c_uint32), ("t_fwd_ns", c_uint64), ("t_bwd_ns", c_uint64),
+                ("t_out_ns", c_uint64), ("t_in_ns", c_uint64)]
+
+
+class Slot1F1B(ctypes.Structure):
+    _fields_ = [(n, c_uint64) for n in ("fwd_start", "fwd_end", "bwd_start", "bwd_end", "live_ns",
+                                        "out_start", "out_end", "in_start", "in_end")] + \
+               [("in_trigger", c_uint32), ("hidden", c_uint32), ("exposed_ns", c_uint64)]
+
+
+class Summary1F1B(ctypes.Structure):
+    _fields_ = [("makespan_ns", c_uint64), ("makespan_noswap_ns", c_uint64),
+                ("peak_resident", c_uint32), ("peak_resident_noswap", c_uint32),
+                ("ops", c_uint32), ("pad", c_uint32)]
+
+
 EXCHANGE_FN = CFUNCTYPE(c_int, c_void_p, c_void_p, c_size_t, c_void_p)
 
 
@@ -76,6 +94,7 @@ def _load():
         "mpress_plan_global": (c_int, [c_int, c_uint32, P, P, P, P, P, P, P, c_uint64, P,
                                        POINTER(c_uint64), POINTER(c_uint64)]),
         "mpress_plan_from_units": (c_int, [c_int, c_int, P, c_uint32, P, c_uint64, POINTER(P)]),
+        "mpress_schedule_1f1b": (c_int, [POINTER(Params1F1B), P, P]),
         "mpress_init": (c_int, [c_int, c_int, c_int, P, EXCHANGE_FN, P, POINTER(P)]),
         "mpress_init_local": (c_int, [c_int, c_int, P, P, POINTER(P)]),
         "mpress_finalize": (c_int, [P]),
@@ -204,6 +223,18 @@ def plan_from_units(world, source, units, sizes, granule=0):
     p.world = world
     p.sizes = [int(s) for s in sizes]
     return p
+
+
+def schedule_1f1b(stages, stage, micro_batches, t_fwd_ns, t_bwd_ns, t_out_ns, t_in_ns, duplex=True):
+    """NEXT-2 (mpress_schedule_1f1b): (slots as dicts, summary dict)."""
+    p = Params1F1B(stages, stage, micro_batches, 1 if duplex else 0, t_fwd_ns, t_bwd_ns,
+                   t_out_ns, t_in_ns)
+    slots = (Slot1F1B * micro_batches)()
+    summ = Summary1F1B()
+    _check(lib.mpress_schedule_1f1b(byref(p), slots, byref(summ)))
+    names = [f[0] for f in Slot1F1B._fields_]
+    return ([{n: getattr(s, n) for n in names} for s in slots],
+            {f[0]: getattr(summ, f[0]) for f in Summary1F1B._fields_ if f[0] != "pad"})
 
 
 def plan_global(world, requests, spare, bw_matrix, egress=None, ingress=None, granule=0):
