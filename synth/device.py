@@ -43,3 +43,21 @@ def check(t, seed, tensor_id, start=0, nbytes=None, stream=None):
     if r < 0:
         raise RuntimeError("synth_check failed")
     return r
+
+
+def stamp(base_u64, stream=None):
+    """Write %globaltimer into base_u64 (a 1-element int64 CUDA tensor)."""
+    lib = _get()
+    lib.synth_stamp.restype = ctypes.c_int
+    lib.synth_stamp.argtypes = [ctypes.c_void_p, ctypes.c_void_p]
+    if lib.synth_stamp(base_u64.data_ptr(), _stream(stream)) != 0:
+        raise RuntimeError("synth_stamp failed")
+
+
+def gate(base_u64, offset_ns, stream=None):
+    """Hold the stream until %globaltimer >= base + offset_ns."""
+    lib = _get()
+    lib.synth_gate.restype = ctypes.c_int
+    lib.synth_gate.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_void_p]
+    if lib.synth_gate(base_u64.data_ptr(), int(offset_ns), _stream(stream)) != 0:
+        raise RuntimeError("synth_gate failed")

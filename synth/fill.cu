@@ -77,3 +77,30 @@ extern "C" long long synth_check(const void* buf, uint64_t n, uint64_t seed, uin
   cudaFree(d_bad);
   return e == cudaSuccess ? (long long)h_bad : -1;
 }
+
+// ---- pipeline-replay helpers (tools/replay_1f1b.py) -------------------------
+// A replayed stage must wait for the other (absent) pipeline stages: stamp a
+// base time on the device, then gate each op until %globaltimer reaches
+// base + offset.  No method arithmetic.
+namespace {
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+__global__ void stamp_kernel(unsigned long long* base) { *base = gtimer(); }
+__global__ void gate_kernel(const unsigned long long* base, unsigned long long offset) {
+  const unsigned long long until = *base + offset;
+  while (gtimer() < until) __nanosleep(500);
+}
+}  // namespace
+
+extern "C" int synth_stamp(void* base, void* stream) {
+  stamp_kernel<<<1, 1, 0, (cudaStream_t)stream>>>((unsigned long long*)base);
+  return (int)cudaGetLastError();
+}
+
+extern "C" int synth_gate(const void* base, uint64_t offset_ns, void* stream) {
+  gate_kernel<<<1, 1, 0, (cudaStream_t)stream>>>((const unsigned long long*)base, offset_ns);
+  return (int)cudaGetLastError();
+}
