@@ -207,6 +207,7 @@ typedef struct mpress_1f1b_params {
   uint64_t t_bwd_ns;
   uint64_t t_out_ns;       /* swap-out of one micro-batch's activations            */
   uint64_t t_in_ns;        /* swap-in of them (from the measured GB/s)             */
+  uint64_t t_slack_ns;     /* extra lead the swap-in keeps before the backward     */
 } mpress_1f1b_params;
 
 typedef struct mpress_1f1b_slot {  /* one micro-batch at the exporter stage */

@@ -24,7 +24,7 @@ Model (reading R24), all times integers (ns):
     its own F(m)); at the exporter stage e, B(m)@e also needs swap-in(m);
     swap-out(m) needs F(m)@e; swap-in(m) needs swap-out(m) and its trigger op;
   * trigger op j(m) = the last op of stage e (in stage order, from F(m) up to
-    before B(m)) whose no-swap end <= B_start_noswap(m) - t_in: the swap-in
+    before B(m)) whose no-swap end <= B_start_noswap(m) - t_in - slack: the swap-in
     is issued as late as the no-swap timeline allows it to still be hidden;
   * swap-op order = the executor's enqueue order: after op j of stage e,
     first the swap-out of the micro-batch j produced (if j is a forward), then
@@ -91,7 +91,7 @@ def timeline_noswap(S, M, tf, tb):
                 lambda op: tf if op[1] == "F" else tb)
 
 
-def schedule(S, e, M, tf, tb, t_out, t_in, duplex=True):
+def schedule(S, e, M, tf, tb, t_out, t_in, duplex=True, slack=0):
     """(slots, summary) for exporter stage e; slots[m] has the fields of
     mpress_1f1b_slot, summary those of mpress_1f1b_summary (include/mpress.h)."""
     assert 0 <= e < S and M >= 1
@@ -100,7 +100,7 @@ def schedule(S, e, M, tf, tb, t_out, t_in, duplex=True):
     idx = {op: j for j, op in enumerate(ops)}
     trig = []
     for m in range(M):
-        target = s0[(e, "B", m)] - t_in
+        target = s0[(e, "B", m)] - t_in - slack
         j = idx[("F", m)]
         for jj in range(idx[("F", m)], idx[("B", m)]):
             if e0[(e,) + ops[jj]] <= target:

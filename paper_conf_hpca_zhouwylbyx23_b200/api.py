@@ -60,7 +60,7 @@ class PlanInfo(ctypes.Structure):
 class Params1F1B(ctypes.Structure):
     _fields_ = [("stages", c_uint32), ("stage", c_uint32), ("micro_batches", c_uint32),
                 ("duplex", c_uint32), ("t_fwd_ns", c_uint64), ("t_bwd_ns", c_uint64),
-                ("t_out_ns", c_uint64), ("t_in_ns", c_uint64)]
+                ("t_out_ns", c_uint64), ("t_in_ns", c_uint64), ("t_slack_ns", c_uint64)]
 
 
 class Slot1F1B(ctypes.Structure):
@@ -225,10 +225,11 @@ def plan_from_units(world, source, units, sizes, granule=0):
     return p
 
 
-def schedule_1f1b(stages, stage, micro_batches, t_fwd_ns, t_bwd_ns, t_out_ns, t_in_ns, duplex=True):
+def schedule_1f1b(stages, stage, micro_batches, t_fwd_ns, t_bwd_ns, t_out_ns, t_in_ns, duplex=True,
+                  slack_ns=0):
     """NEXT-2 (mpress_schedule_1f1b): (slots as dicts, summary dict)."""
     p = Params1F1B(stages, stage, micro_batches, 1 if duplex else 0, t_fwd_ns, t_bwd_ns,
-                   t_out_ns, t_in_ns)
+                   t_out_ns, t_in_ns, slack_ns)
     slots = (Slot1F1B * micro_batches)()
     summ = Summary1F1B()
     _check(lib.mpress_schedule_1f1b(byref(p), slots, byref(summ)))

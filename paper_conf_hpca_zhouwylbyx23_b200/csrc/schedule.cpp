@@ -147,7 +147,7 @@ extern "C" int mpress_schedule_1f1b(const mpress_1f1b_params* p, mpress_1f1b_slo
       int j = jf[m];
       for (int jj = jf[m]; jj < jb[m]; ++jj) {
         const uint64_t end = e0[node_of(base, e, jj)];
-        if (end + p->t_in_ns <= bs) j = jj;  // end <= bs - t_in without underflow
+        if (end + p->t_in_ns + p->t_slack_ns <= bs) j = jj;  // end <= bs - t_in - slack, no underflow
       }
       trig[m] = j;
     }

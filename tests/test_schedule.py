@@ -59,7 +59,9 @@ def test_library_matches_oracle_random():
         e = rng.randrange(S)
         args = (S, e, M, rng.randint(1, 50), rng.randint(1, 90), rng.randint(0, 120), rng.randint(0, 120))
         duplex = rng.random() < 0.5
-        assert mp.schedule_1f1b(*args, duplex=duplex) == P.schedule(*args, duplex=duplex), (args, duplex)
+        slack = rng.choice([0, 0, 5, 40])
+        assert mp.schedule_1f1b(*args, duplex=duplex, slack_ns=slack) == \
+            P.schedule(*args, duplex=duplex, slack=slack), (args, duplex, slack)
 
 
 def test_bert_stage0_scale():
