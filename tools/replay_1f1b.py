@@ -127,32 +127,39 @@ def replay(S, e, M, scale, n_fwd_gemms, max_ctas, seed=7000, slack=0.5):
                 synth_dev.gate(base, start_of[(kind, m)], comp)
                 if kind == "B" and with_swap:
                     ctx.wait(hs[m], comp)
+                b4 = torch.cuda.Event(enable_timing=True)
+                b4.record(comp)
                 (fwd if kind == "F" else bwd)()
-                x = torch.cuda.Event()
+                x = torch.cuda.Event(enable_timing=True)
                 x.record(comp)
-                ev.append(x)
+                ev.append((b4, x))
                 if not with_swap:
                     continue
                 if kind == "F":
-                    hs[m] = ctx.swap_out(pl, src[m], stream=s_out, after=x)
+                    hs[m] = ctx.swap_out(pl, src[m], stream=s_out, after=ev[-1][1])
                 for mm in range(M):
                     if sched[mm]["in_trigger"] == j:
-                        s_in.wait_event(x)
+                        s_in.wait_event(ev[-1][1])
                         ctx.swap_in(hs[mm], dst[mm], stream=s_in)
             t1 = torch.cuda.Event(enable_timing=True)
             t1.record(comp)
             torch.cuda.synchronize()
             for hh in hs.values():
                 hh.free()
-            return t0.elapsed_time(t1) * 1e6
+            compute = sum(a.elapsed_time(b) for a, b in ev) * 1e6
+            return t0.elapsed_time(t1) * 1e6, compute
 
         step(False)
         step(True)
-        no = statistics.median([step(False) for _ in range(3)])
+        runs = [step(False) for _ in range(3)]
+        no = statistics.median(r[0] for r in runs)
+        comp_no = statistics.median(r[1] for r in runs)
         for m in range(M):
             for t in dst[m]:
                 t.zero_()
-        yes = statistics.median([step(True) for _ in range(3)])
+        runs = [step(True) for _ in range(3)]
+        yes = statistics.median(r[0] for r in runs)
+        comp_yes = statistics.median(r[1] for r in runs)
         bad = sum(synth_dev.check(t, seed + m, i) for m in range(M) for i, t in enumerate(dst[m]))
         mb = sum(sizes)
         return {
@@ -168,6 +175,8 @@ def replay(S, e, M, scale, n_fwd_gemms, max_ctas, seed=7000, slack=0.5):
             "memory_saved_gib": (summ["peak_resident_noswap"] - summ["peak_resident"]) * mb / 2**30,
             "measured_stage_ms_noswap": no / 1e6, "measured_stage_ms_swap": yes / 1e6,
             "measured_overhead": yes / no - 1,
+            "compute_ms_noswap": comp_no / 1e6, "compute_ms_swap": comp_yes / 1e6,
+            "compute_slowdown": comp_yes / comp_no - 1,
             "restored_bytes_wrong": int(bad),
         }
     finally:
