@@ -194,6 +194,28 @@ MPRESS_API int mpress_plan_from_units(int world, int source, const uint64_t* uni
                                       uint32_t n_tensors, const uint64_t* tensor_bytes,
                                       uint64_t granule, mpress_plan_t** out);
 
+/*
+ * mpress_map_search -- NEXT-3: device-stage mapping search (Fig. 6 lines
+ * 10-26; reading R25).  Every mapping of the n
+ * pipeline stages onto the n GPUs is enumerated in lexicographic order of
+ * (gpu of stage 0, gpu of stage 1, ...); each is scored by the joint optimum
+ * of mpress_plan_global (the overflowed stages' demands on the light stages'
+ * spare, over the GPUs' links); the first mapping with the smallest swap
+ * time wins.  n! mappings: n <= 10.  On symmetric links every mapping scores
+ * the same and the paper skips the search.
+ *   demand [n] bytes each stage must swap out (0 = light stage)
+ *   spare  [n] spare bytes of each light stage (ignored for overflowed ones)
+ *   link   [n*n] link weights between GPUs (0 = not an NVLink neighbour)
+ *   egress / ingress [n] per-GPU port weights or NULL
+ *   stage_to_gpu [n] out; makespan_num / makespan_den / evaluated may be NULL.
+ * Errors: MPRESS_ERR_ARG, MPRESS_ERR_NO_SPACE (no mapping fits).
+ */
+MPRESS_API int mpress_map_search(int n, const uint64_t* demand, const uint64_t* spare,
+                                 const uint64_t* link, const uint64_t* egress,
+                                 const uint64_t* ingress, uint64_t granule, int32_t* stage_to_gpu,
+                                 uint64_t* makespan_num, uint64_t* makespan_den,
+                                 uint64_t* evaluated);
+
 /* ---- NEXT-2: 1F1B swap schedule with the live-interval check ------------------ */
 
 /* Inputs (all times in ns, integers).  Computation-balanced stages:

@@ -30,3 +30,4 @@ from .bytemodel import swap_out, swap_in, stash_sizes  # noqa: F401
 from .brute import brute_force_makespan, makespan  # noqa: F401
 from .partition import sequential_partition  # noqa: F401
 from .global_plan import brute_force_global, scan_global, assignment_time  # noqa: F401
+from .mapping import mapping_search  # noqa: F401

@@ -32,7 +32,8 @@ _ERR_NAMES = {ERR_ARG: "ERR_ARG", ERR_NO_SPACE: "ERR_NO_SPACE", ERR_ALIGN: "ERR_
 EXPORTED = [
     "mpress_plan", "mpress_plan_stripes", "mpress_plan_units", "mpress_plan_get_info",
     "mpress_plan_free", "mpress_partition_sequential", "mpress_plan_global",
-    "mpress_plan_from_units", "mpress_schedule_1f1b", "mpress_init", "mpress_init_local",
+    "mpress_plan_from_units", "mpress_schedule_1f1b", "mpress_map_search", "mpress_init",
+    "mpress_init_local",
     "mpress_finalize", "mpress_stash_free", "mpress_set_option", "mpress_get_option",
     "mpress_swap_out", "mpress_swap_in", "mpress_wait", "mpress_query", "mpress_handle_state",
     "mpress_handle_slices", "mpress_handle_free", "mpress_peer_read", "mpress_last_launches",
@@ -95,6 +96,8 @@ def _load():
                                        POINTER(c_uint64), POINTER(c_uint64)]),
         "mpress_plan_from_units": (c_int, [c_int, c_int, P, c_uint32, P, c_uint64, POINTER(P)]),
         "mpress_schedule_1f1b": (c_int, [POINTER(Params1F1B), P, P]),
+        "mpress_map_search": (c_int, [c_int, P, P, P, P, P, c_uint64, P, POINTER(c_uint64),
+                                      POINTER(c_uint64), POINTER(c_uint64)]),
         "mpress_init": (c_int, [c_int, c_int, c_int, P, EXCHANGE_FN, P, POINTER(P)]),
         "mpress_init_local": (c_int, [c_int, c_int, P, P, POINTER(P)]),
         "mpress_finalize": (c_int, [P]),
@@ -236,6 +239,17 @@ def schedule_1f1b(stages, stage, micro_batches, t_fwd_ns, t_bwd_ns, t_out_ns, t_
     names = [f[0] for f in Slot1F1B._fields_]
     return ([{n: getattr(s, n) for n in names} for s in slots],
             {f[0]: getattr(summ, f[0]) for f in Summary1F1B._fields_ if f[0] != "pad"})
+
+
+def map_search(demand, spare, link, egress=None, ingress=None, granule=0):
+    """NEXT-3 (mpress_map_search): (stage_to_gpu, (num, den), mappings evaluated)."""
+    n = len(demand)
+    out = (c_int32 * n)()
+    num, den, ev = c_uint64(), c_uint64(), c_uint64()
+    _check(lib.mpress_map_search(n, _u64(demand), _u64(spare), _u64([w for row in link for w in row]),
+                                 _u64(egress) if egress else None, _u64(ingress) if ingress else None,
+                                 granule, out, byref(num), byref(den), byref(ev)))
+    return list(out), (num.value, den.value), ev.value
 
 
 def plan_global(world, requests, spare, bw_matrix, egress=None, ingress=None, granule=0):

@@ -134,10 +134,113 @@ bool feasible(const Problem& P, uint64_t k, uint64_t w, std::vector<uint64_t>* x
   return true;
 }
 
+// T* = min over the model's weights w of (least k with feasible(k / w)) / w.
+// Returns false when no T places every unit (capacity).
+bool solve(const Problem& P, uint64_t* best_k, uint64_t* best_w) {
+  const int world = P.world;
+  u128 total = 0;
+  for (uint64_t k : P.K) total += k;
+  std::vector<uint64_t> weights;  // every usable link, egress and ingress port
+  for (int s : P.src)
+    for (int p = 0; p < world; ++p)
+      if (link(P, s, p)) weights.push_back(P.bw[(size_t)s * world + p]);
+  for (int s : P.src)
+    if (P.egress && P.egress[s] > 0) weights.push_back(P.egress[s]);
+  for (int p = 0; p < world; ++p)
+    if (P.ingress && P.ingress[p] > 0) weights.push_back(P.ingress[p]);
+  std::sort(weights.begin(), weights.end());
+  weights.erase(std::unique(weights.begin(), weights.end()), weights.end());
+  if (weights.empty() || !feasible(P, (uint64_t)total * weights.back() + 1, 1, nullptr)) return false;
+  *best_k = 0;
+  *best_w = 0;
+  for (uint64_t w : weights) {
+    // a smaller k/w than the best so far is all that matters: start there
+    uint64_t hi = *best_w ? (uint64_t)(((u128)*best_k * w) / *best_w) + 1 : (uint64_t)total;
+    if (*best_w && !feasible(P, hi, w, nullptr)) continue;  // cannot beat the best
+    uint64_t lo = 0;
+    while (!*best_w && !feasible(P, hi, w, nullptr)) {
+      if (hi > kInf / 2) { hi = 0; break; }
+      lo = hi;
+      hi *= 2;
+    }
+    if (hi == 0) continue;
+    while (hi - lo > 1) {  // invariant: lo infeasible (or 0), hi feasible
+      const uint64_t mid = lo + (hi - lo) / 2;
+      if (feasible(P, mid, w, nullptr)) hi = mid; else lo = mid;
+    }
+    if (*best_w == 0 || (u128)hi * *best_w < (u128)*best_k * w) {
+      *best_k = hi;
+      *best_w = w;
+    }
+  }
+  return *best_w != 0;
+}
+
 }  // namespace
 }  // namespace mpress
 
 using namespace mpress;
+
+extern "C" int mpress_map_search(int n, const uint64_t* demand, const uint64_t* spare, const uint64_t* link,
+                                 const uint64_t* egress, const uint64_t* ingress, uint64_t granule,
+                                 int32_t* stage_to_gpu, uint64_t* makespan_num, uint64_t* makespan_den,
+                                 uint64_t* evaluated) {
+  if (n < 1 || n > 10 || !demand || !spare || !link || !stage_to_gpu)
+    return fail(MPRESS_ERR_ARG, "mpress_map_search: bad argument (1 <= n <= 10)");
+  const uint64_t G = granule ? granule : MPRESS_DEFAULT_GRANULE;
+  if (G % MPRESS_ALIGN != 0) return fail(MPRESS_ERR_ARG, "mpress_map_search: granule not a multiple of 256");
+  std::vector<uint64_t> units(n, 0);
+  bool any = false;
+  for (int s = 0; s < n; ++s) {
+    if (demand[s] == 0) continue;
+    uint64_t V;
+    if (demand[s] > UINT64_MAX - 255) return fail(MPRESS_ERR_ARG, "mpress_map_search: demand too large");
+    V = roundup(demand[s], MPRESS_ALIGN);
+    units[s] = V / G + (V % G != 0);
+    any = true;
+  }
+  if (!any) return fail(MPRESS_ERR_ARG, "mpress_map_search: no stage overflows");
+  std::vector<int> perm(n);
+  for (int i = 0; i < n; ++i) perm[i] = i;
+  uint64_t best_k = 0, best_w = 0, count = 0;
+  std::vector<int> best_perm;
+  Problem P;
+  P.world = n;
+  P.bw = link;
+  P.egress = egress;
+  P.ingress = ingress;
+  try {
+    do {  // lexicographic order of (gpu of stage 0, gpu of stage 1, ...)
+      ++count;
+      P.src.clear();
+      P.K.clear();
+      P.cap.assign(n, 0);
+      for (int s = 0; s < n; ++s) {
+        if (demand[s] > 0) {
+          P.src.push_back(perm[s]);
+          P.K.push_back(units[s]);
+        } else {
+          P.cap[perm[s]] = spare[s] / G;
+        }
+      }
+      uint64_t k, w;
+      if (!solve(P, &k, &w)) continue;
+      if (best_w == 0 || (u128)k * best_w < (u128)best_k * w) {
+        best_k = k;
+        best_w = w;
+        best_perm = perm;
+      }
+    } while (std::next_permutation(perm.begin(), perm.end()));
+  } catch (const std::bad_alloc&) {
+    return fail(MPRESS_ERR_ARG, "mpress_map_search: out of host memory");
+  }
+  if (evaluated) *evaluated = count;
+  if (best_w == 0) return fail(MPRESS_ERR_NO_SPACE, "mpress_map_search: no mapping fits the demand");
+  for (int s = 0; s < n; ++s) stage_to_gpu[s] = best_perm[s];
+  if (makespan_num) *makespan_num = best_k;
+  if (makespan_den) *makespan_den = best_w;
+  return MPRESS_OK;
+}
 
 extern "C" int mpress_plan_global(int world, uint32_t n_sources, const int32_t* sources,
                                   const uint32_t* n_tensors, const uint64_t* sizes_flat,
@@ -177,37 +280,9 @@ extern "C" int mpress_plan_global(int world, uint32_t n_sources, const int32_t* 
     total += P.K.back();
   }
   if (total > kInf) return fail(MPRESS_ERR_ARG, "mpress_plan_global: too many units");
-  // weights of the model: every usable link, egress and ingress port
-  std::vector<uint64_t> weights;
-  for (int s : P.src)
-    for (int p = 0; p < world; ++p)
-      if (link(P, s, p)) weights.push_back(bw_matrix[(size_t)s * world + p]);
-  for (int s : P.src)
-    if (egress && egress[s] > 0) weights.push_back(egress[s]);
-  for (int p = 0; p < world; ++p)
-    if (ingress && ingress[p] > 0) weights.push_back(ingress[p]);
-  std::sort(weights.begin(), weights.end());
-  weights.erase(std::unique(weights.begin(), weights.end()), weights.end());
-  if (weights.empty() || !feasible(P, (uint64_t)total * weights.back() + 1, 1, nullptr))
-    return fail(MPRESS_ERR_NO_SPACE, "mpress_plan_global: the importers' spare memory cannot hold all batches");
-  // T* = min over weights w of (least k with feasible(k / w)) / w
   uint64_t best_k = 0, best_w = 0;
-  for (uint64_t w : weights) {
-    uint64_t lo = 0, hi = (uint64_t)total;  // feasible(hi / w)?  extend if not
-    while (!feasible(P, hi, w, nullptr)) {
-      if (hi > kInf / 2) { hi = 0; break; }
-      hi *= 2;
-    }
-    if (hi == 0) continue;
-    while (hi - lo > 1) {  // invariant: lo infeasible (or 0), hi feasible
-      const uint64_t mid = lo + (hi - lo) / 2;
-      if (feasible(P, mid, w, nullptr)) hi = mid; else lo = mid;
-    }
-    if (best_w == 0 || (u128)hi * best_w < (u128)best_k * w) {
-      best_k = hi;
-      best_w = w;
-    }
-  }
+  if (!solve(P, &best_k, &best_w))
+    return fail(MPRESS_ERR_NO_SPACE, "mpress_plan_global: the importers' spare memory cannot hold all batches");
   std::vector<uint64_t> x;
   feasible(P, best_k, best_w, &x);
   for (size_t i = 0; i < (size_t)n_sources * world; ++i) units_out[i] = x[i];
