@@ -244,8 +244,11 @@ def main():
     device = local_rank % ngpu
     torch.cuda.set_device(device)
     if n > 1:
-        shared = int(os.environ.get("LOCAL_WORLD_SIZE", n)) > ngpu
-        dist.init_process_group("gloo" if shared else "cpu:gloo,cuda:nccl")
+        # The swap path has no collective: the process group
+        # only carries the init-time all-gathers and the CPU-side max-over-
+        # ranks reductions, so gloo serves every layout (also ranks sharing
+        # a GPU in the 1-GPU test of this path).
+        dist.init_process_group("gloo")
     local_rank = device
 
     import paper_conf_hpca_zhouwylbyx23_b200 as mp
