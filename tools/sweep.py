@@ -92,9 +92,28 @@ def sizes_sweep():
                 ctx.set_option(mp.OPT_PATH, PATHS[name])
                 reps = 20 if size < (256 << 20) else 5
                 to, ti = time_swaps(ctx, pl, src, dst, reps, s)
+                # back to back: R swap pairs enqueued while the GPU is busy, so
+                # host enqueue time hides behind the previous pair
+                R = 50 if size < (64 << 20) else 4
+                torch.cuda.synchronize()
+                warm = ctx.swap_out(pl, src, stream=s)   # keeps the GPU busy first
+                ctx.swap_in(warm, dst, stream=s)
+                e0 = torch.cuda.Event(enable_timing=True)
+                e1 = torch.cuda.Event(enable_timing=True)
+                e0.record(s)
+                for _ in range(R):
+                    h = ctx.swap_out(pl, src, stream=s)
+                    ctx.swap_in(h, dst, stream=s)
+                    h.free()
+                e1.record(s)
+                torch.cuda.synchronize()
+                warm.free()
+                pair_us = e0.elapsed_time(e1) * 1e3 / R
                 print(json.dumps({"sweep": "sizes", "peers": peers_n, "bytes": size, "path": name,
                                   "out_gbs": size / to / 1e6, "in_gbs": size / ti / 1e6,
-                                  "out_us": to * 1e3, "in_us": ti * 1e3}), flush=True)
+                                  "out_us": to * 1e3, "in_us": ti * 1e3,
+                                  "b2b_pair_us": pair_us,
+                                  "b2b_gbs": 2 * size / pair_us / 1e3}), flush=True)
             ctx.finalize()
             del src, dst
             torch.cuda.empty_cache()
