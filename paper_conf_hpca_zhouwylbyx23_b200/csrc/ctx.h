@@ -4,12 +4,15 @@
 #include <cuda.h>
 #include <cuda_runtime.h>
 
+#include <deque>
 #include <map>
+#include <memory>
 #include <mutex>
 #include <set>
 #include <vector>
 
 #include "common.h"
+#include "swap_kernels.h"
 
 namespace mpress {
 
@@ -54,10 +57,15 @@ struct Mapping {
   bool reserved = false, mapped = false, has_handle = false;
 };
 
+// A CUDA event shared by a handle and the fences its swap-in leaves behind;
+// it returns to the context's pool when the last owner releases it.
+using EvRef = std::shared_ptr<CUevent_st>;
+using EvPool = std::shared_ptr<std::vector<cudaEvent_t>>;
+
 // A released slice whose bytes a pending swap-in may still be reading.
 struct Fence {
   uint64_t off, len;
-  cudaEvent_t ev;
+  EvRef ev;
 };
 
 // This source's partition of one peer's stash pool (R21).
@@ -65,7 +73,7 @@ struct Partition {
   uint8_t* base = nullptr;            // local VA of the partition start
   uint64_t size = 0;
   std::map<uint64_t, uint64_t> free;  // first-fit free list: offset -> length
-  std::vector<Fence> fences;
+  std::deque<Fence> fences;           // in release order (oldest first)
 };
 
 }  // namespace mpress
@@ -89,8 +97,10 @@ struct mpress_ctx_s {
   int order = MPRESS_ORDER_INTERLEAVE;
   int last_launches = 0;
   std::vector<cudaStream_t> ce_streams;  // copy-engine comparator, one per peer
-  std::vector<cudaEvent_t> ev_pool;
+  mpress::EvPool ev_pool = std::make_shared<std::vector<cudaEvent_t>>();
   std::set<mpress_handle_s*> handles;
+  std::vector<mpress::CopyDesc> scratch_desc;  // per-call buffers, reused
+  std::vector<int> scratch_peer;
   std::mutex mu;
 };
 
@@ -98,10 +108,10 @@ struct mpress_handle_s {
   mpress_ctx_s* ctx = nullptr;
   int state = 0;
   std::vector<mpress_stripe> stripes;
-  std::vector<uint64_t> sizes;
+  uint32_t n_tensors = 0;
   std::vector<uint64_t> slice_off;    // [world], UINT64_MAX if unused
   std::vector<uint64_t> slice_len;    // [world]
-  cudaEvent_t out_done = nullptr;
-  cudaEvent_t in_done = nullptr;
+  mpress::EvRef out_done;
+  mpress::EvRef in_done;
   bool slices_held = false;
 };

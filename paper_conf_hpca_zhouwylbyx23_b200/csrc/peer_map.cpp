@@ -116,14 +116,10 @@ void destroy(mpress_ctx_s* c) {
     for (auto& m : c->maps) unmap(d, &m);
     unmap(d, &c->own);
   }
-  for (auto* h : c->handles) {
-    if (h->out_done) cudaEventDestroy(h->out_done);
-    if (h->in_done) cudaEventDestroy(h->in_done);
-    delete h;
-  }
-  for (auto& p : c->parts)
-    for (auto& f : p.fences) cudaEventDestroy(f.ev);
-  for (auto e : c->ev_pool) cudaEventDestroy(e);
+  for (auto* h : c->handles) delete h;   // their events go back to the pool
+  for (auto& p : c->parts) p.fences.clear();
+  for (auto e : *c->ev_pool) cudaEventDestroy(e);
+  c->ev_pool->clear();
   for (auto s : c->ce_streams) if (s) cudaStreamDestroy(s);
   delete c;
 }
@@ -195,6 +191,11 @@ extern "C" int mpress_init_local(int world, int source, const int* devices,
       return rc;
     }
     init_partition(&c->parts[p], reinterpret_cast<uint8_t*>(c->maps[p].va), want);
+  }
+  const int rc = preload_kernels();
+  if (rc != MPRESS_OK) {
+    destroy(c);
+    return rc;
   }
   *out = c;
   return MPRESS_OK;
@@ -277,6 +278,7 @@ extern "C" int mpress_init(int device, int world, int rank, const uint64_t* part
     if (fds[p] >= 0) close(fds[p]);
 
   // 4. agree on success
+  if (rc == MPRESS_OK) rc = preload_kernels();
   int32_t ok = rc == MPRESS_OK;
   std::vector<int32_t> okv(world);
   if (exchange(exchange_user, &ok, sizeof ok, okv.data()) != 0 && rc == MPRESS_OK)

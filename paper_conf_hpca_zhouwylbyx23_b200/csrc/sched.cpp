@@ -11,6 +11,11 @@
 // events carry completion: every call only enqueues work, and
 // mpress_wait / mpress_query are enqueue-only / non-blocking, so no helper
 // thread is needed.
+//
+// Host cost per call is kept small (a swap of a few KiB is latency-bound by
+// the host): events are pooled and shared by reference between a handle and
+// the fences of its slices, fences are reaped oldest-first, and descriptor
+// buffers are reused.
 #include <algorithm>
 #include <cstring>
 
@@ -20,31 +25,30 @@
 namespace mpress {
 namespace {
 
-cudaEvent_t take_event(mpress_ctx_s* c) {
-  if (!c->ev_pool.empty()) {
-    cudaEvent_t e = c->ev_pool.back();
-    c->ev_pool.pop_back();
-    return e;
-  }
+EvRef take_event(mpress_ctx_s* c) {
   cudaEvent_t e = nullptr;
-  if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) return nullptr;
-  return e;
-}
-
-void give_event(mpress_ctx_s* c, cudaEvent_t e) {
-  if (e) c->ev_pool.push_back(e);
-}
-
-// Drop fences whose swap-in has completed.
-void reap_fences(mpress_ctx_s* c, Partition* part) {
-  auto& f = part->fences;
-  size_t w = 0;
-  for (size_t r = 0; r < f.size(); ++r) {
-    if (cudaEventQuery(f[r].ev) == cudaSuccess) give_event(c, f[r].ev);
-    else f[w++] = f[r];
+  EvPool pool = c->ev_pool;
+  if (!pool->empty()) {
+    e = pool->back();
+    pool->pop_back();
+  } else if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) {
+    return EvRef();
   }
-  f.resize(w);
-  cudaGetLastError();  // cudaEventQuery's cudaErrorNotReady is not sticky; clear it
+  return EvRef(e, [pool](CUevent_st* ev) { pool->push_back(ev); });
+}
+
+// Drop the fences whose swap-in has completed (oldest first; stops at the
+// first one still pending, so the cost is O(1) amortised).
+void reap_fences(Partition* part) {
+  auto& f = part->fences;
+  while (!f.empty()) {
+    const cudaError_t r = cudaEventQuery(f.front().ev.get());
+    if (r != cudaSuccess) {
+      if (r == cudaErrorNotReady) cudaGetLastError();  // not sticky; clear it
+      break;
+    }
+    f.pop_front();
+  }
 }
 
 // First fit, lowest address.
@@ -97,8 +101,8 @@ int run_copy(mpress_ctx_s* c, int dir, const std::vector<CopyDesc>& d,
   c->last_launches = 0;
   if (c->path != MPRESS_PATH_CE)
     return launch_copy(c->path, c->variant, dir, d.data(),
-                       c->order == MPRESS_ORDER_INTERLEAVE ? desc_peer.data() : nullptr, d.size(), c->max_ctas, stream,
-                       &c->last_launches);
+                       c->order == MPRESS_ORDER_INTERLEAVE ? desc_peer.data() : nullptr, d.size(), c->max_ctas,
+                       stream, &c->last_launches);
 
   // Copy-engine comparator: cudaMemcpyAsync per stripe, one side stream per
   // peer so the engines of different peers overlap; fork/join by events.
@@ -109,31 +113,26 @@ int run_copy(mpress_ctx_s* c, int dir, const std::vector<CopyDesc>& d,
       if (e != cudaSuccess) return cuda_fail(e, "cudaStreamCreate (copy-engine path)");
     }
   }
-  cudaEvent_t fork = take_event(c);
+  EvRef fork = take_event(c);
   if (!fork) return fail(MPRESS_ERR_CUDA, "cudaEventCreate failed");
-  cudaEventRecord(fork, stream);
+  cudaEventRecord(fork.get(), stream);
   std::vector<char> used(c->world, 0);
   for (int p : desc_peer) used[p] = 1;
-  int rc = MPRESS_OK;
-  std::vector<cudaEvent_t> joins;
-  for (int p = 0; p < c->world && rc == MPRESS_OK; ++p) {
+  for (int p = 0; p < c->world; ++p) {
     if (!used[p]) continue;
     cudaStream_t s = c->ce_streams[p];
-    cudaStreamWaitEvent(s, fork, 0);
+    cudaStreamWaitEvent(s, fork.get(), 0);
     for (size_t i = 0; i < d.size(); ++i) {
       if (desc_peer[i] != p) continue;
       cudaError_t e = cudaMemcpyAsync(d[i].dst, d[i].src, d[i].len, cudaMemcpyDefault, s);
-      if (e != cudaSuccess) { rc = cuda_fail(e, "cudaMemcpyAsync (copy-engine path)"); break; }
+      if (e != cudaSuccess) return cuda_fail(e, "cudaMemcpyAsync (copy-engine path)");
     }
-    cudaEvent_t j = take_event(c);
-    cudaEventRecord(j, s);
-    cudaStreamWaitEvent(stream, j, 0);
-    joins.push_back(j);
-  }
-  // Events may be re-recorded once the waits above are enqueued.
-  give_event(c, fork);
-  for (auto j : joins) give_event(c, j);
-  return rc;
+    EvRef join = take_event(c);
+    if (!join) return fail(MPRESS_ERR_CUDA, "cudaEventCreate failed");
+    cudaEventRecord(join.get(), s);
+    cudaStreamWaitEvent(stream, join.get(), 0);
+  }  // the events may be re-recorded once the waits above are enqueued
+  return MPRESS_OK;
 }
 
 }  // namespace
@@ -164,7 +163,6 @@ extern "C" int mpress_swap_out(mpress_ctx_t* c, const mpress_plan_t* plan_, void
   h->ctx = c;
   h->slice_off.assign(c->world, UINT64_MAX);
   h->slice_len.assign(c->world, 0);
-  std::vector<cudaEvent_t> waits;
   int rc = MPRESS_OK;
   for (int p = 0; p < c->world && rc == MPRESS_OK; ++p) {
     if (units[p] == 0) continue;
@@ -173,7 +171,7 @@ extern "C" int mpress_swap_out(mpress_ctx_t* c, const mpress_plan_t* plan_, void
       rc = fail(MPRESS_ERR_PEER, "mpress_swap_out: peer %d is not mapped (partition 0)", p);
       break;
     }
-    reap_fences(c, &part);
+    reap_fences(&part);
     const uint64_t len = units[p] * info.granule;
     uint64_t off;
     if (!alloc_slice(&part, len, &off)) {
@@ -183,8 +181,9 @@ extern "C" int mpress_swap_out(mpress_ctx_t* c, const mpress_plan_t* plan_, void
     }
     h->slice_off[p] = off;
     h->slice_len[p] = len;
-    for (auto& f : part.fences)  // earlier swap-ins still reading these bytes
-      if (f.off < off + len && off < f.off + f.len) waits.push_back(f.ev);
+    // earlier swap-ins still reading these bytes: order this swap-out after them
+    for (const Fence& f : part.fences)
+      if (f.off < off + len && off < f.off + f.len) cudaStreamWaitEvent(stream, f.ev.get(), 0);
   }
   if (rc != MPRESS_OK) {
     for (int p = 0; p < c->world; ++p)
@@ -194,10 +193,12 @@ extern "C" int mpress_swap_out(mpress_ctx_t* c, const mpress_plan_t* plan_, void
   }
   h->slices_held = true;
   h->stripes.assign(st, st + n_st);
-  h->sizes.resize(info.n_tensors);
+  h->n_tensors = info.n_tensors;
 
-  std::vector<CopyDesc> d(n_st);
-  std::vector<int> dp(n_st);
+  std::vector<CopyDesc>& d = c->scratch_desc;
+  std::vector<int>& dp = c->scratch_peer;
+  d.resize(n_st);
+  dp.resize(n_st);
   for (uint32_t i = 0; i < n_st; ++i) {
     const mpress_stripe& s = st[i];
     d[i].src = static_cast<const uint8_t*>(tensors[s.tensor]) + s.src_off;
@@ -205,12 +206,11 @@ extern "C" int mpress_swap_out(mpress_ctx_t* c, const mpress_plan_t* plan_, void
     d[i].len = s.len;
     dp[i] = (int)s.peer;
   }
-  for (auto e : waits) cudaStreamWaitEvent(stream, e, 0);
   if (after) cudaStreamWaitEvent(stream, static_cast<cudaEvent_t>(after), 0);
   h->out_done = take_event(c);
   rc = h->out_done ? run_copy(c, kDirOut, d, dp, stream) : fail(MPRESS_ERR_CUDA, "cudaEventCreate failed");
   if (rc == MPRESS_OK) {
-    cudaError_t e = cudaEventRecord(h->out_done, stream);
+    cudaError_t e = cudaEventRecord(h->out_done.get(), stream);
     if (e != cudaSuccess) rc = cuda_fail(e, "cudaEventRecord(out_done)");
   }
   if (rc != MPRESS_OK) {
@@ -218,7 +218,6 @@ extern "C" int mpress_swap_out(mpress_ctx_t* c, const mpress_plan_t* plan_, void
     cudaStreamSynchronize(stream);
     for (int p = 0; p < c->world; ++p)
       if (h->slice_off[p] != UINT64_MAX) free_slice(&c->parts[p], h->slice_off[p], h->slice_len[p]);
-    give_event(c, h->out_done);
     delete h;
     return rc;
   }
@@ -234,12 +233,14 @@ extern "C" int mpress_swap_in(mpress_ctx_t* c, mpress_handle_t* h, void* const* 
   if (h->ctx != c || !c->handles.count(h)) return fail(MPRESS_ERR_ARG, "mpress_swap_in: handle not of this context");
   if (h->state != MPRESS_STATE_OUT_PENDING && h->state != MPRESS_STATE_OUT)
     return fail(MPRESS_ERR_STATE, "mpress_swap_in: handle is in state %d, not swapped out", h->state);
-  MP_TRY(check_ptrs(dst, h->sizes.size(), "mpress_swap_in(dst)"));
+  MP_TRY(check_ptrs(dst, h->n_tensors, "mpress_swap_in(dst)"));
   DeviceGuard g(c->device);
   cudaStream_t stream = static_cast<cudaStream_t>(stream_);
 
-  std::vector<CopyDesc> d(h->stripes.size());
-  std::vector<int> dp(h->stripes.size());
+  std::vector<CopyDesc>& d = c->scratch_desc;
+  std::vector<int>& dp = c->scratch_peer;
+  d.resize(h->stripes.size());
+  dp.resize(h->stripes.size());
   for (size_t i = 0; i < h->stripes.size(); ++i) {
     const mpress_stripe& s = h->stripes[i];
     d[i].src = c->parts[s.peer].base + h->slice_off[s.peer] + s.dst_off;
@@ -247,26 +248,21 @@ extern "C" int mpress_swap_in(mpress_ctx_t* c, mpress_handle_t* h, void* const* 
     d[i].len = s.len;
     dp[i] = (int)s.peer;
   }
-  cudaStreamWaitEvent(stream, h->out_done, 0);
-  if (!h->in_done) h->in_done = take_event(c);
-  if (!h->in_done) return fail(MPRESS_ERR_CUDA, "cudaEventCreate failed");
+  cudaStreamWaitEvent(stream, h->out_done.get(), 0);
+  EvRef in_done = take_event(c);
+  if (!in_done) return fail(MPRESS_ERR_CUDA, "cudaEventCreate failed");
   int rc = run_copy(c, kDirIn, d, dp, stream);
   if (rc != MPRESS_OK) return rc;
-  cudaError_t e = cudaEventRecord(h->in_done, stream);
+  cudaError_t e = cudaEventRecord(in_done.get(), stream);
   if (e != cudaSuccess) return cuda_fail(e, "cudaEventRecord(in_done)");
+  h->in_done = in_done;
   h->state = MPRESS_STATE_IN_PENDING;
 
-  // Release the slices now; bytes stay fenced until this swap-in completes
-  // (the table entry is "updated when it completes").
+  // Release the slices now; their bytes stay fenced by the swap-in's event
+  // until it completes (the table entry is "updated when it completes").
   for (int p = 0; p < c->world; ++p) {
     if (h->slice_off[p] == UINT64_MAX) continue;
-    cudaEvent_t f = take_event(c);
-    if (!f || cudaEventRecord(f, stream) != cudaSuccess) {
-      cudaStreamSynchronize(stream);  // cannot fence: wait instead
-      give_event(c, f);
-    } else {
-      c->parts[p].fences.push_back({h->slice_off[p], h->slice_len[p], f});
-    }
+    c->parts[p].fences.push_back({h->slice_off[p], h->slice_len[p], in_done});
     free_slice(&c->parts[p], h->slice_off[p], h->slice_len[p]);
   }
   h->slices_held = false;
@@ -276,9 +272,9 @@ extern "C" int mpress_swap_in(mpress_ctx_t* c, mpress_handle_t* h, void* const* 
 extern "C" int mpress_wait(mpress_ctx_t* c, mpress_handle_t* h, void* consumer) {
   if (!c || !h || h->ctx != c) return fail(MPRESS_ERR_ARG, "mpress_wait: bad argument");
   DeviceGuard g(c->device);
-  cudaEvent_t e = (h->state == MPRESS_STATE_IN_PENDING || h->state == MPRESS_STATE_IN) ? h->in_done : h->out_done;
+  const EvRef& e = (h->state == MPRESS_STATE_IN_PENDING || h->state == MPRESS_STATE_IN) ? h->in_done : h->out_done;
   if (!e) return fail(MPRESS_ERR_STATE, "mpress_wait: nothing enqueued");
-  cudaError_t r = cudaStreamWaitEvent(static_cast<cudaStream_t>(consumer), e, 0);
+  cudaError_t r = cudaStreamWaitEvent(static_cast<cudaStream_t>(consumer), e.get(), 0);
   if (r != cudaSuccess) return cuda_fail(r, "mpress_wait: cudaStreamWaitEvent");
   return MPRESS_OK;
 }
@@ -290,8 +286,8 @@ extern "C" int mpress_query(mpress_ctx_t* c, mpress_handle_t* h) {
   int next;
   switch (h->state) {
     case MPRESS_STATE_OUT: case MPRESS_STATE_IN: return 1;
-    case MPRESS_STATE_OUT_PENDING: e = h->out_done; next = MPRESS_STATE_OUT; break;
-    case MPRESS_STATE_IN_PENDING: e = h->in_done; next = MPRESS_STATE_IN; break;
+    case MPRESS_STATE_OUT_PENDING: e = h->out_done.get(); next = MPRESS_STATE_OUT; break;
+    case MPRESS_STATE_IN_PENDING: e = h->in_done.get(); next = MPRESS_STATE_IN; break;
     default: return fail(MPRESS_ERR_STATE, "mpress_query: bad state %d", h->state);
   }
   cudaError_t r = cudaEventQuery(e);
@@ -316,16 +312,11 @@ extern "C" int mpress_handle_free(mpress_ctx_t* c, mpress_handle_t* h, int force
   if (h->slices_held) {
     if (!force)
       return fail(MPRESS_ERR_STATE, "mpress_handle_free: data still only in the stash (state %d); swap in or force", h->state);
-    cudaEventSynchronize(h->out_done);  // swap-out kernels may still write the slices
+    cudaEventSynchronize(h->out_done.get());  // swap-out kernels may still write the slices
     for (int p = 0; p < c->world; ++p)
       if (h->slice_off[p] != UINT64_MAX) free_slice(&c->parts[p], h->slice_off[p], h->slice_len[p]);
   }
-  // An IN_PENDING handle's slices are covered by fences with their own events;
-  // its events go back to the pool only once they can no longer be waited on
-  // by this handle (it is being destroyed), and re-recording them later is
-  // ordered after everything already enqueued.
-  give_event(c, h->out_done);
-  give_event(c, h->in_done);
+  // An IN_PENDING handle's slices stay fenced: the fences share its event.
   c->handles.erase(h);
   delete h;
   return MPRESS_OK;

@@ -444,6 +444,34 @@ int copy_wave_ctas(int path, int variant) {
   return w;
 }
 
+namespace {
+template <int CAP>
+int preload_cap() {
+  for (int path : {MPRESS_PATH_DIRECT, MPRESS_PATH_BULK}) {
+    const int nvar = path == MPRESS_PATH_BULK ? kBulkVariants : kDirectVariants;
+    for (int v = 0; v < nvar; ++v)
+      for (int dir : {kDirOut, kDirIn})
+        for (bool pf : {false, true}) {
+          cudaFuncAttributes a;
+          KernelFn<CAP> k = kernel_for<CAP>(path, v, dir, pf);
+          if (cudaFuncGetAttributes(&a, (const void*)k) != cudaSuccess)
+            return fail(MPRESS_ERR_CUDA, "cannot load the swap kernels");
+          MP_TRY(prepare<CAP>(k, shape_of(path, v)));
+        }
+  }
+  return MPRESS_OK;
+}
+}  // namespace
+
+// With lazy module loading (the CUDA 12 default) a kernel's first launch may
+// wait for the whole device; loading every swap kernel at context creation
+// keeps that stall out of the training step.
+int preload_kernels() {
+  MP_TRY(preload_cap<16>());
+  MP_TRY(preload_cap<128>());
+  return preload_cap<kMaxDescPerLaunch>();
+}
+
 int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* group, size_t n,
                 int max_ctas, cudaStream_t stream, int* launches) {
   int dev = 0, sms = 0;

@@ -34,4 +34,7 @@ int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* gr
 // Default grid of a path/variant on the current device (SMs x CTAs per SM).
 int copy_wave_ctas(int path, int variant);
 
+// Load every swap kernel on the current device (no lazy-loading stall later).
+int preload_kernels();
+
 }  // namespace mpress
