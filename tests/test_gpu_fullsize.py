@@ -36,6 +36,9 @@ def _sampled_roundtrip(world, source, spare, bw, sizes, seed, samples=64):
             t = torch.empty(n, dtype=torch.uint8, device="cuda")
             synth_dev.fill(t, seed, i)
             src.append(t)
+        # the fills run on the current stream; the swap stream does not wait
+        # for it on its own (non-blocking streams)
+        torch.cuda.synchronize()
         s = torch.cuda.Stream()
         h = ctx.swap_out(pl, src, stream=s)
         s.synchronize()

@@ -19,6 +19,7 @@ def run(world, spare, bw, sizes, seed, reads=True):
         t = torch.empty(n, dtype=torch.uint8, device="cuda")
         synth_dev.fill(t, seed, i)
         src.append(t)
+    torch.cuda.synchronize()   # fills ran on the current stream
     s = torch.cuda.Stream()
     h = ctx.swap_out(pl, src, stream=s)
     s.synchronize()
