@@ -262,7 +262,16 @@ extern "C" int mpress_swap_in(mpress_ctx_t* c, mpress_handle_t* h, void* const* 
   // until it completes (the table entry is "updated when it completes").
   for (int p = 0; p < c->world; ++p) {
     if (h->slice_off[p] == UINT64_MAX) continue;
-    c->parts[p].fences.push_back({h->slice_off[p], h->slice_len[p], in_done});
+    // Older fences inside this slice are dominated: this handle's swap-out
+    // waited on every fence overlapping the slice (none can appear while the
+    // slice is held), so the new event completes after them.
+    auto& fs = c->parts[p].fences;
+    const uint64_t a = h->slice_off[p], b = a + h->slice_len[p];
+    for (auto it = fs.begin(); it != fs.end();) {
+      if (it->off >= a && it->off + it->len <= b) it = fs.erase(it);
+      else ++it;
+    }
+    fs.push_back({h->slice_off[p], h->slice_len[p], in_done});
     free_slice(&c->parts[p], h->slice_off[p], h->slice_len[p]);
   }
   h->slices_held = false;
