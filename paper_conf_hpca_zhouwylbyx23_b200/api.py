@@ -144,6 +144,18 @@ def _ptr(x):
     return int(x)
 
 
+def pointers(tensors):
+    """A reusable C array of the tensors' device addresses (marshal once,
+    pass to swap_out / swap_in many times; the tensors must stay alive)."""
+    return (c_void_p * len(tensors))(*[_ptr(t) for t in tensors])
+
+
+def _ptr_array(x):
+    if isinstance(x, ctypes.Array):
+        return x
+    return pointers(x)
+
+
 def _stream(s, device=None):
     if s is None:
         import torch
@@ -384,15 +396,15 @@ class Context:
         return list(out)
 
     def swap_out(self, plan_, tensors, stream=None, after=None):
-        ptrs = (c_void_p * len(tensors))(*[_ptr(t) for t in tensors])
+        """tensors: a list of tensors / addresses, or a `pointers(...)` array
+        built once and reused (saves the per-call marshalling)."""
         h = c_void_p()
-        _check(lib.mpress_swap_out(self._h, plan_.handle, ptrs, _stream(stream, self.device),
-                                   _event(after), byref(h)))
+        _check(lib.mpress_swap_out(self._h, plan_.handle, _ptr_array(tensors),
+                                   _stream(stream, self.device), _event(after), byref(h)))
         return Handle(self, h, plan_)
 
     def swap_in(self, handle, dst, stream=None):
-        ptrs = (c_void_p * len(dst))(*[_ptr(t) for t in dst])
-        _check(lib.mpress_swap_in(self._h, handle._h, ptrs, _stream(stream, self.device)))
+        _check(lib.mpress_swap_in(self._h, handle._h, _ptr_array(dst), _stream(stream, self.device)))
 
     def wait(self, handle, stream=None):
         _check(lib.mpress_wait(self._h, handle._h, _stream(stream, self.device)))

@@ -53,12 +53,14 @@ constexpr int kMaxGroups = 64;  // peers per launch (NVSwitch domains up to 64 G
 // 28 KB parameter block with its launch (launch latency grows with it).
 template <int CAP>
 struct CopyTable {
+  // every group holds >= 1 descriptor, so a table needs <= CAP groups
+  static constexpr int kGroups = CAP < kMaxGroups ? CAP : kMaxGroups;
   uint32_t n;                        // descriptors
   uint32_t n_groups;                 // runs of descriptors with the same peer
   uint32_t rounds_log2;              // R = 2^rounds_log2 >= chunks of the largest group
   uint32_t pad;
-  uint32_t g_chunk[kMaxGroups + 1];  // first chunk of each group (prefix)
-  uint32_t g_desc[kMaxGroups + 1];   // first descriptor of each group (prefix)
+  uint32_t g_chunk[kGroups + 1];     // first chunk of each group (prefix)
+  uint32_t g_desc[kGroups + 1];      // first descriptor of each group (prefix)
   uint32_t first_chunk[CAP + 1];     // first chunk of each descriptor (prefix)
   CopyDesc d[CAP];
 };
@@ -393,7 +395,7 @@ int launch_batch(int path, int variant, int dir, const CopyDesc* d, const int* g
   uint32_t ng = 0;
   for (uint32_t i = 0; i < n; ++i) {
     if (i == 0 || (gid && gid[i] != gid[i - 1])) {
-      if (ng == (uint32_t)kMaxGroups) return fail(MPRESS_ERR_ARG, "more than %d peers in one swap", kMaxGroups);
+      if (ng == (uint32_t)CopyTable<CAP>::kGroups) return fail(MPRESS_ERR_ARG, "more than %d peers in one swap", CopyTable<CAP>::kGroups);
       t.g_desc[ng] = i;
       t.g_chunk[ng++] = (uint32_t)chunks;
     }
