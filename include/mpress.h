@@ -216,6 +216,41 @@ MPRESS_API int mpress_map_search(int n, const uint64_t* demand, const uint64_t* 
                                  uint64_t* makespan_num, uint64_t* makespan_den,
                                  uint64_t* evaluated);
 
+/* ---- NEXT-4: memory-compaction decision rule (§III-D) ---------------------------- */
+
+/* Cost statistics of one tensor (Table III; all times ns). */
+typedef struct mpress_tensor_stat {
+  uint64_t bytes;
+  uint64_t live_ns;       /* live interval (P:226 fn.1)                        */
+  uint64_t recompute_ns;  /* extra forward time; MPRESS_NOT_RECOMPUTABLE for
+                             non-activations (optimizer states, gradients)     */
+  uint64_t cpu_swap_ns;   /* GPU-CPU swap out + in over PCIe                   */
+  uint64_t d2d_swap_ns;   /* D2D swap out + in over NVLink                     */
+} mpress_tensor_stat;
+
+#define MPRESS_NOT_RECOMPUTABLE  UINT64_MAX
+#define MPRESS_CHOICE_CPU_SWAP   1u
+#define MPRESS_CHOICE_RECOMPUTE  2u
+#define MPRESS_CHOICE_D2D        3u
+
+/*
+ * mpress_compaction_plan -- NEXT-4: which optimization frees each tensor
+ * (§III-D; reading R26).  A swap costs max(0, cost - live
+ * interval) (fn.2 P:238), recomputation its forward time; the initial
+ * assignment is the cheaper of GPU-CPU swap and recomputation (ties -> swap,
+ * P:224-228); then tensors in order of decreasing overhead move to D2D swap
+ * when it is strictly cheaper and they fit in the remaining d2d_capacity bytes
+ * (P:229-232); ties keep the option that spends no spare GPU memory
+ * (Table III discussion).
+ *   choice [n] out (MPRESS_CHOICE_*); overhead_ns [n] out or NULL;
+ *   total_overhead_ns out; d2d_bytes out or NULL.
+ * Errors: MPRESS_ERR_ARG.
+ */
+MPRESS_API int mpress_compaction_plan(uint32_t n, const mpress_tensor_stat* stats,
+                                      uint64_t d2d_capacity, uint32_t* choice,
+                                      uint64_t* overhead_ns, uint64_t* total_overhead_ns,
+                                      uint64_t* d2d_bytes);
+
 /* ---- NEXT-2: 1F1B swap schedule with the live-interval check ------------------ */
 
 /* Inputs (all times in ns, integers).  Computation-balanced stages:
@@ -302,7 +337,13 @@ MPRESS_API int mpress_init(int device, int world, int rank, const uint64_t* part
  * bytes).  With every devices[p] equal it is the 1-GPU "loopback" mode: the
  * peers are disjoint VMM pools of the same GPU, so the whole data path
  * (planner, mapping, kernels, scheduler) runs with HBM standing in for NVLink.
+ * devices[p] == MPRESS_DEVICE_HOST makes peer p a pinned host pool (NEXT-4,
+ * the GPU-CPU swap tier of P:105/P:145/P:236): the same plan, kernels and
+ * events move the bytes over PCIe; give it a link weight in proportion to
+ * PCIe bandwidth and the planner stripes between NVLink peers and the host
+ * (P:153).  devices[source] must be a GPU.
  */
+#define MPRESS_DEVICE_HOST (-1)
 MPRESS_API int mpress_init_local(int world, int source, const int* devices,
                       const uint64_t* partition, mpress_ctx_t** out);
 

@@ -21,6 +21,7 @@ ALIGN = 256
 DEFAULT_GRANULE = 65536
 OPT_PATH, OPT_MAX_CTAS, OPT_VARIANT, OPT_ORDER = 1, 2, 3, 4
 ORDER_INTERLEAVE, ORDER_PLAN = 0, 1
+DEVICE_HOST = -1   # mpress_init_local: a pinned host pool as a peer (NEXT-4)
 VARIANT_AUTO = -1
 PATH_DIRECT, PATH_BULK, PATH_CE = 0, 1, 2
 STATE_OUT_PENDING, STATE_OUT, STATE_IN_PENDING, STATE_IN = 1, 2, 3, 4
@@ -32,7 +33,8 @@ _ERR_NAMES = {ERR_ARG: "ERR_ARG", ERR_NO_SPACE: "ERR_NO_SPACE", ERR_ALIGN: "ERR_
 EXPORTED = [
     "mpress_plan", "mpress_plan_stripes", "mpress_plan_units", "mpress_plan_get_info",
     "mpress_plan_free", "mpress_partition_sequential", "mpress_plan_global",
-    "mpress_plan_from_units", "mpress_schedule_1f1b", "mpress_map_search", "mpress_init",
+    "mpress_plan_from_units", "mpress_schedule_1f1b", "mpress_map_search",
+    "mpress_compaction_plan", "mpress_init",
     "mpress_init_local",
     "mpress_finalize", "mpress_stash_free", "mpress_set_option", "mpress_get_option",
     "mpress_swap_out", "mpress_swap_in", "mpress_wait", "mpress_query", "mpress_handle_state",
@@ -96,6 +98,8 @@ def _load():
                                        POINTER(c_uint64), POINTER(c_uint64)]),
         "mpress_plan_from_units": (c_int, [c_int, c_int, P, c_uint32, P, c_uint64, POINTER(P)]),
         "mpress_schedule_1f1b": (c_int, [POINTER(Params1F1B), P, P]),
+        "mpress_compaction_plan": (c_int, [c_uint32, P, c_uint64, P, P, POINTER(c_uint64),
+                                           POINTER(c_uint64)]),
         "mpress_map_search": (c_int, [c_int, P, P, P, P, P, c_uint64, P, POINTER(c_uint64),
                                       POINTER(c_uint64), POINTER(c_uint64)]),
         "mpress_init": (c_int, [c_int, c_int, c_int, P, EXCHANGE_FN, P, POINTER(P)]),
@@ -251,6 +255,29 @@ def schedule_1f1b(stages, stage, micro_batches, t_fwd_ns, t_bwd_ns, t_out_ns, t_
     names = [f[0] for f in Slot1F1B._fields_]
     return ([{n: getattr(s, n) for n in names} for s in slots],
             {f[0]: getattr(summ, f[0]) for f in Summary1F1B._fields_ if f[0] != "pad"})
+
+
+class TensorStat(ctypes.Structure):
+    _fields_ = [("bytes", c_uint64), ("live_ns", c_uint64), ("recompute_ns", c_uint64),
+                ("cpu_swap_ns", c_uint64), ("d2d_swap_ns", c_uint64)]
+
+
+NOT_RECOMPUTABLE = (1 << 64) - 1
+CHOICE_CPU_SWAP, CHOICE_RECOMPUTE, CHOICE_D2D = 1, 2, 3
+
+
+def compaction_plan(stats, d2d_capacity):
+    """NEXT-4 (mpress_compaction_plan).  stats: dicts with bytes, live_ns,
+    recompute_ns, cpu_swap_ns, d2d_swap_ns.  Returns (choices, overheads,
+    total, d2d_bytes)."""
+    n = len(stats)
+    arr = (TensorStat * max(1, n))(*[TensorStat(t["bytes"], t["live_ns"], t["recompute_ns"],
+                                                t["cpu_swap_ns"], t["d2d_swap_ns"]) for t in stats])
+    ch = (c_uint32 * max(1, n))()
+    ov = (c_uint64 * max(1, n))()
+    tot, used = c_uint64(), c_uint64()
+    _check(lib.mpress_compaction_plan(n, arr, d2d_capacity, ch, ov, byref(tot), byref(used)))
+    return list(ch)[:n], list(ov)[:n], tot.value, used.value
 
 
 def map_search(demand, spare, link, egress=None, ingress=None, granule=0):

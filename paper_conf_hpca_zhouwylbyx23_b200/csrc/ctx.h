@@ -55,6 +55,7 @@ struct Mapping {
   CUdeviceptr va = 0;
   size_t size = 0;
   bool reserved = false, mapped = false, has_handle = false;
+  void* host = nullptr;  // NEXT-4: pinned host pool (cudaHostAlloc, mapped)
 };
 
 // A CUDA event shared by a handle and the fences its swap-in leaves behind;

@@ -107,7 +107,27 @@ void unmap(const Driver* d, Mapping* m) {
   if (m->mapped) d->mem_unmap(m->va, m->size);
   if (m->reserved) d->mem_address_free(m->va, m->size);
   if (m->has_handle) d->mem_release(m->handle);
+  if (m->host) cudaFreeHost(m->host);
   *m = Mapping();
+}
+
+// NEXT-4 (GPU-CPU swap tier): a "peer" whose pool is
+// pinned host memory, allocated once ("a host pinned memory pool that is not
+// part of the PyTorch runtime") and mapped into the device's address
+// space, so the same stripes and kernels move bytes over PCIe.
+int map_host_pool(Mapping* m, uint64_t bytes) {
+  m->size = roundup(bytes, 2u << 20);
+  cudaError_t e = cudaHostAlloc(&m->host, m->size, cudaHostAllocMapped | cudaHostAllocPortable);
+  if (e != cudaSuccess) {
+    m->host = nullptr;
+    return fail(MPRESS_ERR_CUDA, "cudaHostAlloc (host stash pool, %llu B): %s", (unsigned long long)m->size,
+                cudaGetErrorString(e));
+  }
+  void* dev = nullptr;
+  e = cudaHostGetDevicePointer(&dev, m->host, 0);
+  if (e != cudaSuccess) return fail(MPRESS_ERR_CUDA, "cudaHostGetDevicePointer: %s", cudaGetErrorString(e));
+  m->va = reinterpret_cast<CUdeviceptr>(dev);
+  return MPRESS_OK;
 }
 
 void destroy(mpress_ctx_s* c) {
@@ -154,6 +174,7 @@ extern "C" int mpress_init_local(int world, int source, const int* devices,
     return fail(MPRESS_ERR_ARG, "mpress_init_local: bad argument");
   *out = nullptr;
   MP_TRY(check_partition(world, partition));
+  if (devices[source] < 0) return fail(MPRESS_ERR_ARG, "mpress_init_local: the source must be a GPU");
   const Driver* d;
   MP_TRY(driver(&d));
   auto* c = new mpress_ctx_s();
@@ -172,6 +193,15 @@ extern "C" int mpress_init_local(int world, int source, const int* devices,
   for (int p = 0; p < world; ++p) {
     const uint64_t want = partition[(size_t)source * world + p];
     if (p == source || want == 0) continue;
+    if (devices[p] == MPRESS_DEVICE_HOST) {
+      const int rc = map_host_pool(&c->maps[p], want);
+      if (rc != MPRESS_OK) {
+        destroy(c);
+        return rc;
+      }
+      init_partition(&c->parts[p], reinterpret_cast<uint8_t*>(c->maps[p].va), want);
+      continue;
+    }
     size_t gran;
     int rc = granularity(d, devices[p], false, &gran);
     if (rc == MPRESS_OK) {
