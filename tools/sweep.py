@@ -119,6 +119,27 @@ def sizes_sweep():
             torch.cuda.empty_cache()
 
 
+def host():
+    """NEXT-4: the pinned host pool as the only peer (GPU-CPU swap over PCIe)."""
+    s = torch.cuda.Stream()
+    for size in (64 << 20, 256 << 20, 1 << 30):
+        sizes = [size]
+        pl = mp.plan(2, 0, [0, 4 << 30], [0, 1], sizes)
+        part = [[0, pl.units[1] * mp.DEFAULT_GRANULE], [0, 0]]
+        ctx = mp.Context.local(2, 0, [0, mp.DEVICE_HOST], part)
+        src = [torch.empty(size, dtype=torch.uint8, device="cuda")]
+        synth_dev.fill(src[0], 5, 0)
+        dst = [torch.empty(size, dtype=torch.uint8, device="cuda")]
+        torch.cuda.synchronize()
+        for name, cap in (("direct", 0), ("direct", 32), ("bulk", 0), ("ce", 0)):
+            ctx.set_option(mp.OPT_PATH, PATHS[name])
+            ctx.set_option(mp.OPT_MAX_CTAS, cap)
+            to, ti = time_swaps(ctx, pl, src, dst, 4, s)
+            print(json.dumps({"sweep": "host", "bytes": size, "path": name, "max_ctas": cap,
+                              "out_gbs": size / to / 1e6, "in_gbs": size / ti / 1e6}), flush=True)
+        ctx.finalize()
+
+
 def gemm():
     """GEMM slowdown with the bench's protocol: for every (path, variant, cap)
     an alone round and a with-swap round of 24 GEMMs alternate, and only GEMMs
@@ -193,4 +214,4 @@ def gemm():
 
 if __name__ == "__main__":
     what = sys.argv[1] if len(sys.argv) > 1 else "paths"
-    {"paths": paths, "sizes": sizes_sweep, "gemm": gemm}[what]()
+    {"paths": paths, "sizes": sizes_sweep, "gemm": gemm, "host": host}[what]()
