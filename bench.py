@@ -58,6 +58,8 @@ def parse():
     ap.add_argument("--gemm-cap", type=int, default=64,
                     help="swap grid cap (CTAs = SMs touched) while the concurrent GEMM runs")
     ap.add_argument("--no-gemm", action="store_true")
+    ap.add_argument("--no-configs", action="store_true",
+                    help="skip the other BASELINE configs (1, 3, 4) reported beside the headline")
     return ap.parse_args()
 
 
@@ -397,6 +399,11 @@ def main():
     e2e = run_e2e(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap_stream, n, dist)
     gemm = None if args.no_gemm else gemm_interference(args, ctx, mp, world, source, per_copy, bw,
                                                         sizes, src, dst, swap_stream, n, dist)
+    others = None
+    if n == 1 and not args.no_configs:
+        del src, dst
+        torch.cuda.empty_cache()
+        others = other_configs(args, mp, local_rank)
 
     cpu = None
     planner = None
@@ -414,7 +421,7 @@ def main():
             "per_direction_gbs": per_dir,
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": launches[0], "clocks": clk, "gemm_slowdown": gemm,
-            "planner": planner,
+            "planner": planner, "other_configs": others,
             "parity": "round trip bit-exact vs generator (all %d tensors x %d ranks)" % (47 * mb, n),
         }
         print(json.dumps(line))
@@ -422,6 +429,66 @@ def main():
     if n > 1:
         dist.destroy_process_group()
     return 0
+
+
+def other_configs(args, mp, device):
+    """BASELINE configs 1, 3 and 4 on this GPU (loopback peers), same kernel
+    path and grid as the headline: swapped GB/s (out + in) of one round trip,
+    median of 5 after 2 warm-ups, every byte checked against the generator.
+    Config 5 needs 8 GPUs (its topology runs in tests/test_gpu_multiprocess.py)."""
+    import torch
+    from synth import device as synth_dev
+    from synth import workloads
+    path = {"direct": mp.PATH_DIRECT, "bulk": mp.PATH_BULK, "ce": mp.PATH_CE}[args.path]
+    c3 = workloads.CONFIGS[3]
+    cases = [
+        ("cfg1 16 x 4 MiB fp16 activations -> 1 peer", 2, [1], [0, 1 << 30], workloads.cfg1_sizes()),
+        ("cfg3 GPT-10.3B stage-0 Adam m/v (100 tensors, 12.21 GB) -> 3 peers, 2 GiB cap on one", 8,
+         c3["peers"], workloads.spare_vector(8, 0, c3["peers"], spare_by_peer=c3["spare_by_peer"]),
+         workloads.cfg3_sizes()),
+        ("cfg4 one 4 GiB uint8 tensor -> 7 peers", 8, list(range(1, 8)),
+         workloads.spare_vector(8, 0, list(range(1, 8)), spare=8 << 30), [4 << 30]),
+        ("cfg4 one 4 MiB uint8 tensor -> 7 peers", 8, list(range(1, 8)),
+         workloads.spare_vector(8, 0, list(range(1, 8)), spare=8 << 30), [4 << 20]),
+    ]
+    out = []
+    s = torch.cuda.Stream()
+    for name, world, peers, spare, sizes in cases:
+        bw = workloads.bw_vector(world, 0, peers)
+        pl = mp.plan(world, 0, spare, bw, sizes)
+        part = [[0] * world for _ in range(world)]
+        part[0] = [u * mp.DEFAULT_GRANULE for u in pl.units]
+        ctx = mp.Context.local(world, 0, [device] * world, part)
+        try:
+            ctx.set_option(mp.OPT_PATH, path)
+            ctx.set_option(mp.OPT_MAX_CTAS, args.max_ctas)
+            src = [torch.empty(b, dtype=torch.uint8, device="cuda") for b in sizes]
+            dst = [torch.empty(b, dtype=torch.uint8, device="cuda") for b in sizes]
+            for i, t in enumerate(src):
+                synth_dev.fill(t, 1000 * (len(out) + 1), i)
+            torch.cuda.synchronize()
+            ts = []
+            for r in range(7):
+                e0 = torch.cuda.Event(enable_timing=True)
+                e1 = torch.cuda.Event(enable_timing=True)
+                e0.record(s)
+                h = ctx.swap_out(pl, src, stream=s)
+                ctx.swap_in(h, dst, stream=s)
+                e1.record(s)
+                torch.cuda.synchronize()
+                h.free()
+                if r >= 2:
+                    ts.append(e0.elapsed_time(e1))
+            ms = statistics.median(ts)
+            bad = sum(synth_dev.check(t, 1000 * (len(out) + 1), i) for i, t in enumerate(dst))
+            out.append({"config": name, "bytes": sum(sizes), "stripes": len(pl.stripes),
+                        "round_trip_ms": ms, "gbs": 2 * sum(sizes) / (ms / 1e3) / 1e9,
+                        "bit_exact": bad == 0})
+            del src, dst
+            torch.cuda.empty_cache()
+        finally:
+            ctx.finalize()
+    return out
 
 
 def planner_timing(mp, world, source, spare, bw, sizes):
