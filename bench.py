@@ -396,20 +396,28 @@ def main():
                 "peak_source": "B200_PROFILING.md measured peer copy per direction"}
     per_dir = {k: bytes_per_mb / (statistics.mean(v) / 1e3) / 1e9 for k, v in dur.items()}
 
-    e2e = run_e2e(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap_stream, n, dist)
-    gemm = None if args.no_gemm else gemm_interference(args, ctx, mp, world, source, per_copy, bw,
-                                                        sizes, src, dst, swap_stream, n, dist)
+    # The legs below add context to the headline; a failure in one is
+    # reported in its key instead of losing the measured line.
+    def leg(fn, *a):
+        try:
+            return fn(*a)
+        except Exception as exc:  # pragma: no cover - reported, not hidden
+            return {"error": "%s: %s" % (type(exc).__name__, exc)}
+
+    e2e = leg(run_e2e, args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap_stream, n, dist)
+    gemm = None if args.no_gemm else leg(gemm_interference, args, ctx, mp, world, source, per_copy, bw,
+                                         sizes, src, dst, swap_stream, n, dist)
     others = None
     if n == 1 and not args.no_configs:
         del src, dst
         torch.cuda.empty_cache()
-        others = other_configs(args, mp, local_rank)
+        others = leg(other_configs, args, mp, local_rank)
 
     cpu = None
     planner = None
     if rank == 0 and n == 1 and not args.no_cpu_baseline:
-        cpu = oracle_sample(args.cpu_seconds)
-        planner = planner_timing(mp, world, source, per_copy, bw, sizes)
+        cpu = leg(oracle_sample, args.cpu_seconds)
+        planner = leg(planner_timing, mp, world, source, per_copy, bw, sizes)
 
     if rank == 0:
         line = {
