@@ -194,7 +194,7 @@ class Plan:
 
     def __del__(self):
         h = getattr(self, "_h", None)
-        if h is not None and h.value:
+        if h is not None and h.value and lib is not None:
             lib.mpress_plan_free(h)
             self._h = None
 
@@ -355,10 +355,22 @@ def share_fds(world, rank, my_fd, want, exchange_cb):
 # --------------------------------------------------------------- context / swap
 
 class Handle:
+    """An mpress_handle_t (one swapped batch).  Released by free(), by the
+    garbage collector (forced), or when its context is finalized."""
+
     def __init__(self, ctx, h, plan):
         self._ctx = ctx
         self._h = h
         self.plan = plan  # keeps the Plan alive while the handle exists
+        ctx._handles.add(self)
+
+    def __del__(self):
+        try:
+            if self._h is not None and self._h.value and self._ctx._h is not None:
+                lib.mpress_handle_free(self._ctx._h, self._h, 1)
+        except Exception:  # pragma: no cover - interpreter shutdown
+            pass
+        self._h = None
 
     @property
     def state(self):
@@ -379,11 +391,22 @@ class Context:
     """An mpress_ctx_t: this source's view of the peers' stash pools."""
 
     def __init__(self, h, world, source, device, exchange_cb=None):
+        import weakref
         self._h = h
         self.world = world
         self.source = source
         self.device = device
         self._exchange = exchange_cb  # keep the ctypes callback alive
+        self._handles = weakref.WeakSet()
+
+    def __del__(self):
+        # A local context can be released here; a distributed one must be
+        # finalized collectively by the caller (mpress_finalize is a barrier).
+        try:
+            if self._h is not None and self._exchange is None:
+                self.finalize()
+        except Exception:  # pragma: no cover - interpreter shutdown
+            pass
 
     @classmethod
     def local(cls, world, source, devices, partition):
@@ -406,8 +429,10 @@ class Context:
 
     def finalize(self):
         if self._h is not None:
-            _check(lib.mpress_finalize(self._h))
-            self._h = None
+            for hd in list(self._handles):   # the library frees them with the context
+                hd._h = None
+            h, self._h = self._h, None
+            _check(lib.mpress_finalize(h))
 
     def set_option(self, key, value):
         _check(lib.mpress_set_option(self._h, key, int(value)))

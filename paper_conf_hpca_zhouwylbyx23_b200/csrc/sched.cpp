@@ -280,6 +280,7 @@ extern "C" int mpress_swap_in(mpress_ctx_t* c, mpress_handle_t* h, void* const* 
 
 extern "C" int mpress_wait(mpress_ctx_t* c, mpress_handle_t* h, void* consumer) {
   if (!c || !h || h->ctx != c) return fail(MPRESS_ERR_ARG, "mpress_wait: bad argument");
+  std::lock_guard<std::mutex> lk(c->mu);
   DeviceGuard g(c->device);
   const EvRef& e = (h->state == MPRESS_STATE_IN_PENDING || h->state == MPRESS_STATE_IN) ? h->in_done : h->out_done;
   if (!e) return fail(MPRESS_ERR_STATE, "mpress_wait: nothing enqueued");
@@ -290,6 +291,7 @@ extern "C" int mpress_wait(mpress_ctx_t* c, mpress_handle_t* h, void* consumer) 
 
 extern "C" int mpress_query(mpress_ctx_t* c, mpress_handle_t* h) {
   if (!c || !h || h->ctx != c) return fail(MPRESS_ERR_ARG, "mpress_query: bad argument");
+  std::lock_guard<std::mutex> lk(c->mu);
   DeviceGuard g(c->device);
   cudaEvent_t e;
   int next;
