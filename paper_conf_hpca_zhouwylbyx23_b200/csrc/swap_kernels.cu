@@ -128,6 +128,47 @@ __device__ __forceinline__ void st_stream(int4* p, const int4& v) {
                :: "l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
 }
 
+// sm_100 moves 32 bytes per thread per instruction (SASS LDG/STG .256), which
+// halves the load/store instructions of a chunk; the L2 eviction-priority
+// qualifiers exist only at this width.
+struct alignas(32) V8 {
+  uint32_t v[8];
+};
+
+template <bool EVICT_FIRST>
+__device__ __forceinline__ V8 ld_stream(const V8* p) {
+  V8 r;
+  if (EVICT_FIRST)
+    asm volatile("ld.global.nc.L1::no_allocate.L2::evict_first.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=r"(r.v[0]), "=r"(r.v[1]), "=r"(r.v[2]), "=r"(r.v[3]), "=r"(r.v[4]), "=r"(r.v[5]),
+                   "=r"(r.v[6]), "=r"(r.v[7]) : "l"(p));
+  else
+    asm volatile("ld.global.nc.L1::no_allocate.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=r"(r.v[0]), "=r"(r.v[1]), "=r"(r.v[2]), "=r"(r.v[3]), "=r"(r.v[4]), "=r"(r.v[5]),
+                   "=r"(r.v[6]), "=r"(r.v[7]) : "l"(p));
+  return r;
+}
+
+__device__ __forceinline__ void st_stream(V8* p, const V8& r) {
+  asm volatile("st.global.L1::no_allocate.v8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};"
+               :: "l"(p), "r"(r.v[0]), "r"(r.v[1]), "r"(r.v[2]), "r"(r.v[3]), "r"(r.v[4]), "r"(r.v[5]),
+                  "r"(r.v[6]), "r"(r.v[7]) : "memory");
+}
+
+// One vector load of width VB (16 or 32 bytes); HINT = L2 evict-first (32 only).
+template <int VB, bool HINT>
+struct Vec;
+template <bool HINT>
+struct Vec<16, HINT> {
+  using T = int4;
+  static __device__ __forceinline__ T ld(const T* p) { return ld_stream(p); }
+};
+template <bool HINT>
+struct Vec<32, HINT> {
+  using T = V8;
+  static __device__ __forceinline__ T ld(const T* p) { return ld_stream<HINT>(p); }
+};
+
 // ---------------------------------------------------------------- direct path
 
 struct Span {
@@ -142,12 +183,14 @@ __device__ __forceinline__ Span span_of(const CopyTable<CAP>& t, uint32_t c, uin
   const uint64_t off = (uint64_t)(c - t.first_chunk[s]) << SHIFT;
   return Span{static_cast<const uint8_t*>(d.src) + off, static_cast<uint8_t*>(d.dst) + off, d.len - off};
 }
-// THREADS threads each keep UNROLL independent 16-B loads in flight, then
-// store them: one chunk = THREADS*UNROLL*16 bytes per CTA iteration.
-template <int DIR, int THREADS, int UNROLL, bool PF, int CAP>
+// THREADS threads each keep UNROLL independent VB-byte loads in flight, then
+// store them: one chunk = THREADS*UNROLL*VB bytes per CTA iteration.  VB = 32
+// needs 32-byte aligned descriptors (checked on the host, else VB = 16).
+template <int DIR, int THREADS, int UNROLL, int VB, bool HINT, bool PF, int CAP>
 __global__ void __launch_bounds__(THREADS)
 mp_swap_direct(const __grid_constant__ CopyTable<CAP> t) {
-  constexpr uint32_t kChunk = THREADS * UNROLL * 16;
+  using VT = typename Vec<VB, HINT>::T;
+  constexpr uint32_t kChunk = THREADS * UNROLL * VB;
   static_assert((kChunk & (kChunk - 1)) == 0, "chunk must be a power of two");
   constexpr uint32_t kShift = __builtin_ctz(kChunk);
   // PF: the next chunk's address is resolved while the current chunk's loads
@@ -163,11 +206,11 @@ mp_swap_direct(const __grid_constant__ CopyTable<CAP> t) {
     Span nx;
     bool more;
     if (sp.rem >= kChunk) {
-      const int4* sv = reinterpret_cast<const int4*>(sp.src) + threadIdx.x;
-      int4* dv = reinterpret_cast<int4*>(sp.dst) + threadIdx.x;
-      int4 r[UNROLL];
+      const VT* sv = reinterpret_cast<const VT*>(sp.src) + threadIdx.x;
+      VT* dv = reinterpret_cast<VT*>(sp.dst) + threadIdx.x;
+      VT r[UNROLL];
 #pragma unroll
-      for (int j = 0; j < UNROLL; ++j) r[j] = ld_stream(sv + j * THREADS);
+      for (int j = 0; j < UNROLL; ++j) r[j] = Vec<VB, HINT>::ld(sv + j * THREADS);
       if (PF) {
         more = cur.next(&c, &s);
         if (more) nx = span_of<kShift>(t, c, s);
@@ -321,14 +364,20 @@ struct Shape {
   uint32_t shift;   // log2 bytes per chunk / bulk piece
   size_t smem;      // dynamic shared memory
   int per_sm;       // default CTAs per SM when MPRESS_OPT_MAX_CTAS = 0
+  int vb;           // vector bytes per thread access (direct path)
+  int fallback;     // variant used when a 32-byte variant meets 16-byte-aligned data
 };
 
-// direct: (threads, unroll) = (256,8) (512,8) (256,16) (1024,4) (128,8)
-// bulk:   (piece, stages)   = (32K,6) (16K,12) (64K,3)
+// direct (threads, unroll, vector bytes): 0 (256,8,16) 1 (512,8,16)
+// 2 (256,16,16) 3 (1024,4,16) 4 (128,8,16) 5 (256,4,32) 6 (256,8,32)
+// 7 (128,4,32) 8 (256,4,32 + L2 evict-first loads) 9 (128,8,32)
+// bulk (piece, stages): 0 (32K,6) 1 (16K,12) 2 (64K,3)
 constexpr Shape kDirect[kDirectVariants] = {
-    {256, 15, 0, 2}, {512, 16, 0, 1}, {256, 16, 0, 2}, {1024, 16, 0, 1}, {128, 14, 0, 4}};
+    {256, 15, 0, 2, 16, 0}, {512, 16, 0, 1, 16, 1}, {256, 16, 0, 2, 16, 2}, {1024, 16, 0, 1, 16, 3},
+    {128, 14, 0, 4, 16, 4}, {256, 15, 0, 2, 32, 0}, {256, 16, 0, 2, 32, 2}, {128, 14, 0, 4, 32, 4},
+    {256, 15, 0, 2, 32, 0}, {128, 15, 0, 4, 32, 4}};
 constexpr Shape kBulk[kBulkVariants] = {
-    {32, 15, 6u << 15, 1}, {32, 14, 12u << 14, 1}, {32, 16, 3u << 16, 1}};
+    {32, 15, 6u << 15, 1, 16, 0}, {32, 14, 12u << 14, 1, 16, 1}, {32, 16, 3u << 16, 1, 16, 2}};
 
 template <int CAP>
 using KernelFn = void (*)(CopyTable<CAP>);
@@ -343,15 +392,20 @@ KernelFn<CAP> kernel_for(int path, int variant, int dir, bool pf) {
       default: return o ? mp_swap_bulk<kDirOut, 15, 6, CAP> : mp_swap_bulk<kDirIn, 15, 6, CAP>;
     }
   }
-#define MP_DIRECT(T, U) \
-  (o ? (pf ? mp_swap_direct<kDirOut, T, U, true, CAP> : mp_swap_direct<kDirOut, T, U, false, CAP>) \
-     : (pf ? mp_swap_direct<kDirIn, T, U, true, CAP> : mp_swap_direct<kDirIn, T, U, false, CAP>))
+#define MP_DIRECT(T, U, VB, H)                                                                        \
+  (o ? (pf ? mp_swap_direct<kDirOut, T, U, VB, H, true, CAP> : mp_swap_direct<kDirOut, T, U, VB, H, false, CAP>) \
+     : (pf ? mp_swap_direct<kDirIn, T, U, VB, H, true, CAP> : mp_swap_direct<kDirIn, T, U, VB, H, false, CAP>))
   switch (variant) {
-    case 1: return MP_DIRECT(512, 8);
-    case 2: return MP_DIRECT(256, 16);
-    case 3: return MP_DIRECT(1024, 4);
-    case 4: return MP_DIRECT(128, 8);
-    default: return MP_DIRECT(256, 8);
+    case 1: return MP_DIRECT(512, 8, 16, false);
+    case 2: return MP_DIRECT(256, 16, 16, false);
+    case 3: return MP_DIRECT(1024, 4, 16, false);
+    case 4: return MP_DIRECT(128, 8, 16, false);
+    case 5: return MP_DIRECT(256, 4, 32, false);
+    case 6: return MP_DIRECT(256, 8, 32, false);
+    case 7: return MP_DIRECT(128, 4, 32, false);
+    case 8: return MP_DIRECT(256, 4, 32, true);
+    case 9: return MP_DIRECT(128, 8, 32, false);
+    default: return MP_DIRECT(256, 8, 16, false);
   }
 #undef MP_DIRECT
 }
@@ -363,7 +417,7 @@ const Shape& shape_of(int path, int variant) {
 // Per-device cache of the default grid.
 struct DevCache {
   std::mutex mu;
-  int wave[2][8][64] = {};
+  int wave[2][16][64] = {};
 };
 DevCache g_cache;
 
@@ -489,6 +543,13 @@ int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* gr
   }
   const int nvar = path == MPRESS_PATH_BULK ? kBulkVariants : kDirectVariants;
   if (variant < 0 || variant >= nvar) return fail(MPRESS_ERR_ARG, "kernel variant %d out of range", variant);
+  if (shape_of(path, variant).vb == 32) {  // 32-byte vectors need 32-byte aligned addresses
+    for (size_t i = 0; i < n; ++i)
+      if ((reinterpret_cast<uintptr_t>(d[i].src) | reinterpret_cast<uintptr_t>(d[i].dst)) & 31) {
+        variant = shape_of(path, variant).fallback;
+        break;
+      }
+  }
   const int wave = copy_wave_ctas(path, variant);
   if (wave <= 0) return fail(MPRESS_ERR_CUDA, "occupancy query failed");
   const int cap = max_ctas > 0 ? max_ctas : wave;

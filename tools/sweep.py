@@ -64,10 +64,20 @@ def paths():
     nbytes = sum(sizes)
     ctx, pl, src, dst = setup(sizes, 3)
     s = torch.cuda.Stream()
-    nvar = {"direct": 4, "bulk": 3, "ce": 1}  # plus -1 = auto
+    nvar = {"direct": 10, "bulk": 3, "ce": 1}  # plus -1 = auto
+    only = os.environ.get("SWEEP_PATHS")        # e.g. "direct"
+    var_sel = os.environ.get("SWEEP_VARIANTS")  # e.g. "0,5,6,8"
+    cap_sel = os.environ.get("SWEEP_CAPS")      # e.g. "0,148,296"
     for name, path in PATHS.items():
+        if only and name not in only.split(","):
+            continue
         caps = [0] if name == "ce" else [0, 8, 16, 32, 64, 148, 296, 444, 592]
-        for var in ([-1] if name != "ce" else []) + list(range(nvar[name])):
+        if cap_sel and name != "ce":
+            caps = [int(x) for x in cap_sel.split(",")]
+        variants = ([-1] if name != "ce" else []) + list(range(nvar[name]))
+        if var_sel and name != "ce":
+            variants = [int(x) for x in var_sel.split(",")]
+        for var in variants:
             for cap in caps:
                 ctx.set_option(mp.OPT_PATH, path)
                 if name != "ce":
