@@ -365,9 +365,12 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
  * the SM-count cap that protects a concurrent GEMM.
  * MPRESS_OPT_VARIANT: kernel shape within the path -- direct: 0 = 256
  * threads x 8 vectors (2 CTAs/SM by default), 1 = 512x8, 2 = 256x16,
- * 3 = 1024x4, 4 = 128x8; bulk: 0 = 6 slots x 32 KiB, 1 = 12 x 16 KiB, 2 = 3 x 64 KiB;
- * MPRESS_VARIANT_AUTO (-1, default) = direct 4 when the grid is capped at
- * <= one CTA per SM (small CTAs co-reside with a GEMM), else 0.
+ * 3 = 1024x4, 4 = 128x8 (16-byte vectors), 5 = 256x4, 6 = 256x8, 7 = 128x4,
+ * 8 = 256x4 with L2 evict-first loads, 9 = 128x8 (32-byte vectors, used
+ * only when every address is 32-byte aligned, else the 16-byte shape);
+ * bulk: 0 = 6 slots x 32 KiB, 1 = 12 x 16 KiB, 2 = 3 x 64 KiB;
+ * MPRESS_VARIANT_AUTO (-1, default) = direct 7 when the grid is capped at
+ * <= one CTA per SM (small CTAs co-reside with a GEMM), else 5.
  * MPRESS_OPT_ORDER: chunk order inside one launch -- 0 = interleave the
  * peers by a weighted round robin, so every peer link carries its share of
  * the swap at every moment (default; needed when several sources share

@@ -538,8 +538,13 @@ int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* gr
     // CTAs fit in the registers and shared memory a cuBLAS GEMM CTA leaves
     // free (168 regs x 256 threads + 214 KB smem, profiles/r01), so they
     // co-reside instead of taking SMs away from it; full grid: 2 x 256-thread
-    // CTAs per SM saturate HBM (profiles/r01 sweeps).  bulk: 6 x 32 KiB.
-    variant = (path == MPRESS_PATH_DIRECT && max_ctas > 0 && max_ctas <= sms) ? 4 : 0;
+    // CTAs per SM saturate HBM (profiles/r01 sweeps).  Both use 32-byte
+    // vectors (LDG/STG .256, +1% over 16-byte ones; 16-byte fallback when the
+    // data is only 16-byte aligned).  bulk: 6 x 32 KiB.
+    if (path == MPRESS_PATH_DIRECT)
+      variant = (max_ctas > 0 && max_ctas <= sms) ? 7 : 5;
+    else
+      variant = 0;
   }
   const int nvar = path == MPRESS_PATH_BULK ? kBulkVariants : kDirectVariants;
   if (variant < 0 || variant >= nvar) return fail(MPRESS_ERR_ARG, "kernel variant %d out of range", variant);
