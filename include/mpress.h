@@ -305,6 +305,40 @@ typedef struct mpress_1f1b_summary {
 MPRESS_API int mpress_schedule_1f1b(const mpress_1f1b_params* params, mpress_1f1b_slot* slots,
                                     mpress_1f1b_summary* summary);
 
+/*
+ * The swap executor (the runtime "executor executes the memory saving
+ * operators ... swap-out ... and state recovering ones ... swap-in") of the
+ * exporter stage in a 1F1B pipeline, driven by mpress_schedule_1f1b.  The
+ * caller runs its compute ops in 1F1B order (mpress_executor_ops() of them)
+ * on its compute stream and brackets each op j:
+ *   mpress_executor_before(x, j, compute, &kind, &m)  -- kind 0 = F(m),
+ *       1 = B(m); for B(m) the compute stream waits for m's swap-in;
+ *   <enqueue the op on `compute`>
+ *   mpress_executor_after(x, j, compute, activations) -- for F(m), swaps out
+ *       `activations` ([n_tensors] device pointers of the plan's batch) on the
+ *       swap-out stream after the op; then enqueues every swap-in this op
+ *       triggers on the swap-in stream, into the buffers given by
+ *       mpress_executor_restore_to(x, m, dst) beforehand.
+ * Enqueue-only.  One executor serves any number of steps.
+ * Free executors before mpress_finalize of their context.
+ * Errors: MPRESS_ERR_ARG, MPRESS_ERR_STATE (op order violated, no restore
+ * buffers), plus those of swap_out / swap_in.
+ */
+typedef struct mpress_executor_s mpress_executor_t;
+MPRESS_API int mpress_executor_create(mpress_ctx_t* ctx, const mpress_plan_t* plan,
+                                      const mpress_1f1b_params* params, void* out_stream,
+                                      void* in_stream, mpress_executor_t** out);
+MPRESS_API int mpress_executor_ops(const mpress_executor_t* x);
+MPRESS_API int mpress_executor_slot(const mpress_executor_t* x, uint32_t micro_batch,
+                                    mpress_1f1b_slot* slot);
+MPRESS_API int mpress_executor_restore_to(mpress_executor_t* x, uint32_t micro_batch,
+                                          void* const* dst);
+MPRESS_API int mpress_executor_before(mpress_executor_t* x, uint32_t op, void* compute_stream,
+                                      uint32_t* kind, uint32_t* micro_batch);
+MPRESS_API int mpress_executor_after(mpress_executor_t* x, uint32_t op, void* compute_stream,
+                                     void* const* activations);
+MPRESS_API int mpress_executor_free(mpress_executor_t* x);
+
 /* ---- peer-memory layer ----------------------------------------------------- */
 
 /* All-gather callback, implemented by the caller over its process group:

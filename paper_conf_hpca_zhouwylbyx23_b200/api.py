@@ -34,7 +34,9 @@ EXPORTED = [
     "mpress_plan", "mpress_plan_stripes", "mpress_plan_units", "mpress_plan_get_info",
     "mpress_plan_free", "mpress_partition_sequential", "mpress_plan_global",
     "mpress_plan_from_units", "mpress_schedule_1f1b", "mpress_map_search",
-    "mpress_compaction_plan", "mpress_init",
+    "mpress_compaction_plan", "mpress_executor_create", "mpress_executor_ops",
+    "mpress_executor_slot", "mpress_executor_restore_to", "mpress_executor_before",
+    "mpress_executor_after", "mpress_executor_free", "mpress_init",
     "mpress_init_local",
     "mpress_finalize", "mpress_stash_free", "mpress_set_option", "mpress_get_option",
     "mpress_swap_out", "mpress_swap_in", "mpress_wait", "mpress_query", "mpress_handle_state",
@@ -98,6 +100,13 @@ def _load():
                                        POINTER(c_uint64), POINTER(c_uint64)]),
         "mpress_plan_from_units": (c_int, [c_int, c_int, P, c_uint32, P, c_uint64, POINTER(P)]),
         "mpress_schedule_1f1b": (c_int, [POINTER(Params1F1B), P, P]),
+        "mpress_executor_create": (c_int, [P, P, POINTER(Params1F1B), P, P, POINTER(P)]),
+        "mpress_executor_ops": (c_int, [P]),
+        "mpress_executor_slot": (c_int, [P, c_uint32, POINTER(Slot1F1B)]),
+        "mpress_executor_restore_to": (c_int, [P, c_uint32, P]),
+        "mpress_executor_before": (c_int, [P, c_uint32, P, POINTER(c_uint32), POINTER(c_uint32)]),
+        "mpress_executor_after": (c_int, [P, c_uint32, P, P]),
+        "mpress_executor_free": (c_int, [P]),
         "mpress_compaction_plan": (c_int, [c_uint32, P, c_uint64, P, P, POINTER(c_uint64),
                                            POINTER(c_uint64)]),
         "mpress_map_search": (c_int, [c_int, P, P, P, P, P, c_uint64, P, POINTER(c_uint64),
@@ -385,6 +394,44 @@ class Handle:
         if self._h is not None and self._h.value:
             _check(lib.mpress_handle_free(self._ctx._h, self._h, 1 if force else 0))
         self._h = None
+
+
+class Executor:
+    """mpress_executor_t: the paper's swap executor for the exporter
+    stage of a 1F1B pipeline (see include/mpress.h)."""
+
+    def __init__(self, ctx, plan_, stages, stage, micro_batches, t_fwd_ns, t_bwd_ns, t_out_ns, t_in_ns,
+                 out_stream, in_stream, duplex=True, slack_ns=0):
+        p = Params1F1B(stages, stage, micro_batches, 1 if duplex else 0, t_fwd_ns, t_bwd_ns,
+                       t_out_ns, t_in_ns, slack_ns)
+        h = c_void_p()
+        _check(lib.mpress_executor_create(ctx._h, plan_.handle, byref(p), _stream(out_stream),
+                                          _stream(in_stream), byref(h)))
+        self._h, self._ctx, self.plan = h, ctx, plan_
+        self.ops = _check(lib.mpress_executor_ops(h))
+
+    def slot(self, m):
+        s = Slot1F1B()
+        _check(lib.mpress_executor_slot(self._h, m, byref(s)))
+        return {f[0]: getattr(s, f[0]) for f in Slot1F1B._fields_}
+
+    def restore_to(self, m, dst):
+        _check(lib.mpress_executor_restore_to(self._h, m, _ptr_array(dst)))
+
+    def before(self, op, compute=None):
+        """Returns ('F' | 'B', micro-batch) of op `op`."""
+        k, m = c_uint32(), c_uint32()
+        _check(lib.mpress_executor_before(self._h, op, _stream(compute), byref(k), byref(m)))
+        return ("F" if k.value == 0 else "B"), m.value
+
+    def after(self, op, compute=None, activations=None):
+        _check(lib.mpress_executor_after(self._h, op, _stream(compute),
+                                         None if activations is None else _ptr_array(activations)))
+
+    def free(self):
+        if self._h is not None:
+            _check(lib.mpress_executor_free(self._h))
+            self._h = None
 
 
 class Context:

@@ -116,3 +116,8 @@ struct mpress_handle_s {
   mpress::EvRef in_done;
   bool slices_held = false;
 };
+
+namespace mpress {
+// A pooled CUDA event (disable-timing) owned by reference; sched.cpp.
+EvRef take_event(mpress_ctx_s* c);
+}  // namespace mpress

@@ -23,7 +23,6 @@
 #include "swap_kernels.h"
 
 namespace mpress {
-namespace {
 
 EvRef take_event(mpress_ctx_s* c) {
   cudaEvent_t e = nullptr;
@@ -36,6 +35,8 @@ EvRef take_event(mpress_ctx_s* c) {
   }
   return EvRef(e, [pool](CUevent_st* ev) { pool->push_back(ev); });
 }
+
+namespace {
 
 // Drop the fences whose swap-in has completed (oldest first; stops at the
 // first one still pending, so the cost is O(1) amortised).

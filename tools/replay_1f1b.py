@@ -117,35 +117,35 @@ def replay(S, e, M, scale, n_fwd_gemms, max_ctas, seed=7000, slack=0.5):
         start_of.update({("B", m): base_sched[m]["bwd_start"] for m in range(M)})
         base = torch.zeros(1, dtype=torch.int64, device="cuda")
 
+        # the native executor issues the swaps: swap-out after F(m),
+        # swap-in after its scheduled trigger op, B(m) waits for it
+        ex = mp.Executor(ctx, pl, S, e, M, t_f, t_b, t_out, t_in, s_out, s_in,
+                         slack_ns=int(slack * t_in))
+        assert ex.ops == len(ops)
+        src_ptr = [mp.pointers(src[m]) for m in range(M)]
+        for m in range(M):
+            ex.restore_to(m, dst[m])
+
         def step(with_swap):
             ev = []
-            hs = {}
             synth_dev.stamp(base, comp)
             t0 = torch.cuda.Event(enable_timing=True)
             t0.record(comp)
             for j, (kind, m) in enumerate(ops):
                 synth_dev.gate(base, start_of[(kind, m)], comp)
-                if kind == "B" and with_swap:
-                    ctx.wait(hs[m], comp)
+                if with_swap:
+                    assert ex.before(j, comp) == (kind, m)
                 b4 = torch.cuda.Event(enable_timing=True)
                 b4.record(comp)
                 (fwd if kind == "F" else bwd)()
                 x = torch.cuda.Event(enable_timing=True)
                 x.record(comp)
                 ev.append((b4, x))
-                if not with_swap:
-                    continue
-                if kind == "F":
-                    hs[m] = ctx.swap_out(pl, src[m], stream=s_out, after=ev[-1][1])
-                for mm in range(M):
-                    if sched[mm]["in_trigger"] == j:
-                        s_in.wait_event(ev[-1][1])
-                        ctx.swap_in(hs[mm], dst[mm], stream=s_in)
+                if with_swap:
+                    ex.after(j, comp, src_ptr[m] if kind == "F" else None)
             t1 = torch.cuda.Event(enable_timing=True)
             t1.record(comp)
             torch.cuda.synchronize()
-            for hh in hs.values():
-                hh.free()
             compute = sum(a.elapsed_time(b) for a, b in ev) * 1e6
             return t0.elapsed_time(t1) * 1e6, compute
 
@@ -161,6 +161,7 @@ def replay(S, e, M, scale, n_fwd_gemms, max_ctas, seed=7000, slack=0.5):
         yes = statistics.median(r[0] for r in runs)
         comp_yes = statistics.median(r[1] for r in runs)
         bad = sum(synth_dev.check(t, seed + m, i) for m in range(M) for i, t in enumerate(dst[m]))
+        ex.free()
         mb = sum(sizes)
         return {
             "stages": S, "stage": e, "micro_batches": M, "micro_batch_bytes": mb,
