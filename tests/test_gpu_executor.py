@@ -1,0 +1,74 @@
+"""The native swap executor on the GPU: op order, restore buffers and
+misuse errors; the byte-exact replay runs in test_gpu_pipeline.py."""
+import pytest
+import torch
+
+import paper_conf_hpca_zhouwylbyx23_b200 as mp
+from synth import device as synth_dev
+
+pytestmark = pytest.mark.gpu
+
+
+def _setup(M):
+    sizes = [4096, 10000, 333]
+    world = 3
+    spare, bw = [0, 1 << 24, 1 << 24], [0, 1, 1]
+    pl = mp.plan(world, 0, spare, bw, sizes, 4096)
+    part = [[0] * world for _ in range(world)]
+    part[0] = [M * u * 4096 for u in pl.units]
+    ctx = mp.Context.local(world, 0, [0] * world, part)
+    return ctx, pl, sizes
+
+
+def test_executor_steps_and_errors():
+    M = 3
+    ctx, pl, sizes = _setup(M)
+    s_out, s_in = torch.cuda.Stream(), torch.cuda.Stream()
+    comp = torch.cuda.current_stream()
+    try:
+        ex = mp.Executor(ctx, pl, 2, 0, M, 10_000, 20_000, 5_000, 5_000, s_out, s_in)
+        assert ex.ops == 2 * M
+        # B(0) before anything was swapped out
+        with pytest.raises(mp.MPressError) as ei:
+            ex.before(2, comp)
+        assert ei.value.code == mp.ERR_STATE
+        # F without activations
+        with pytest.raises(mp.MPressError) as ei:
+            ex.after(0, comp, None)
+        assert ei.value.code == mp.ERR_ARG
+        src = [[torch.empty(n, dtype=torch.uint8, device="cuda") for n in sizes] for _ in range(M)]
+        dst = [[torch.zeros(n, dtype=torch.uint8, device="cuda") for n in sizes] for _ in range(M)]
+        for step in range(3):                       # the executor serves many steps
+            for m in range(M):
+                for i, t in enumerate(src[m]):
+                    synth_dev.fill(t, 50 * step + m, i)
+                ex.restore_to(m, dst[m])
+            for j in range(ex.ops):
+                kind, m = ex.before(j, comp)
+                ex.after(j, comp, src[m] if kind == "F" else None)
+            torch.cuda.synchronize()
+            for m in range(M):
+                for i, t in enumerate(dst[m]):
+                    assert synth_dev.check(t, 50 * step + m, i) == 0, (step, m, i)
+        ex.free()
+    finally:
+        ctx.finalize()
+
+
+def test_executor_missing_restore_buffers():
+    M = 2
+    ctx, pl, sizes = _setup(M)
+    s_out, s_in = torch.cuda.Stream(), torch.cuda.Stream()
+    comp = torch.cuda.current_stream()
+    try:
+        ex = mp.Executor(ctx, pl, 1, 0, M, 10_000, 20_000, 5_000, 5_000, s_out, s_in)
+        src = [torch.zeros(n, dtype=torch.uint8, device="cuda") for n in sizes]
+        kind, m = ex.before(0, comp)
+        assert (kind, m) == ("F", 0)
+        with pytest.raises(mp.MPressError) as ei:   # F(0) triggers its own swap-in (S = 1)
+            ex.after(0, comp, src)
+        assert ei.value.code == mp.ERR_STATE
+        torch.cuda.synchronize()
+        ex.free()
+    finally:
+        ctx.finalize()
