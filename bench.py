@@ -431,6 +431,13 @@ def main():
             "gpu_launches": launches[0], "clocks": clk, "gemm_slowdown": gemm,
             "planner": planner, "other_configs": others,
             "parity": "round trip bit-exact vs generator (all %d tensors x %d ranks)" % (47 * mb, n),
+            "per_rank_gbs": value / n,
+            "link": ("HBM loopback (1 GPU: the peers are pools on the same GPU, bound by the HBM copy "
+                     "roofline, not NVLink)" if n == 1 else
+                     "NVLink 5 / NVSwitch (every rank swaps to all others; bound by 900 GB/s nominal, "
+                     "770 GB/s measured, per direction per GPU)"),
+            "note": "N=1 and N>1 cross different links, so value(N) / (N * value(1)) is not a "
+                    "scaling efficiency; compare per_rank_gbs with the NVLink roofline",
         }
         print(json.dumps(line))
     ctx.finalize()
