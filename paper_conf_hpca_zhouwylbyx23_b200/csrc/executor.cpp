@@ -25,7 +25,6 @@ struct mpress_executor_s {
   std::vector<std::vector<uint32_t>> trig;   // per op: micro-batches whose swap-in it triggers
   std::vector<mpress_handle_t*> handle;      // per micro-batch
   std::vector<std::vector<void*>> restore;   // per micro-batch: destination pointers
-  std::vector<mpress::EvRef> op_done;        // per op: event after its compute
   std::vector<mpress_1f1b_slot> slots;
 };
 
@@ -68,7 +67,6 @@ extern "C" int mpress_executor_create(mpress_ctx_t* ctx, const mpress_plan_t* pl
     for (uint32_t m = 0; m < M; ++m) x->trig[x->slots[m].in_trigger].push_back(m);
     x->handle.assign(M, nullptr);
     x->restore.assign(M, {});
-    x->op_done.assign(x->kind.size(), EvRef());
   } catch (const std::bad_alloc&) {
     delete x;
     return fail(MPRESS_ERR_ARG, "mpress_executor_create: out of host memory");
@@ -110,7 +108,8 @@ extern "C" int mpress_executor_after(mpress_executor_t* x, uint32_t op, void* co
   if (!done) return fail(MPRESS_ERR_CUDA, "cudaEventCreate failed");
   cudaError_t e = cudaEventRecord(done.get(), static_cast<cudaStream_t>(compute_stream));
   if (e != cudaSuccess) return fail(MPRESS_ERR_CUDA, "cudaEventRecord: %s", cudaGetErrorString(e));
-  x->op_done[op] = done;
+  // `done` may go back to the pool when this call returns: the swap-out's
+  // and swap-in stream's waits below captured its record already
   const int m = x->mb[op];
   if (x->kind[op] == 0) {  // F(m) produced the activations: swap them out
     if (!activations) return fail(MPRESS_ERR_ARG, "mpress_executor_after: F(%d) needs its activations", m);

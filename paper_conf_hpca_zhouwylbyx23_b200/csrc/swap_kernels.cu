@@ -186,6 +186,8 @@ __device__ __forceinline__ Span span_of(const CopyTable<CAP>& t, uint32_t c, uin
 // THREADS threads each keep UNROLL independent VB-byte loads in flight, then
 // store them: one chunk = THREADS*UNROLL*VB bytes per CTA iteration.  VB = 32
 // needs 32-byte aligned descriptors (checked on the host, else VB = 16).
+// DIR only names the instantiation (swap-out vs swap-in in profiles): the
+// byte movement is the same, the descriptors say which side is the peer.
 template <int DIR, int THREADS, int UNROLL, int VB, bool HINT, bool PF, int CAP>
 __global__ void __launch_bounds__(THREADS)
 mp_swap_direct(const __grid_constant__ CopyTable<CAP> t) {

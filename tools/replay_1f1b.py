@@ -82,10 +82,6 @@ def replay(S, e, M, scale, n_fwd_gemms, max_ctas, seed=7000, slack=0.5):
         t_f = int(timed(fwd, comp))
         t_b = int(timed(bwd, comp))
 
-        def swap_pair():
-            hh = ctx.swap_out(pl, src[0], stream=s_out)
-            ctx.swap_in(hh, dst[0], stream=s_out)
-            return hh
         # swap times of one micro-batch, alone
         outs, ins = [], []
         for _ in range(4):
