@@ -458,6 +458,8 @@ def other_configs(args, mp, device):
     c3 = workloads.CONFIGS[3]
     cases = [
         ("cfg1 16 x 4 MiB fp16 activations -> 1 peer", 2, [1], [0, 1 << 30], workloads.cfg1_sizes()),
+        ("cfg2 x8 micro-batches batched into one plan (376 tensors, 7.03 GiB, P:209) -> 3 peers", 4,
+         [1, 2, 3], workloads.spare_vector(4, 0, [1, 2, 3], spare=24 << 30), workloads.cfg2_sizes(8)),
         ("cfg3 GPT-10.3B stage-0 Adam m/v (100 tensors, 12.21 GB) -> 3 peers, 2 GiB cap on one", 8,
          c3["peers"], workloads.spare_vector(8, 0, c3["peers"], spare_by_peer=c3["spare_by_peer"]),
          workloads.cfg3_sizes()),
