@@ -414,6 +414,15 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
 #define MPRESS_OPT_MAX_CTAS  2
 #define MPRESS_OPT_VARIANT   3
 #define MPRESS_OPT_ORDER     4
+/* Read-only (mpress_get_option): how the peer pools were mapped --
+ * MPRESS_TRANSPORT_LOCAL (mpress_init_local), _VMM_FD (cuMem pools exported
+ * as POSIX fds, passed over Unix sockets), or _LEGACY_IPC (cudaMalloc pools
+ * shared with CUDA IPC handles through the all-gather; used when the fd path
+ * fails on any rank, or forced with the environment variable MPRESS_IPC=legacy). */
+#define MPRESS_OPT_TRANSPORT 5
+#define MPRESS_TRANSPORT_LOCAL      0
+#define MPRESS_TRANSPORT_VMM_FD     1
+#define MPRESS_TRANSPORT_LEGACY_IPC 2
 #define MPRESS_VARIANT_AUTO  (-1)
 #define MPRESS_ORDER_INTERLEAVE 0
 #define MPRESS_ORDER_PLAN       1

@@ -22,6 +22,8 @@ DEFAULT_GRANULE = 65536
 OPT_PATH, OPT_MAX_CTAS, OPT_VARIANT, OPT_ORDER = 1, 2, 3, 4
 ORDER_INTERLEAVE, ORDER_PLAN = 0, 1
 DEVICE_HOST = -1   # mpress_init_local: a pinned host pool as a peer (NEXT-4)
+OPT_TRANSPORT = 5  # read-only
+TRANSPORT_LOCAL, TRANSPORT_VMM_FD, TRANSPORT_LEGACY_IPC = 0, 1, 2
 VARIANT_AUTO = -1
 PATH_DIRECT, PATH_BULK, PATH_CE = 0, 1, 2
 STATE_OUT_PENDING, STATE_OUT, STATE_IN_PENDING, STATE_IN = 1, 2, 3, 4

@@ -56,6 +56,8 @@ struct Mapping {
   size_t size = 0;
   bool reserved = false, mapped = false, has_handle = false;
   void* host = nullptr;  // NEXT-4: pinned host pool (cudaHostAlloc, mapped)
+  void* ipc_owned = nullptr;   // legacy-IPC transport: this rank's cudaMalloc pool
+  void* ipc_opened = nullptr;  // legacy-IPC transport: a peer's pool, opened here
 };
 
 // A CUDA event shared by a handle and the fences its swap-in leaves behind;
@@ -96,6 +98,7 @@ struct mpress_ctx_s {
   int max_ctas = 0;
   int variant = MPRESS_VARIANT_AUTO;
   int order = MPRESS_ORDER_INTERLEAVE;
+  int transport = MPRESS_TRANSPORT_LOCAL;
   int last_launches = 0;
   std::vector<cudaStream_t> ce_streams;  // copy-engine comparator, one per peer
   mpress::EvPool ev_pool = std::make_shared<std::vector<cudaEvent_t>>();

@@ -12,6 +12,7 @@
 #include <unistd.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 
@@ -108,6 +109,8 @@ void unmap(const Driver* d, Mapping* m) {
   if (m->reserved) d->mem_address_free(m->va, m->size);
   if (m->has_handle) d->mem_release(m->handle);
   if (m->host) cudaFreeHost(m->host);
+  if (m->ipc_opened) cudaIpcCloseMemHandle(m->ipc_opened);
+  if (m->ipc_owned) cudaFree(m->ipc_owned);
   *m = Mapping();
 }
 
@@ -231,6 +234,80 @@ extern "C" int mpress_init_local(int world, int source, const int* devices,
   return MPRESS_OK;
 }
 
+namespace mpress {
+namespace {
+
+int init_vmm_fd(mpress_ctx_s* c, const Driver* d, int rc);
+
+// All ranks learn whether every rank succeeded (a barrier as well).
+int agree(mpress_ctx_s* c, int rc, const char* what) {
+  int32_t ok = rc == MPRESS_OK;
+  std::vector<int32_t> okv(c->world);
+  if (c->exchange(c->exchange_user, &ok, sizeof ok, okv.data()) != 0)
+    return rc != MPRESS_OK ? rc : fail(MPRESS_ERR_SYS, "mpress_init: exchange failed");
+  for (int r = 0; r < c->world; ++r)
+    if (!okv[r]) return rc != MPRESS_OK ? rc : fail(MPRESS_ERR_PEER, "mpress_init: rank %d failed to %s", r, what);
+  return rc;
+}
+
+void reset_pools(mpress_ctx_s* c, const Driver* d) {
+  for (auto& m : c->maps) unmap(d, &m);
+  unmap(d, &c->own);
+  for (auto& p : c->parts) p = Partition();
+}
+
+uint64_t partition_offset(const mpress_ctx_s* c, int p) {  // where my partition of p's pool starts
+  uint64_t off = 0;
+  for (int s = 0; s < c->source; ++s) off += c->partition[(size_t)s * c->world + p];
+  return off;
+}
+
+// Transport 1 (fallback): the pools are cudaMalloc allocations shared with
+// CUDA IPC handles, which travel through the all-gather itself (no sockets).
+int init_legacy_ipc(mpress_ctx_s* c) {
+  const int world = c->world, rank = c->source;
+  uint64_t pool = 0;
+  for (int s = 0; s < world; ++s) pool += c->partition[(size_t)s * world + rank];
+  struct Info {
+    cudaIpcMemHandle_t h;
+    uint64_t size;
+    int32_t ok, pad;
+  } mine;
+  memset(&mine, 0, sizeof mine);
+  int rc = MPRESS_OK;
+  if (pool > 0) {
+    c->own.size = roundup(pool, 2u << 20);
+    cudaError_t e = cudaMalloc(&c->own.ipc_owned, c->own.size);
+    if (e == cudaSuccess) e = cudaIpcGetMemHandle(&mine.h, c->own.ipc_owned);
+    if (e != cudaSuccess) rc = fail(MPRESS_ERR_CUDA, "CUDA IPC stash pool: %s", cudaGetErrorString(e));
+  }
+  mine.size = c->own.size;
+  mine.ok = rc == MPRESS_OK;
+  std::vector<Info> all(world);
+  if (c->exchange(c->exchange_user, &mine, sizeof mine, all.data()) != 0 && rc == MPRESS_OK)
+    rc = fail(MPRESS_ERR_SYS, "mpress_init: exchange failed");
+  for (int r = 0; r < world && rc == MPRESS_OK; ++r)
+    if (!all[r].ok) rc = fail(MPRESS_ERR_CUDA, "mpress_init: rank %d failed to create its pool", r);
+  for (int p = 0; p < world && rc == MPRESS_OK; ++p) {
+    const uint64_t want = c->partition[(size_t)rank * world + p];
+    if (p == rank || want == 0) continue;
+    Mapping& m = c->maps[p];
+    cudaError_t e = cudaIpcOpenMemHandle(&m.ipc_opened, all[p].h, cudaIpcMemLazyEnablePeerAccess);
+    if (e != cudaSuccess) {
+      m.ipc_opened = nullptr;
+      rc = fail(MPRESS_ERR_PEER, "cudaIpcOpenMemHandle (rank %d's pool): %s", p, cudaGetErrorString(e));
+      break;
+    }
+    m.size = all[p].size;
+    m.va = reinterpret_cast<CUdeviceptr>(m.ipc_opened);
+    init_partition(&c->parts[p], reinterpret_cast<uint8_t*>(m.va) + partition_offset(c, p), want);
+  }
+  return rc;
+}
+
+}  // namespace
+}  // namespace mpress
+
 extern "C" int mpress_init(int device, int world, int rank, const uint64_t* partition,
                            mpress_exchange_fn exchange, void* exchange_user,
                            mpress_ctx_t** out) {
@@ -252,6 +329,41 @@ extern "C" int mpress_init(int device, int world, int rank, const uint64_t* part
   DeviceGuard g(device);
   int rc = cudaFree(nullptr) == cudaSuccess ? MPRESS_OK
                                             : fail(MPRESS_ERR_CUDA, "mpress_init: cannot initialise device %d", device);
+  // MPRESS_IPC=legacy selects CUDA IPC handles from the start; otherwise the
+  // cuMem + fd path runs first and all ranks fall back together if it fails.
+  const char* ipc_env = getenv("MPRESS_IPC");
+  if (ipc_env && strcmp(ipc_env, "legacy") == 0) {
+    c->transport = MPRESS_TRANSPORT_LEGACY_IPC;
+    rc = init_legacy_ipc(c);
+  } else {
+    rc = init_vmm_fd(c, d, rc);
+    if (agree(c, rc, "map its peers") != MPRESS_OK) {
+      reset_pools(c, d);
+      c->transport = MPRESS_TRANSPORT_LEGACY_IPC;
+      rc = init_legacy_ipc(c);
+    }
+  }
+  if (rc == MPRESS_OK) rc = preload_kernels();
+  rc = agree(c, rc, "map its peers");
+  if (rc != MPRESS_OK) {
+    destroy(c);
+    return rc;
+  }
+  *out = c;
+  return MPRESS_OK;
+}
+
+namespace mpress {
+namespace {
+
+// Transport 0: cuMem pool exported as a POSIX fd, passed with SCM_RIGHTS,
+// imported and mapped with peer access (no collective agreement here).
+int init_vmm_fd(mpress_ctx_s* c, const Driver* d, int rc) {
+  const int world = c->world, rank = c->source, device = c->device;
+  const uint64_t* partition = c->partition.data();
+  mpress_exchange_fn exchange = c->exchange;
+  void* exchange_user = c->exchange_user;
+  c->transport = MPRESS_TRANSPORT_VMM_FD;
 
   // 1. my pool = sum of every source's partition on me
   uint64_t pool = 0;
@@ -306,22 +418,11 @@ extern "C" int mpress_init(int device, int world, int rank, const uint64_t* part
   }
   for (int p = 0; p < world; ++p)
     if (fds[p] >= 0) close(fds[p]);
-
-  // 4. agree on success
-  if (rc == MPRESS_OK) rc = preload_kernels();
-  int32_t ok = rc == MPRESS_OK;
-  std::vector<int32_t> okv(world);
-  if (exchange(exchange_user, &ok, sizeof ok, okv.data()) != 0 && rc == MPRESS_OK)
-    rc = fail(MPRESS_ERR_SYS, "mpress_init: exchange failed");
-  for (int r = 0; r < world && rc == MPRESS_OK; ++r)
-    if (!okv[r]) rc = fail(MPRESS_ERR_PEER, "mpress_init: rank %d failed to map its peers", r);
-  if (rc != MPRESS_OK) {
-    destroy(c);
-    return rc;
-  }
-  *out = c;
-  return MPRESS_OK;
+  return rc;
 }
+
+}  // namespace
+}  // namespace mpress
 
 extern "C" int mpress_finalize(mpress_ctx_t* c) {
   if (!c) return MPRESS_OK;
@@ -389,6 +490,7 @@ extern "C" int mpress_get_option(const mpress_ctx_t* c, int key, int64_t* value)
     case MPRESS_OPT_MAX_CTAS: *value = c->max_ctas; return MPRESS_OK;
     case MPRESS_OPT_VARIANT: *value = c->variant; return MPRESS_OK;
     case MPRESS_OPT_ORDER: *value = c->order; return MPRESS_OK;
+    case MPRESS_OPT_TRANSPORT: *value = c->transport; return MPRESS_OK;
   }
   return fail(MPRESS_ERR_ARG, "unknown option %d", key);
 }

@@ -21,12 +21,14 @@ def _free_port():
     return port
 
 
-def _worker(rank, world, port, outdir, path):
+def _worker(rank, world, port, outdir, path, transport="fd"):
     import numpy as np
     import torch
     import torch.distributed as dist
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
+    if transport == "legacy":
+        os.environ["MPRESS_IPC"] = "legacy"   # CUDA IPC handles via the all-gather
     torch.cuda.set_device(0)
     dist.init_process_group("gloo", rank=rank, world_size=world)
     import oracle
@@ -43,6 +45,8 @@ def _worker(rank, world, port, outdir, path):
     err = ""
     try:
         ctx.set_option(mp.OPT_PATH, path)
+        want = mp.TRANSPORT_LEGACY_IPC if transport == "legacy" else mp.TRANSPORT_VMM_FD
+        assert ctx.get_option(mp.OPT_TRANSPORT) == want
         per_copy = [r // 2 for r in spare]
         pl = mp.plan(world, rank, per_copy, bwm[rank], sizes, 4096)
         o = oracle.plan(world, rank, per_copy, bwm[rank], sizes, 4096)
@@ -80,10 +84,10 @@ def _worker(rank, world, port, outdir, path):
     dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("path", [0, 1])
-def test_two_processes_one_gpu(path):
+@pytest.mark.parametrize("path,transport", [(0, "fd"), (1, "fd"), (0, "legacy")])
+def test_two_processes_one_gpu(path, transport):
     with tempfile.TemporaryDirectory() as d:
-        tmp.spawn(_worker, args=(2, _free_port(), d, path), nprocs=2, join=True)
+        tmp.spawn(_worker, args=(2, _free_port(), d, path, transport), nprocs=2, join=True)
         for r in range(2):
             assert open(os.path.join(d, "r%d.txt" % r)).read() == "ok"
 
