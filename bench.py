@@ -432,6 +432,10 @@ def main():
             "planner": planner, "other_configs": others,
             "parity": "round trip bit-exact vs generator (all %d tensors x %d ranks)" % (47 * mb, n),
             "per_rank_gbs": value / n,
+            "transport": {mp.TRANSPORT_LOCAL: "local (mpress_init_local)",
+                          mp.TRANSPORT_VMM_FD: "cuMem pools, POSIX fds over SCM_RIGHTS",
+                          mp.TRANSPORT_LEGACY_IPC: "cudaMalloc pools, CUDA IPC handles"}.get(
+                              ctx.get_option(mp.OPT_TRANSPORT), "?"),
             "link": ("HBM loopback (1 GPU: the peers are pools on the same GPU, bound by the HBM copy "
                      "roofline, not NVLink)" if n == 1 else
                      "NVLink 5 / NVSwitch (every rank swaps to all others; bound by 900 GB/s nominal, "
