@@ -52,7 +52,7 @@ def parse():
     ap.add_argument("--path", default="direct", choices=["direct", "bulk", "ce"])
     ap.add_argument("--max-ctas", type=int, default=0)
     ap.add_argument("--micro-batches", type=int, default=MICRO_BATCHES)
-    ap.add_argument("--e2e-steps", type=int, default=6)
+    ap.add_argument("--e2e-steps", type=int, default=16)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
     ap.add_argument("--gemm-cap", type=int, default=64,
@@ -502,14 +502,48 @@ def other_configs(args, mp, device):
                     ts.append(e0.elapsed_time(e1))
             ms = statistics.median(ts)
             bad = sum(synth_dev.check(t, 1000 * (len(out) + 1), i) for i, t in enumerate(dst))
-            out.append({"config": name, "bytes": sum(sizes), "stripes": len(pl.stripes),
-                        "round_trip_ms": ms, "gbs": 2 * sum(sizes) / (ms / 1e3) / 1e9,
-                        "bit_exact": bad == 0})
+            row = {"config": name, "bytes": sum(sizes), "stripes": len(pl.stripes),
+                   "round_trip_ms": ms, "gbs": 2 * sum(sizes) / (ms / 1e3) / 1e9,
+                   "bit_exact": bad == 0}
+            if sum(sizes) <= 256 << 20:
+                row.update(graph_round_trip(ctx, mp, pl, src, dst, s, synth_dev, 1000 * (len(out) + 1)))
+            out.append(row)
             del src, dst
             torch.cuda.empty_cache()
         finally:
             ctx.finalize()
     return out
+
+
+def graph_round_trip(ctx, mp, pl, src, dst, s, synth_dev, seed):
+    """The same round trip captured once into a CUDA graph (swap-out +
+    swap-in, graph handle) and replayed: what a small, launch-bound swap
+    costs when the pipeline step is a graph.  Median of 5 after 2 warm-ups."""
+    import torch
+    for t in dst:
+        t.zero_()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        h = ctx.swap_out(pl, src)
+        ctx.swap_in(h, dst)
+    ts = []
+    with torch.cuda.stream(s):
+        for r in range(7):
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record()
+            g.replay()
+            e1.record()
+            torch.cuda.synchronize()
+            if r >= 2:
+                ts.append(e0.elapsed_time(e1))
+    bad = sum(synth_dev.check(t, seed, i) for i, t in enumerate(dst))
+    del g
+    h.free()
+    ms = statistics.median(ts)
+    nbytes = sum(int(t.numel()) for t in src)
+    return {"graph_round_trip_ms": ms, "graph_gbs": 2 * nbytes / (ms / 1e3) / 1e9,
+            "graph_bit_exact": bad == 0}
 
 
 def planner_timing(mp, world, source, spare, bw, sizes):
@@ -622,55 +656,62 @@ def run_e2e(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, stream,
     copies the micro-batches' inputs host->device, swaps them out and in, and
     reads the restored tensors back device->host.  With N > 1 ranks on one
     host each rank stages 2 micro-batches (2 x 900 MiB pinned in and out) so N
-    ranks do not pin N x 14 GiB of host memory."""
+    ranks do not pin N x 14 GiB of host memory.
+
+    Pipelined per micro-batch on three streams (host->device, swap,
+    device->host) over two device buffer sets: micro-batch m's swap-out starts
+    as soon as its own upload lands, and its download starts as soon as its
+    own swap-in is done, so both PCIe directions stay busy and the pipeline
+    fills and drains by one micro-batch, not one step.  `pcie` reports the
+    copies alone (no swap) on the same buffers: the ceiling e2e can reach."""
     import torch
     mb = len(src) if n == 1 else min(2, len(src))
     src, dst = src[:mb], dst[:mb]
     steps = max(1, args.e2e_steps)
+    nt = len(sizes)
     hsrc = [[torch.empty(s, dtype=torch.uint8, pin_memory=True) for s in sizes] for _ in range(mb)]
     hdst = [[torch.empty(s, dtype=torch.uint8, pin_memory=True) for s in sizes] for _ in range(mb)]
     for m in range(mb):
-        for i in range(len(sizes)):
+        for i in range(nt):
             hsrc[m][i].copy_(src[m][i])
     torch.cuda.synchronize()
 
-    # Two device buffer sets and three streams: step k+1's host->device copy
-    # overlaps step k's swap and step k-1's device->host copy, so both PCIe
-    # directions work at once (copies overlapped with compute on side streams).
     srcs = [src, [[torch.empty_like(t) for t in row] for row in src]]
     dsts = [dst, [[torch.empty_like(t) for t in row] for row in dst]]
     h2d, d2h = torch.cuda.Stream(), torch.cuda.Stream()
-    swap_done = [None, None]   # per set: after the swap-ins (src read, dst written)
-    d2h_done = [None, None]    # per set: after the device->host copy (dst read)
+    src_free = [[None] * mb for _ in range(2)]   # (set, m): its swap-out has read src
+    dst_free = [[None] * mb for _ in range(2)]   # (set, m): its download has read dst
 
     def step(k):
         x = k % 2
-        if swap_done[x] is not None:
-            h2d.wait_event(swap_done[x])           # set x's previous swap-outs read src
-        with torch.cuda.stream(h2d):
-            for m in range(mb):
-                for i in range(len(sizes)):
-                    srcs[x][m][i].copy_(hsrc[m][i], non_blocking=True)
-        h2d_ev = torch.cuda.Event()
-        h2d_ev.record(h2d)
-        stream.wait_event(h2d_ev)
-        if d2h_done[x] is not None:
-            stream.wait_event(d2h_done[x])         # set x's previous results were read
         pl = mp.plan(world, source, per_copy, bw, sizes)
-        hs = [ctx.swap_out(pl, srcs[x][m], stream=stream) for m in range(mb)]
+        hs = []
         for m in range(mb):
+            if src_free[x][m] is not None:
+                h2d.wait_event(src_free[x][m])
+            with torch.cuda.stream(h2d):
+                for i in range(nt):
+                    srcs[x][m][i].copy_(hsrc[m][i], non_blocking=True)
+            up = torch.cuda.Event()
+            up.record(h2d)
+            stream.wait_event(up)
+            hs.append(ctx.swap_out(pl, srcs[x][m], stream=stream))
+            src_free[x][m] = torch.cuda.Event()
+            src_free[x][m].record(stream)
+        for m in range(mb):
+            if dst_free[x][m] is not None:
+                stream.wait_event(dst_free[x][m])
             ctx.swap_in(hs[m], dsts[x][m], stream=stream)
+            done = torch.cuda.Event()
+            done.record(stream)
+            d2h.wait_event(done)
+            with torch.cuda.stream(d2h):
+                for i in range(nt):
+                    hdst[m][i].copy_(dsts[x][m][i], non_blocking=True)
+            dst_free[x][m] = torch.cuda.Event()
+            dst_free[x][m].record(d2h)
         for h in hs:
             h.free()
-        swap_done[x] = torch.cuda.Event()
-        swap_done[x].record(stream)
-        d2h.wait_event(swap_done[x])
-        with torch.cuda.stream(d2h):
-            for m in range(mb):
-                for i in range(len(sizes)):
-                    hdst[m][i].copy_(dsts[x][m][i], non_blocking=True)
-        d2h_done[x] = torch.cuda.Event()
-        d2h_done[x].record(d2h)
 
     step(0)
     torch.cuda.synchronize()
@@ -678,10 +719,12 @@ def run_e2e(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, stream,
         dist.barrier()
     e0 = torch.cuda.Event(enable_timing=True)
     e1 = torch.cuda.Event(enable_timing=True)
-    e0.record(h2d)
+    e0.record(stream)
+    h2d.wait_stream(stream)
     for k in range(steps):
         step(k + 1)
-    e1.record(d2h)
+    stream.wait_stream(d2h)
+    e1.record(stream)
     torch.cuda.synchronize()
     ms = e0.elapsed_time(e1)
     t = torch.tensor([ms], dtype=torch.float64)
@@ -691,12 +734,56 @@ def run_e2e(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, stream,
     per = 2 * mb * sum(sizes)
     import numpy as np
     ok = all(np.array_equal(hdst[m][i].numpy(), hsrc[m][i].numpy())
-             for m in (0, mb - 1) for i in range(len(sizes)))
+             for m in (0, mb - 1) for i in range(nt))
+    try:
+        pcie = leg_pcie(srcs[0], dsts[0], hsrc, hdst, h2d, d2h, stream)
+    except Exception as exc:  # pragma: no cover - reported, not hidden
+        pcie = {"error": "%s: %s" % (type(exc).__name__, exc)}
     return {"value": n * per / (ms / 1e3) / 1e9, "unit": "GB/s",
             "h2d_bytes_per_step": mb * sum(sizes), "d2h_bytes_per_step": mb * sum(sizes),
             "micro_batches": mb,
             "steps": steps, "ms_per_step": ms, "round_trip_ok": bool(ok),
-            "pipelining": "H2D of step k+1 || swap of step k || D2H of step k-1 (3 streams, 2 buffer sets)"}
+            "pipelining": "per micro-batch: upload(m) -> swap-out(m); swap-in(m) -> download(m); "
+                          "3 streams, 2 device buffer sets",
+            "pcie": pcie,
+            "frac_of_pcie_duplex": ((per / (ms / 1e3) / 1e9) / pcie["duplex_gbs"]
+                                    if "duplex_gbs" in pcie else None)}
+
+
+def leg_pcie(src, dst, hsrc, hdst, h2d, d2h, stream, reps=3):
+    """The e2e ceiling on this box: the same pinned copies with no swap --
+    upload alone, download alone, and both at once (GB/s of copied bytes,
+    best of `reps`).  e2e moves one upload and one download byte per swapped
+    byte, so its ceiling is duplex_gbs."""
+    import torch
+
+    def timed(up, down):
+        best = None
+        for _ in range(reps):
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            h2d.wait_stream(stream)
+            d2h.wait_stream(stream)
+            for m in range(len(src)):
+                for i in range(len(src[m])):
+                    if up:
+                        with torch.cuda.stream(h2d):
+                            src[m][i].copy_(hsrc[m][i], non_blocking=True)
+                    if down:
+                        with torch.cuda.stream(d2h):
+                            hdst[m][i].copy_(dst[m][i], non_blocking=True)
+            stream.wait_stream(h2d)
+            stream.wait_stream(d2h)
+            e1.record(stream)
+            torch.cuda.synchronize()
+            ms = e0.elapsed_time(e1)
+            best = ms if best is None else min(best, ms)
+        nbytes = sum(t.numel() for row in src for t in row) * (int(up) + int(down))
+        return nbytes / (best / 1e3) / 1e9
+
+    return {"h2d_gbs": timed(True, False), "d2h_gbs": timed(False, True),
+            "duplex_gbs": timed(True, True)}
 
 
 if __name__ == "__main__":

@@ -403,8 +403,12 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
  * 8 = 256x4 with L2 evict-first loads, 9 = 128x8 (32-byte vectors, used
  * only when every address is 32-byte aligned, else the 16-byte shape);
  * bulk: 0 = 6 slots x 32 KiB, 1 = 12 x 16 KiB, 2 = 3 x 64 KiB;
+ * copy engines: 0 = cudaMemcpyAsync per stripe on one side stream per peer,
+ * 1 = the whole swap as one cudaMemcpyBatchAsync on the swap stream (not on
+ * the legacy NULL stream);
  * MPRESS_VARIANT_AUTO (-1, default) = direct 7 when the grid is capped at
- * <= one CTA per SM (small CTAs co-reside with a GEMM), else 5.
+ * <= one CTA per SM (small CTAs co-reside with a GEMM), else 5; bulk 0; copy
+ * engines 0.
  * MPRESS_OPT_ORDER: chunk order inside one launch -- 0 = interleave the
  * peers by a weighted round robin, so every peer link carries its share of
  * the swap at every moment (default; needed when several sources share
@@ -472,6 +476,29 @@ MPRESS_API int mpress_swap_out(mpress_ctx_t* ctx, const mpress_plan_t* plan,
  */
 MPRESS_API int mpress_swap_in(mpress_ctx_t* ctx, mpress_handle_t* handle, void* const* dst,
                    void* stream);
+
+/*
+ * CUDA graph capture.  mpress_swap_out / mpress_swap_in / mpress_wait may be
+ * called while their streams are being captured (cudaStreamBeginCapture,
+ * torch.cuda.graph), so a pipeline step that swaps can be captured and
+ * replayed as one graph launch (no per-swap host cost on the replay).  A
+ * swap-out enqueued on a capturing stream makes a GRAPH HANDLE:
+ *   - its stash slices are taken at capture time and stay held until
+ *     mpress_handle_free (every replay writes and reads them again); eager
+ *     swaps of the same context use other slices;
+ *   - its swap-in must be captured into the same capture (else
+ *     MPRESS_ERR_STATE), at most once; an eager handle cannot be swapped in
+ *     under capture (MPRESS_ERR_STATE);
+ *   - mpress_wait inside the capture joins the consumer stream on the
+ *     capture's own event; outside it, waits for the latest replay;
+ *   - mpress_query reports the latest replay's completion (1 before any
+ *     replay) and does not advance the state; do not call it while a capture
+ *     is running;
+ *   - mpress_handle_free releases the slices, fenced by the latest replay's
+ *     swap-in (force is needed if no swap-in was captured).  Free graph
+ *     handles only once their graph will not be launched again.
+ * Replays move the bytes the captured pointers hold at replay time.
+ */
 
 /* Make `consumer` wait (cudaStreamWaitEvent, enqueue-only) for the handle's
  * latest operation: the swap-out if no swap-in was issued, else the swap-in. */

@@ -69,7 +69,10 @@ using EvPool = std::shared_ptr<std::vector<cudaEvent_t>>;
 struct Fence {
   uint64_t off, len;
   EvRef ev;
+  cudaStream_t stream;   // where `ev` was recorded; no_stream() if unknown / a graph
 };
+// Fence::stream of a fence that must always be waited on.
+inline cudaStream_t no_stream() { return reinterpret_cast<cudaStream_t>(~uintptr_t(0)); }
 
 // This source's partition of one peer's stash pool (R21).
 struct Partition {
@@ -117,7 +120,17 @@ struct mpress_handle_s {
   std::vector<uint64_t> slice_len;    // [world]
   mpress::EvRef out_done;
   mpress::EvRef in_done;
+  cudaStream_t out_stream = nullptr;  // the swap-out's stream (a swap-in there needs no wait)
   bool slices_held = false;
+  // Graph handle: the swap-out was enqueued while its stream was being
+  // captured into a CUDA graph.  Every replay re-runs the captured kernels
+  // into the same slices, so the slices stay held until mpress_handle_free.
+  // out_done / in_done are capture-internal (joins inside the capture);
+  // out_ext / in_ext are external event-record nodes, re-recorded by every
+  // replay, which queries, eager waits and slice fences use.
+  bool graph = false;
+  mpress::EvRef out_ext;
+  mpress::EvRef in_ext;
 };
 
 namespace mpress {

@@ -473,7 +473,8 @@ extern "C" int mpress_set_option(mpress_ctx_t* c, int key, int64_t value) {
       c->order = (int)value;
       return MPRESS_OK;
     case MPRESS_OPT_VARIANT: {
-      const int nvar = c->path == MPRESS_PATH_BULK ? kBulkVariants : kDirectVariants;
+      const int nvar = c->path == MPRESS_PATH_BULK ? kBulkVariants
+                       : c->path == MPRESS_PATH_CE ? kCeVariants : kDirectVariants;
       if (value != MPRESS_VARIANT_AUTO && (value < 0 || value >= nvar))
         return fail(MPRESS_ERR_ARG, "variant %lld out of range for path %d", (long long)value, c->path);
       c->variant = (int)value;

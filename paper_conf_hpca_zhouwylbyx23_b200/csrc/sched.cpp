@@ -38,6 +38,18 @@ EvRef take_event(mpress_ctx_s* c) {
 
 namespace {
 
+// Fence lists are reaped only past this length: a fence recorded on the
+// stream of the next swap-out costs nothing (stream order covers it), so the
+// event queries of a reap are spent only when the list grows.
+constexpr size_t kReapAt = 32;
+
+// Can work enqueued on `s` rely on plain stream order after work enqueued on
+// `prev`?  Not for the per-thread default stream (one handle value, one stream
+// per thread) or unknown streams.
+bool same_stream(cudaStream_t prev, cudaStream_t s) {
+  return prev == s && s != cudaStreamPerThread && s != no_stream();
+}
+
 // Drop the fences whose swap-in has completed (oldest first; stops at the
 // first one still pending, so the cost is O(1) amortised).
 void reap_fences(Partition* part) {
@@ -96,6 +108,36 @@ int cuda_fail(cudaError_t e, const char* what) {
   return fail(MPRESS_ERR_CUDA, "%s: %s", what, cudaGetErrorString(e));
 }
 
+// Is `s` being captured into a CUDA graph (cudaStreamBeginCapture /
+// torch.cuda.graph)?  Capture changes what an enqueue-only call may do: no
+// event queries (they are not allowed while a global-mode capture runs), and
+// events from outside the capture are waited on as external nodes.
+bool capturing(cudaStream_t s) {
+  cudaStreamCaptureStatus st = cudaStreamCaptureStatusNone;
+  if (cudaStreamIsCapturing(s, &st) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return st == cudaStreamCaptureStatusActive;
+}
+
+// Record `ev` on `s`; under capture first record `ext` as an external
+// event-record node (re-recorded by every replay of the graph).  The
+// external node goes first so that a join on `ev` also joins it: a node after
+// the last join would be work the capture never rejoins.
+int record_done(mpress_ctx_s* c, cudaStream_t s, bool graph, EvRef* ev, EvRef* ext, const char* what) {
+  if (graph) {
+    *ext = take_event(c);
+    if (!*ext) return fail(MPRESS_ERR_CUDA, "cudaEventCreate failed");
+    const cudaError_t e = cudaEventRecordWithFlags(ext->get(), s, cudaEventRecordExternal);
+    if (e != cudaSuccess) return cuda_fail(e, what);
+  }
+  *ev = take_event(c);
+  if (!*ev) return fail(MPRESS_ERR_CUDA, "cudaEventCreate failed");
+  const cudaError_t e = cudaEventRecord(ev->get(), s);
+  return e == cudaSuccess ? MPRESS_OK : cuda_fail(e, what);
+}
+
 // Move every descriptor on `stream` with the context's path.
 int run_copy(mpress_ctx_s* c, int dir, const std::vector<CopyDesc>& d,
              const std::vector<int>& desc_peer, cudaStream_t stream) {
@@ -105,8 +147,9 @@ int run_copy(mpress_ctx_s* c, int dir, const std::vector<CopyDesc>& d,
                        c->order == MPRESS_ORDER_INTERLEAVE ? desc_peer.data() : nullptr, d.size(), c->max_ctas,
                        stream, &c->last_launches);
 
-  // Copy-engine comparator: cudaMemcpyAsync per stripe, one side stream per
-  // peer so the engines of different peers overlap; fork/join by events.
+  // Copy-engine comparator, variant 1: the whole swap as one
+  // cudaMemcpyBatchAsync on `stream` (CUDA 12.8+); the driver spreads the
+  // copies over the copy engines.  Stream-ordered source access.
   if (c->ce_streams.empty()) {
     c->ce_streams.assign(c->world, nullptr);
     for (int p = 0; p < c->world; ++p) {
@@ -114,6 +157,46 @@ int run_copy(mpress_ctx_s* c, int dir, const std::vector<CopyDesc>& d,
       if (e != cudaSuccess) return cuda_fail(e, "cudaStreamCreate (copy-engine path)");
     }
   }
+  if (c->variant == 1) {
+    const size_t n = d.size();
+    if (n == 0) return MPRESS_OK;
+    // The batch call rejects the legacy NULL stream: there, run it on a side
+    // stream (the source's slot, which no stripe uses) forked and joined by
+    // events.
+    const bool legacy = stream == nullptr || stream == cudaStreamLegacy;
+    cudaStream_t bs = legacy ? c->ce_streams[c->source] : stream;
+    EvRef fork, join;
+    if (legacy) {
+      fork = take_event(c);
+      join = take_event(c);
+      if (!fork || !join) return fail(MPRESS_ERR_CUDA, "cudaEventCreate failed");
+      cudaEventRecord(fork.get(), stream);
+      cudaStreamWaitEvent(bs, fork.get(), 0);
+    }
+    std::vector<void*> dsts(n), srcs(n);
+    std::vector<size_t> lens(n);
+    for (size_t i = 0; i < n; ++i) {
+      dsts[i] = d[i].dst;
+      srcs[i] = const_cast<void*>(d[i].src);
+      lens[i] = d[i].len;
+    }
+    cudaMemcpyAttributes attr;
+    std::memset(&attr, 0, sizeof(attr));
+    attr.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
+    size_t attr_idx = 0, fail_idx = SIZE_MAX;
+    const cudaError_t e = cudaMemcpyBatchAsync(dsts.data(), srcs.data(), lens.data(), n, &attr, &attr_idx, 1,
+                                               &fail_idx, bs);
+    if (legacy) {
+      cudaEventRecord(join.get(), bs);
+      cudaStreamWaitEvent(stream, join.get(), 0);
+    }
+    if (e != cudaSuccess) return cuda_fail(e, "cudaMemcpyBatchAsync (copy-engine path)");
+    return MPRESS_OK;
+  }
+
+  // Copy-engine comparator, variant 0 (default): cudaMemcpyAsync per stripe,
+  // one side stream per peer so the engines of different peers overlap;
+  // fork/join by events.
   EvRef fork = take_event(c);
   if (!fork) return fail(MPRESS_ERR_CUDA, "cudaEventCreate failed");
   cudaEventRecord(fork.get(), stream);
@@ -159,9 +242,11 @@ extern "C" int mpress_swap_out(mpress_ctx_t* c, const mpress_plan_t* plan_, void
   MP_TRY(check_ptrs(tensors, info.n_tensors, "mpress_swap_out(tensors)"));
   DeviceGuard g(c->device);
   cudaStream_t stream = static_cast<cudaStream_t>(stream_);
+  const bool graph = capturing(stream);
 
   auto* h = new mpress_handle_s();
   h->ctx = c;
+  h->graph = graph;
   h->slice_off.assign(c->world, UINT64_MAX);
   h->slice_len.assign(c->world, 0);
   int rc = MPRESS_OK;
@@ -172,7 +257,7 @@ extern "C" int mpress_swap_out(mpress_ctx_t* c, const mpress_plan_t* plan_, void
       rc = fail(MPRESS_ERR_PEER, "mpress_swap_out: peer %d is not mapped (partition 0)", p);
       break;
     }
-    reap_fences(&part);
+    if (!graph && part.fences.size() > kReapAt) reap_fences(&part);
     const uint64_t len = units[p] * info.granule;
     uint64_t off;
     if (!alloc_slice(&part, len, &off)) {
@@ -182,9 +267,13 @@ extern "C" int mpress_swap_out(mpress_ctx_t* c, const mpress_plan_t* plan_, void
     }
     h->slice_off[p] = off;
     h->slice_len[p] = len;
-    // earlier swap-ins still reading these bytes: order this swap-out after them
+    // earlier swap-ins still reading these bytes: order this swap-out after
+    // them -- free when they ran on this stream; under capture the waits
+    // become external wait nodes (every replay waits for the fence's latest
+    // record)
     for (const Fence& f : part.fences)
-      if (f.off < off + len && off < f.off + f.len) cudaStreamWaitEvent(stream, f.ev.get(), 0);
+      if (f.off < off + len && off < f.off + f.len && (graph || !same_stream(f.stream, stream)))
+        cudaStreamWaitEvent(stream, f.ev.get(), graph ? cudaEventWaitExternal : 0);
   }
   if (rc != MPRESS_OK) {
     for (int p = 0; p < c->world; ++p)
@@ -208,21 +297,19 @@ extern "C" int mpress_swap_out(mpress_ctx_t* c, const mpress_plan_t* plan_, void
     dp[i] = (int)s.peer;
   }
   if (after) cudaStreamWaitEvent(stream, static_cast<cudaEvent_t>(after), 0);
-  h->out_done = take_event(c);
-  rc = h->out_done ? run_copy(c, kDirOut, d, dp, stream) : fail(MPRESS_ERR_CUDA, "cudaEventCreate failed");
-  if (rc == MPRESS_OK) {
-    cudaError_t e = cudaEventRecord(h->out_done.get(), stream);
-    if (e != cudaSuccess) rc = cuda_fail(e, "cudaEventRecord(out_done)");
-  }
+  rc = run_copy(c, kDirOut, d, dp, stream);
+  if (rc == MPRESS_OK) rc = record_done(c, stream, graph, &h->out_done, &h->out_ext, "cudaEventRecord(out_done)");
   if (rc != MPRESS_OK) {
-    // Kernels may already be queued: keep the slices fenced by a sync.
-    cudaStreamSynchronize(stream);
+    // Kernels may already be queued: keep the slices fenced by a sync (a
+    // failed capture is invalidated anyway: nothing was enqueued for real).
+    if (!graph) cudaStreamSynchronize(stream);
     for (int p = 0; p < c->world; ++p)
       if (h->slice_off[p] != UINT64_MAX) free_slice(&c->parts[p], h->slice_off[p], h->slice_len[p]);
     delete h;
     return rc;
   }
   h->state = MPRESS_STATE_OUT_PENDING;
+  h->out_stream = graph ? no_stream() : stream;
   c->handles.insert(h);
   *out = h;
   return MPRESS_OK;
@@ -234,9 +321,16 @@ extern "C" int mpress_swap_in(mpress_ctx_t* c, mpress_handle_t* h, void* const* 
   if (h->ctx != c || !c->handles.count(h)) return fail(MPRESS_ERR_ARG, "mpress_swap_in: handle not of this context");
   if (h->state != MPRESS_STATE_OUT_PENDING && h->state != MPRESS_STATE_OUT)
     return fail(MPRESS_ERR_STATE, "mpress_swap_in: handle is in state %d, not swapped out", h->state);
+  if (h->graph && h->in_done)
+    return fail(MPRESS_ERR_STATE, "mpress_swap_in: the graph handle's swap-in was already captured");
   MP_TRY(check_ptrs(dst, h->n_tensors, "mpress_swap_in(dst)"));
   DeviceGuard g(c->device);
   cudaStream_t stream = static_cast<cudaStream_t>(stream_);
+  if (capturing(stream) != h->graph)
+    return fail(MPRESS_ERR_STATE, h->graph ? "mpress_swap_in: the swap-out was captured into a graph; capture the "
+                                             "swap-in into the same capture"
+                                           : "mpress_swap_in: the swap-out ran eagerly; it cannot be swapped in "
+                                             "under graph capture");
 
   std::vector<CopyDesc>& d = c->scratch_desc;
   std::vector<int>& dp = c->scratch_peer;
@@ -249,15 +343,16 @@ extern "C" int mpress_swap_in(mpress_ctx_t* c, mpress_handle_t* h, void* const* 
     d[i].len = s.len;
     dp[i] = (int)s.peer;
   }
-  cudaStreamWaitEvent(stream, h->out_done.get(), 0);
-  EvRef in_done = take_event(c);
-  if (!in_done) return fail(MPRESS_ERR_CUDA, "cudaEventCreate failed");
+  if (h->graph || !same_stream(h->out_stream, stream)) cudaStreamWaitEvent(stream, h->out_done.get(), 0);
   int rc = run_copy(c, kDirIn, d, dp, stream);
   if (rc != MPRESS_OK) return rc;
-  cudaError_t e = cudaEventRecord(in_done.get(), stream);
-  if (e != cudaSuccess) return cuda_fail(e, "cudaEventRecord(in_done)");
+  EvRef in_done, in_ext;
+  MP_TRY(record_done(c, stream, h->graph, &in_done, &in_ext, "cudaEventRecord(in_done)"));
   h->in_done = in_done;
+  h->in_ext = in_ext;
   h->state = MPRESS_STATE_IN_PENDING;
+  // A graph handle keeps its slices: every replay writes and reads them again.
+  if (h->graph) return MPRESS_OK;
 
   // Release the slices now; their bytes stay fenced by the swap-in's event
   // until it completes (the table entry is "updated when it completes").
@@ -272,7 +367,7 @@ extern "C" int mpress_swap_in(mpress_ctx_t* c, mpress_handle_t* h, void* const* 
       if (it->off >= a && it->off + it->len <= b) it = fs.erase(it);
       else ++it;
     }
-    fs.push_back({h->slice_off[p], h->slice_len[p], in_done});
+    fs.push_back({h->slice_off[p], h->slice_len[p], in_done, stream});
     free_slice(&c->parts[p], h->slice_off[p], h->slice_len[p]);
   }
   h->slices_held = false;
@@ -283,7 +378,11 @@ extern "C" int mpress_wait(mpress_ctx_t* c, mpress_handle_t* h, void* consumer) 
   if (!c || !h || h->ctx != c) return fail(MPRESS_ERR_ARG, "mpress_wait: bad argument");
   std::lock_guard<std::mutex> lk(c->mu);
   DeviceGuard g(c->device);
-  const EvRef& e = (h->state == MPRESS_STATE_IN_PENDING || h->state == MPRESS_STATE_IN) ? h->in_done : h->out_done;
+  const bool in = h->state == MPRESS_STATE_IN_PENDING || h->state == MPRESS_STATE_IN;
+  // A graph handle: inside the capture, join on the capture's own event;
+  // outside it, wait for the latest replay (the external record).
+  const bool ext = h->graph && !capturing(static_cast<cudaStream_t>(consumer));
+  const EvRef& e = ext ? (in ? h->in_ext : h->out_ext) : (in ? h->in_done : h->out_done);
   if (!e) return fail(MPRESS_ERR_STATE, "mpress_wait: nothing enqueued");
   cudaError_t r = cudaStreamWaitEvent(static_cast<cudaStream_t>(consumer), e.get(), 0);
   if (r != cudaSuccess) return cuda_fail(r, "mpress_wait: cudaStreamWaitEvent");
@@ -294,6 +393,13 @@ extern "C" int mpress_query(mpress_ctx_t* c, mpress_handle_t* h) {
   if (!c || !h || h->ctx != c) return fail(MPRESS_ERR_ARG, "mpress_query: bad argument");
   std::lock_guard<std::mutex> lk(c->mu);
   DeviceGuard g(c->device);
+  if (h->graph) {  // the latest replay's completion; the state does not move
+    const EvRef& x = h->in_ext ? h->in_ext : h->out_ext;
+    const cudaError_t r = cudaEventQuery(x.get());
+    if (r == cudaSuccess) return 1;
+    if (r == cudaErrorNotReady) { cudaGetLastError(); return 0; }
+    return cuda_fail(r, "mpress_query: cudaEventQuery");
+  }
   cudaEvent_t e;
   int next;
   switch (h->state) {
@@ -321,6 +427,20 @@ extern "C" int mpress_handle_free(mpress_ctx_t* c, mpress_handle_t* h, int force
   std::lock_guard<std::mutex> lk(c->mu);
   if (h->ctx != c || !c->handles.count(h)) return fail(MPRESS_ERR_ARG, "mpress_handle_free: handle not of this context");
   DeviceGuard g(c->device);
+  if (h->graph) {
+    // The caller no longer replays the graph.  Release the slices fenced by
+    // the latest replay's swap-in (or swap-out, if no swap-in was captured).
+    if (!h->in_ext && !force)
+      return fail(MPRESS_ERR_STATE, "mpress_handle_free: graph handle without a captured swap-in; force to drop "
+                                    "the stashed data");
+    const EvRef& fence = h->in_ext ? h->in_ext : h->out_ext;
+    for (int p = 0; p < c->world; ++p) {
+      if (h->slice_off[p] == UINT64_MAX) continue;
+      c->parts[p].fences.push_back({h->slice_off[p], h->slice_len[p], fence, no_stream()});
+      free_slice(&c->parts[p], h->slice_off[p], h->slice_len[p]);
+    }
+    h->slices_held = false;
+  }
   if (h->slices_held) {
     if (!force)
       return fail(MPRESS_ERR_STATE, "mpress_handle_free: data still only in the stash (state %d); swap in or force", h->state);

@@ -97,9 +97,11 @@ def sizes_sweep():
     s = torch.cuda.Stream()
     for peers_n in (1, 3, 7):
         for size in workloads.cfg4_sizes():
-            ctx, pl, src, dst = setup([size], peers_n)
-            for name in ("direct", "bulk", "ce"):
-                ctx.set_option(mp.OPT_PATH, PATHS[name])
+            ctx, pl, src, dst = setup([size], peers_n, copies=2)
+            for name in ("direct", "bulk", "ce", "ce_batch"):
+                ctx.set_option(mp.OPT_PATH, PATHS[name.split("_")[0]])
+                if name == "ce_batch":
+                    ctx.set_option(mp.OPT_VARIANT, 1)   # one cudaMemcpyBatchAsync
                 reps = 20 if size < (256 << 20) else 5
                 to, ti = time_swaps(ctx, pl, src, dst, reps, s)
                 # back to back: R swap pairs enqueued while the GPU is busy, so
@@ -119,11 +121,31 @@ def sizes_sweep():
                 torch.cuda.synchronize()
                 warm.free()
                 pair_us = e0.elapsed_time(e1) * 1e3 / R
+                graph_us = None
+                if name != "ce_batch":
+                    # the pair captured once into a CUDA graph, one replay timed
+                    g = torch.cuda.CUDAGraph()
+                    with torch.cuda.graph(g, stream=s):
+                        gh = ctx.swap_out(pl, src)
+                        ctx.swap_in(gh, dst)
+                    ts = []
+                    with torch.cuda.stream(s):
+                        for r in range(12):
+                            e0.record()
+                            g.replay()
+                            e1.record()
+                            torch.cuda.synchronize()
+                            if r >= 2:
+                                ts.append(e0.elapsed_time(e1) * 1e3)
+                    del g
+                    gh.free()
+                    graph_us = statistics.median(ts)
                 print(json.dumps({"sweep": "sizes", "peers": peers_n, "bytes": size, "path": name,
                                   "out_gbs": size / to / 1e6, "in_gbs": size / ti / 1e6,
                                   "out_us": to * 1e3, "in_us": ti * 1e3,
                                   "b2b_pair_us": pair_us,
-                                  "b2b_gbs": 2 * size / pair_us / 1e3}), flush=True)
+                                  "b2b_gbs": 2 * size / pair_us / 1e3,
+                                  "graph_pair_us": graph_us}), flush=True)
             ctx.finalize()
             del src, dst
             torch.cuda.empty_cache()
