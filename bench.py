@@ -58,6 +58,9 @@ def parse():
     ap.add_argument("--gemm-cap", type=int, default=64,
                     help="swap grid cap (CTAs = SMs touched) while the concurrent GEMM runs")
     ap.add_argument("--no-gemm", action="store_true")
+    ap.add_argument("--gemm-n", type=int, default=8192, help="GEMM size of the N>1 config-5 leg")
+    ap.add_argument("--no-cfg5", action="store_true",
+                    help="N>1: skip the config-5 leg (imbalanced swap + GEMM on every rank)")
     ap.add_argument("--no-configs", action="store_true",
                     help="skip the other BASELINE configs (1, 3, 4) reported beside the headline")
     return ap.parse_args()
@@ -407,6 +410,9 @@ def main():
     e2e = leg(run_e2e, args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap_stream, n, dist)
     gemm = None if args.no_gemm else leg(gemm_interference, args, ctx, mp, world, source, per_copy, bw,
                                          sizes, src, dst, swap_stream, n, dist)
+    cfg5 = None
+    if n > 1 and not args.no_gemm and not args.no_cfg5:
+        cfg5 = leg(cfg5_leg, args, mp, rank, n, local_rank, dist)
     others = None
     if n == 1 and not args.no_configs:
         del src, dst
@@ -429,7 +435,7 @@ def main():
             "per_direction_gbs": per_dir,
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": launches[0], "clocks": clk, "gemm_slowdown": gemm,
-            "planner": planner, "other_configs": others,
+            "planner": planner, "other_configs": others, "cfg5": cfg5,
             "parity": "round trip bit-exact vs generator (all %d tensors x %d ranks)" % (47 * mb, n),
             "per_rank_gbs": value / n,
             "transport": {mp.TRANSPORT_LOCAL: "local (mpress_init_local)",
@@ -647,8 +653,146 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
             "swap_path": args.path, "swap_max_ctas": args.gemm_cap,
             "swap_gbs_during": statistics.median(swap_gbs),
             "gemms_counted": len(during),
-            "note": "N=1 loopback: the swap's bytes also load the GEMM's HBM (2 B per swapped "
-                    "byte), a harsher case than NVLink (1 B of source HBM per byte)"}
+            "note": ("N=1 loopback: the swap's bytes also load the GEMM's HBM (2 B per swapped "
+                     "byte), a harsher case than NVLink (1 B of source HBM per byte)") if n == 1 else
+                    ("every rank swaps to all others while running the GEMM; max over ranks")}
+
+
+def cfg5_leg(args, mp, rank, n, device, dist):
+    """BASELINE config 5 (BJ:11, reading R20) at N GPUs: the
+    first half of the ranks are the heavy stages (sources), the second half
+    the light ones (pure importers).  Source s swaps (N/2 - s) Bert stage-0
+    micro-batch sets (900 MiB each) batched into one plan -- at N = 8:
+    3.52 / 2.64 / 1.76 / 0.88 GiB from sources 0-3 into peers 4-7 --
+    sequential partition (R12), grid capped at --gemm-cap CTAs, while EVERY
+    rank runs back-to-back bf16 GEMMs on its compute stream.  Reports each
+    source's swap GB/s (out + in) under contention and the GEMM slowdown on
+    sources and importers.  Every collective is reached by all ranks even if
+    a rank's local work fails (the failure is reported, not hung on)."""
+    import torch
+    from synth import device as synth_dev
+    from synth import workloads
+    H = n // 2
+    sources, peers = list(range(H)), list(range(H, n))
+    is_src = rank in sources
+    sizes = workloads.cfg2_sizes(H - rank) if is_src else []
+    spare = [0] * n
+    for p in peers:
+        spare[p] = 16 * GiB
+    bwm = [[1 if (s in sources and p in peers) else 0 for p in range(n)] for s in range(n)]
+    part = mp.partition_sequential(n, spare, bwm, [(s, workloads.cfg2_sizes(H - s), 1) for s in sources])
+    ctx = mp.Context.distributed(device, n, rank, part)
+    comp = torch.cuda.current_stream()
+    swap = torch.cuda.Stream()
+    M = args.gemm_n
+    G = 24
+    err = []
+
+    def guard(fn):
+        if err:
+            return None
+        try:
+            return fn()
+        except Exception as exc:  # pragma: no cover - reported below
+            err.append("rank %d: %s: %s" % (rank, type(exc).__name__, exc))
+            return None
+
+    st = {}
+
+    def setup():
+        rem = list(spare)
+        for s in sources:
+            if s == rank:
+                st["pl"] = mp.plan(n, rank, rem, bwm[rank], sizes)
+            for p in range(n):
+                rem[p] -= part[s][p]
+        ctx.set_option(mp.OPT_MAX_CTAS, args.gemm_cap)
+        st["a"] = torch.randn(M, M, dtype=torch.bfloat16, device="cuda")
+        st["b"] = torch.randn(M, M, dtype=torch.bfloat16, device="cuda")
+        st["c"] = torch.empty(M, M, dtype=torch.bfloat16, device="cuda")
+        if is_src:
+            st["src"] = [torch.empty(x, dtype=torch.uint8, device="cuda") for x in sizes]
+            st["dst"] = [torch.empty(x, dtype=torch.uint8, device="cuda") for x in sizes]
+            for i, t in enumerate(st["src"]):
+                synth_dev.fill(t, 5000 + rank, i)
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(swap)
+            h = ctx.swap_out(st["pl"], st["src"], stream=swap)
+            ctx.swap_in(h, st["dst"], stream=swap)
+            e1.record(swap)
+            h.free()
+            torch.cuda.synchronize()
+            st["per_swap_ms"] = e0.elapsed_time(e1)
+        torch.cuda.synchronize()
+
+    def gemms():
+        evs = []
+        for _ in range(G):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(comp)
+            torch.matmul(st["a"], st["b"], out=st["c"])
+            e1.record(comp)
+            evs.append((e0, e1))
+        return evs
+
+    alone, during, gbs = [], [], []
+
+    def run_alone():
+        evs = gemms()
+        torch.cuda.synchronize()
+        alone.extend(x.elapsed_time(y) for x, y in evs[4:])
+
+    def run_with_swap():
+        s0 = s1 = None
+        if is_src:
+            n_swap = int(2.0 * G * statistics.median(alone) / st["per_swap_ms"]) + 2
+            s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            s0.record(swap)
+            for _ in range(n_swap):
+                h = ctx.swap_out(st["pl"], st["src"], stream=swap)
+                ctx.swap_in(h, st["dst"], stream=swap)
+                h.free()
+            s1.record(swap)
+        evs = gemms()
+        torch.cuda.synchronize()
+        if is_src:
+            win = s0.elapsed_time(s1)
+            during.extend(x.elapsed_time(y) for x, y in evs[4:]
+                          if s0.elapsed_time(x) >= 0 and s0.elapsed_time(y) <= win)
+            gbs.append(2 * n_swap * sum(sizes) / win / 1e6)
+        else:   # importers: the middle of the run, inside every source's window
+            during.extend(x.elapsed_time(y) for x, y in evs[4:G - 4])
+
+    guard(setup)
+    for _ in range(4):
+        dist.barrier()
+        guard(run_alone)
+        dist.barrier()
+        guard(run_with_swap)
+    bad = 0
+    if is_src and not err:
+        bad = guard(lambda: sum(synth_dev.check(t, 5000 + rank, i) for i, t in enumerate(st["dst"]))) or 0
+    row = torch.zeros(n, 5, dtype=torch.float64)
+    row[rank] = torch.tensor([statistics.median(alone) if alone else float("nan"),
+                              statistics.median(during) if during else float("nan"),
+                              statistics.median(gbs) if gbs else 0.0, float(bad), float(len(err))],
+                             dtype=torch.float64)
+    dist.all_reduce(row)
+    ctx.finalize()
+    if float(row[:, 4].sum()) > 0:
+        return {"error": err[0] if err else "a rank failed (see its stderr)"}
+    slow = [float(row[r, 1] / row[r, 0] - 1) for r in range(n)]
+    return {"config": "cfg5 imbalanced all-stage swap: sources %s -> importers %s, source s swaps %s micro-batch "
+                      "sets (900 MiB each, one plan), bf16 %dx%dx%d GEMMs on every rank" %
+                      (sources, peers, [H - s for s in sources], M, M, M),
+            "swap_max_ctas": args.gemm_cap,
+            "per_source_gbs": [float(row[s, 2]) for s in sources],
+            "per_source_bytes": [sum(workloads.cfg2_sizes(H - s)) for s in sources],
+            "gemm_alone_ms": [float(row[r, 0]) for r in range(n)],
+            "gemm_slowdown_per_rank": slow,
+            "max_slowdown_sources": max(slow[s] for s in sources),
+            "max_slowdown_importers": max(slow[p] for p in peers),
+            "bit_exact": float(row[:, 3].sum()) == 0}
 
 
 def run_e2e(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, stream, n, dist):

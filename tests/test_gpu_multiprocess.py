@@ -181,3 +181,25 @@ def test_bench_torchrun_two_ranks_one_gpu():
     line = json.loads([l for l in r.stdout.splitlines() if l.startswith("{")][-1])
     assert line["n_gpus"] == 2 and line["value"] > 0 and line["roofline"]["bound"] == "nvlink"
     assert "bit-exact" in line["parity"]
+
+
+def test_bench_cfg5_leg_two_ranks_one_gpu():
+    """bench.py's config-5 leg (sources = first half of the ranks, importers =
+    second half, GEMMs on every rank) under torchrun, both ranks on one GPU:
+    every collective is reached, bytes come back bit-exact, the line carries
+    per-source GB/s and per-rank GEMM slowdowns."""
+    import json
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
+           "--master-addr=127.0.0.1", "--master-port=%d" % _free_port(), "bench.py", "--gpus", "2",
+           "--steps", "2", "--warmup", "1", "--micro-batches", "1", "--e2e-steps", "1", "--gemm-n", "2048"]
+    r = subprocess.run(cmd, cwd=root, capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0, r.stderr[-3000:]
+    line = json.loads([l for l in r.stdout.splitlines() if l.startswith("{")][-1])
+    c5 = line["cfg5"]
+    assert "error" not in c5, c5
+    assert c5["bit_exact"] and len(c5["per_source_gbs"]) == 1 and c5["per_source_gbs"][0] > 0
+    assert len(c5["gemm_slowdown_per_rank"]) == 2
+    assert "error" not in line["gemm_slowdown"], line["gemm_slowdown"]
