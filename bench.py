@@ -51,6 +51,7 @@ def parse():
     ap.add_argument("--impl", default="mpress", choices=["mpress", "reference"])
     ap.add_argument("--path", default="direct", choices=["direct", "bulk", "ce"])
     ap.add_argument("--max-ctas", type=int, default=0)
+    ap.add_argument("--variant", type=int, default=-1, help="kernel shape within --path (-1 = auto)")
     ap.add_argument("--micro-batches", type=int, default=MICRO_BATCHES)
     ap.add_argument("--e2e-steps", type=int, default=16)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -225,7 +226,7 @@ def workload_config(args, n):
              "ranks over NVLink (every rank a source and an importer)" % (args.micro_batches, n - 1)
     return {"workload": wl, "tensors_per_micro_batch": 47, "micro_batch_bytes": 900 << 20,
             "micro_batches": args.micro_batches, "peers": 3 if n == 1 else n - 1,
-            "path": args.path, "max_ctas": args.max_ctas,
+            "path": args.path, "variant": args.variant, "max_ctas": args.max_ctas,
             "l2": "inputs %.2f GiB per rank > 126 MB L2: no flush needed" %
                   (args.micro_batches * 900 / 1024)}
 
@@ -292,6 +293,7 @@ def main():
             for p in range(world):
                 rem[p] -= part[s][p]
     ctx.set_option(mp.OPT_PATH, path)
+    ctx.set_option(mp.OPT_VARIANT, args.variant)
     ctx.set_option(mp.OPT_MAX_CTAS, args.max_ctas)
 
     seed0 = 2000 + 100 * rank
@@ -582,6 +584,24 @@ def traffic_from_profile():
     return None
 
 
+class _Local:
+    """Runs a rank's local work and remembers the first failure, so that the
+    collectives after it are still reached by every rank (a leg that fails on
+    one rank reports the error instead of hanging the others)."""
+
+    def __init__(self):
+        self.err = None
+
+    def __call__(self, fn, *a):
+        if self.err is not None:
+            return None
+        try:
+            return fn(*a)
+        except Exception as exc:  # pragma: no cover - reported in the line
+            self.err = "%s: %s" % (type(exc).__name__, exc)
+            return None
+
+
 def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap, n, dist):
     """Second half of the metric: slowdown of a bf16 GEMM (8192^3, the shape
     MEASURED_PEAKS.json is quoted on) on the compute stream while swaps loop on
@@ -591,10 +611,10 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
     import torch
     comp = torch.cuda.current_stream()
     M = K = N = 8192
-    a = torch.randn(M, K, dtype=torch.bfloat16, device="cuda")
-    b = torch.randn(K, N, dtype=torch.bfloat16, device="cuda")
-    c = torch.empty(M, N, dtype=torch.bfloat16, device="cuda")
     G = 24
+    L = _Local()
+    st = {}
+    alone, during, swap_gbs = [], [], []
 
     def gemms():
         evs = []
@@ -602,51 +622,63 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
             e0 = torch.cuda.Event(enable_timing=True)
             e1 = torch.cuda.Event(enable_timing=True)
             e0.record(comp)
-            torch.matmul(a, b, out=c)
+            torch.matmul(st["a"], st["b"], out=st["c"])
             e1.record(comp)
             evs.append((e0, e1))
         return evs
 
-    pl = mp.plan(world, source, per_copy, bw, sizes)
-    old_cap = ctx.get_option(mp.OPT_MAX_CTAS)
-    ctx.set_option(mp.OPT_MAX_CTAS, args.gemm_cap)
-    # swap time at this cap, to size the loop that must cover the GEMM window
-    e0 = torch.cuda.Event(enable_timing=True)
-    e1 = torch.cuda.Event(enable_timing=True)
-    e0.record(swap)
-    h = ctx.swap_out(pl, src[0], stream=swap)
-    ctx.swap_in(h, dst[0], stream=swap)
-    e1.record(swap)
-    h.free()
-    gemms()
-    torch.cuda.synchronize()
-    per_swap_ms = e0.elapsed_time(e1)
-    alone, during, swap_gbs = [], [], []
-    for _ in range(4):
+    def setup():
+        st["a"] = torch.randn(M, K, dtype=torch.bfloat16, device="cuda")
+        st["b"] = torch.randn(K, N, dtype=torch.bfloat16, device="cuda")
+        st["c"] = torch.empty(M, N, dtype=torch.bfloat16, device="cuda")
+        st["pl"] = mp.plan(world, source, per_copy, bw, sizes)
+        st["old_cap"] = ctx.get_option(mp.OPT_MAX_CTAS)
+        ctx.set_option(mp.OPT_MAX_CTAS, args.gemm_cap)
+        # swap time at this cap, to size the loop that must cover the GEMM window
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(swap)
+        h = ctx.swap_out(st["pl"], src[0], stream=swap)
+        ctx.swap_in(h, dst[0], stream=swap)
+        e1.record(swap)
+        h.free()
+        gemms()
+        torch.cuda.synchronize()
+        st["per_swap_ms"] = e0.elapsed_time(e1)
+
+    def round_():
         evs = gemms()
         torch.cuda.synchronize()
-        alone += [x.elapsed_time(y) for x, y in evs[4:]]
+        alone.extend(x.elapsed_time(y) for x, y in evs[4:])
         gemm_ms = statistics.median(alone)
-        n_swap = int(2.0 * G * gemm_ms / per_swap_ms) + 2
+        n_swap = int(2.0 * G * gemm_ms / st["per_swap_ms"]) + 2
         s0 = torch.cuda.Event(enable_timing=True)
         s1 = torch.cuda.Event(enable_timing=True)
         s0.record(swap)
         for _ in range(n_swap):
-            h = ctx.swap_out(pl, src[0], stream=swap)
+            h = ctx.swap_out(st["pl"], src[0], stream=swap)
             ctx.swap_in(h, dst[0], stream=swap)
             h.free()
         s1.record(swap)
         evs = gemms()
         torch.cuda.synchronize()
         win = s0.elapsed_time(s1)
-        during += [x.elapsed_time(y) for x, y in evs[4:]
-                   if s0.elapsed_time(x) >= 0 and s0.elapsed_time(y) <= win]
+        during.extend(x.elapsed_time(y) for x, y in evs[4:]
+                      if s0.elapsed_time(x) >= 0 and s0.elapsed_time(y) <= win)
         swap_gbs.append(2 * n_swap * sum(sizes) / win / 1e6)
-    ctx.set_option(mp.OPT_MAX_CTAS, old_cap)
-    t = torch.tensor([statistics.median(alone), statistics.median(during) if during else float("nan")],
-                     dtype=torch.float64)
+
+    L(setup)
+    for _ in range(4):
+        L(round_)
+    if "old_cap" in st:
+        L(ctx.set_option, mp.OPT_MAX_CTAS, st["old_cap"])
+    t = torch.tensor([statistics.median(alone) if alone else float("nan"),
+                      statistics.median(during) if during else float("nan"),
+                      1.0 if L.err is not None else 0.0], dtype=torch.float64)
     if n > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    if float(t[2]) > 0:
+        return {"error": L.err or "another rank failed"}
     a_ms, d_ms = float(t[0]), float(t[1])
     return {"gemm": "bf16 8192x8192x8192 torch.matmul (cuBLAS) on the compute stream",
             "alone_ms": a_ms, "with_swap_ms": d_ms, "slowdown": d_ms / a_ms - 1,
@@ -809,25 +841,30 @@ def run_e2e(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, stream,
     fills and drains by one micro-batch, not one step.  `pcie` reports the
     copies alone (no swap) on the same buffers: the ceiling e2e can reach."""
     import torch
+    import numpy as np
     mb = len(src) if n == 1 else min(2, len(src))
     src, dst = src[:mb], dst[:mb]
     steps = max(1, args.e2e_steps)
     nt = len(sizes)
-    hsrc = [[torch.empty(s, dtype=torch.uint8, pin_memory=True) for s in sizes] for _ in range(mb)]
-    hdst = [[torch.empty(s, dtype=torch.uint8, pin_memory=True) for s in sizes] for _ in range(mb)]
-    for m in range(mb):
-        for i in range(nt):
-            hsrc[m][i].copy_(src[m][i])
-    torch.cuda.synchronize()
-
-    srcs = [src, [[torch.empty_like(t) for t in row] for row in src]]
-    dsts = [dst, [[torch.empty_like(t) for t in row] for row in dst]]
-    h2d, d2h = torch.cuda.Stream(), torch.cuda.Stream()
+    L = _Local()
+    st = {}
     src_free = [[None] * mb for _ in range(2)]   # (set, m): its swap-out has read src
     dst_free = [[None] * mb for _ in range(2)]   # (set, m): its download has read dst
 
+    def setup():
+        st["hsrc"] = [[torch.empty(s, dtype=torch.uint8, pin_memory=True) for s in sizes] for _ in range(mb)]
+        st["hdst"] = [[torch.empty(s, dtype=torch.uint8, pin_memory=True) for s in sizes] for _ in range(mb)]
+        for m in range(mb):
+            for i in range(nt):
+                st["hsrc"][m][i].copy_(src[m][i])
+        st["srcs"] = [src, [[torch.empty_like(t) for t in row] for row in src]]
+        st["dsts"] = [dst, [[torch.empty_like(t) for t in row] for row in dst]]
+        st["h2d"], st["d2h"] = torch.cuda.Stream(), torch.cuda.Stream()
+        torch.cuda.synchronize()
+
     def step(k):
         x = k % 2
+        h2d, d2h, srcs, dsts = st["h2d"], st["d2h"], st["srcs"], st["dsts"]
         pl = mp.plan(world, source, per_copy, bw, sizes)
         hs = []
         for m in range(mb):
@@ -835,7 +872,7 @@ def run_e2e(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, stream,
                 h2d.wait_event(src_free[x][m])
             with torch.cuda.stream(h2d):
                 for i in range(nt):
-                    srcs[x][m][i].copy_(hsrc[m][i], non_blocking=True)
+                    srcs[x][m][i].copy_(st["hsrc"][m][i], non_blocking=True)
             up = torch.cuda.Event()
             up.record(h2d)
             stream.wait_event(up)
@@ -851,36 +888,45 @@ def run_e2e(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, stream,
             d2h.wait_event(done)
             with torch.cuda.stream(d2h):
                 for i in range(nt):
-                    hdst[m][i].copy_(dsts[x][m][i], non_blocking=True)
+                    st["hdst"][m][i].copy_(dsts[x][m][i], non_blocking=True)
             dst_free[x][m] = torch.cuda.Event()
             dst_free[x][m].record(d2h)
         for h in hs:
             h.free()
 
-    step(0)
-    torch.cuda.synchronize()
+    def first():
+        step(0)
+        torch.cuda.synchronize()
+
+    def timed():
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        st["h2d"].wait_stream(stream)
+        for k in range(steps):
+            step(k + 1)
+        stream.wait_stream(st["d2h"])
+        e1.record(stream)
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1)
+
+    L(setup)
+    L(first)
     if n > 1:
         dist.barrier()
-    e0 = torch.cuda.Event(enable_timing=True)
-    e1 = torch.cuda.Event(enable_timing=True)
-    e0.record(stream)
-    h2d.wait_stream(stream)
-    for k in range(steps):
-        step(k + 1)
-    stream.wait_stream(d2h)
-    e1.record(stream)
-    torch.cuda.synchronize()
-    ms = e0.elapsed_time(e1)
-    t = torch.tensor([ms], dtype=torch.float64)
+    ms = L(timed)
+    t = torch.tensor([ms or 0.0, 1.0 if L.err is not None else 0.0], dtype=torch.float64)
     if n > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    ms = float(t.item()) / steps
+    if float(t[1]) > 0:
+        return {"error": L.err or "another rank failed"}
+    ms = float(t[0]) / steps
     per = 2 * mb * sum(sizes)
-    import numpy as np
+    hsrc, hdst = st["hsrc"], st["hdst"]
     ok = all(np.array_equal(hdst[m][i].numpy(), hsrc[m][i].numpy())
              for m in (0, mb - 1) for i in range(nt))
     try:
-        pcie = leg_pcie(srcs[0], dsts[0], hsrc, hdst, h2d, d2h, stream)
+        pcie = leg_pcie(st["srcs"][0], st["dsts"][0], hsrc, hdst, st["h2d"], st["d2h"], stream)
     except Exception as exc:  # pragma: no cover - reported, not hidden
         pcie = {"error": "%s: %s" % (type(exc).__name__, exc)}
     return {"value": n * per / (ms / 1e3) / 1e9, "unit": "GB/s",

@@ -402,12 +402,16 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
  * 3 = 1024x4, 4 = 128x8 (16-byte vectors), 5 = 256x4, 6 = 256x8, 7 = 128x4,
  * 8 = 256x4 with L2 evict-first loads, 9 = 128x8 (32-byte vectors, used
  * only when every address is 32-byte aligned, else the 16-byte shape);
- * bulk: 0 = 6 slots x 32 KiB, 1 = 12 x 16 KiB, 2 = 3 x 64 KiB;
+ * bulk: 0 = 6 slots x 32 KiB, 1 = 12 x 16 KiB, 2 = 3 x 64 KiB (one CTA per
+ * SM), 3 = 3 x 32 KiB (one per SM; twice as many fit), 4 = 4 x 16 KiB (three
+ * per SM),
+ * 5 = 2 x 8 KiB, 6 = 3 x 4 KiB (one per SM; small enough to share an SM
+ * with a GEMM CTA);
  * copy engines: 0 = cudaMemcpyAsync per stripe on one side stream per peer,
  * 1 = the whole swap as one cudaMemcpyBatchAsync on the swap stream (not on
  * the legacy NULL stream);
  * MPRESS_VARIANT_AUTO (-1, default) = direct 7 when the grid is capped at
- * <= one CTA per SM (small CTAs co-reside with a GEMM), else 5; bulk 0; copy
+ * <= one CTA per SM (small CTAs co-reside with a GEMM), else 5; bulk 3; copy
  * engines 0.
  * MPRESS_OPT_ORDER: chunk order inside one launch -- 0 = interleave the
  * peers by a weighted round robin, so every peer link carries its share of

@@ -87,12 +87,13 @@ struct Cursor {
   const CopyTable<CAP>& t;
   uint32_t g, gm, gd;
   uint64_t r;
-  __device__ explicit Cursor(const CopyTable<CAP>& tt) : t(tt) {
-    g = blockIdx.x % t.n_groups;
-    r = blockIdx.x / t.n_groups;
-
-    gm = gridDim.x % t.n_groups;
-    gd = gridDim.x / t.n_groups;
+  __device__ explicit Cursor(const CopyTable<CAP>& tt) : Cursor(tt, blockIdx.x, gridDim.x) {}
+  // positions start, start + stride, ...
+  __device__ Cursor(const CopyTable<CAP>& tt, uint32_t start, uint32_t stride) : t(tt) {
+    g = start % t.n_groups;
+    r = start / t.n_groups;
+    gm = stride % t.n_groups;
+    gd = stride / t.n_groups;
   }
   // Next chunk of this CTA: its index *c and its descriptor *s.
   __device__ bool next(uint32_t* c, uint32_t* s) {
@@ -255,14 +256,23 @@ __device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
                :: "r"(smem_u32(bar)), "r"(bytes) : "memory");
 }
 
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+// The wait loop is C++ around a predicate-returning try_wait (no branch
+// inside inline asm), so the compiler sees the divergent loop and reconverges
+// the warp before the shuffles that follow it.
+__device__ __forceinline__ bool mbar_try(uint64_t* bar, uint32_t parity) {
+  uint32_t ok;
   asm volatile(
       "{\n"
       ".reg .pred p;\n"
-      "WAIT_%=:\n"
-      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
-      "@!p bra WAIT_%=;\n"
-      "}\n" :: "r"(smem_u32(bar)), "r"(parity) : "memory");
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n"
+      "selp.u32 %0, 1, 0, p;\n"
+      "}\n" : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity) : "memory");
+  return ok != 0;
+}
+
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  while (!mbar_try(bar, parity)) {
+  }
 }
 
 __device__ __forceinline__ void bulk_load(void* smem, const void* gsrc, uint32_t bytes, uint64_t* bar) {
@@ -298,65 +308,98 @@ __device__ __forceinline__ Piece bulk_piece(const CopyTable<CAP>& t, uint32_t c,
   return p;
 }
 
+// 64-bit warp shuffle.
+__device__ __forceinline__ uint64_t shfl64(uint64_t v, int lane) {
+  const uint32_t lo = __shfl_sync(0xffffffffu, (uint32_t)v, lane);
+  const uint32_t hi = __shfl_sync(0xffffffffu, (uint32_t)(v >> 32), lane);
+  return ((uint64_t)hi << 32) | lo;
+}
+
 // One warp per CTA: lane 0 streams pieces of 2^SHIFT bytes through STAGES
 // shared-memory slots with the SM's bulk-copy engine (cp.async.bulk G->S with
-// mbarrier completion, then S->G bulk stores); the warp first copies the
-// <16-byte tails the bulk engine cannot move.
+// mbarrier completion, then S->G bulk stores).  The 32 lanes resolve the
+// chunk sequence in parallel -- lane j walks positions blockIdx.x +
+// (j + 32i) * gridDim.x with its own cursor -- and hand the pieces to lane 0
+// by shuffles, so the descriptor lookups (dependent constant-bank loads) are
+// off the issuing thread's critical path (profiles/r01: with one cursor on
+// lane 0 they took ~75% of its issue samples).  Each lane also copies the
+// <16-byte tail of a descriptor whose last chunk it resolved.  A ring in
+// shared memory remembers each slot's destination for its store.  Order:
+// piece k's load is issued once the store of piece k - STAGES has been read
+// out of its slot, keeping one store in flight behind the newest
+// (wait_group.read 1).
 template <int DIR, int SHIFT, int STAGES, int CAP>
 __global__ void __launch_bounds__(32)
 mp_swap_bulk(const __grid_constant__ CopyTable<CAP> t) {
   constexpr uint32_t kSlot = 1u << SHIFT;
   extern __shared__ __align__(128) uint8_t smem[];
   __shared__ __align__(8) uint64_t bars[STAGES];
+  __shared__ uint8_t* ring_dst[STAGES];
+  __shared__ uint32_t ring_bytes[STAGES];
+  const uint32_t lane = threadIdx.x;
 
-  {  // tails, by the whole warp
-    Cursor<CAP> cur(t);
-    uint32_t c, s;
-    while (cur.next(&c, &s)) {
-      if (c + 1 != t.first_chunk[s + 1]) continue;  // not the last chunk of desc s
-      const CopyDesc& d = t.d[s];
-      const uint32_t tail = (uint32_t)(d.len & 15u);
-      if (threadIdx.x < tail) {
-        const uint64_t b = (d.len & ~15ull) + threadIdx.x;
-        static_cast<uint8_t*>(d.dst)[b] = static_cast<const uint8_t*>(d.src)[b];
-      }
-    }
+  if (lane == 0) {
+    for (int k = 0; k < STAGES; ++k) mbar_init(&bars[k], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  if (threadIdx.x != 0) return;
+  __syncwarp();
 
-  for (int k = 0; k < STAGES; ++k) mbar_init(&bars[k], 1);
-  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-
-  // Two cursors over the same chunk sequence: loads run STAGES ahead of stores.
-  Cursor<CAP> ld(t), st(t);
-  uint32_t issued = 0;
-  auto issue_load = [&]() -> bool {
-    uint32_t c, s;
-    if (!ld.next(&c, &s)) return false;
-    const Piece p = bulk_piece<SHIFT>(t, c, s);
-    uint64_t* bar = &bars[issued % STAGES];
-    mbar_expect_tx(bar, p.bytes);
-    if (p.bytes) bulk_load(smem + (size_t)(issued % STAGES) * kSlot, p.src, p.bytes, bar);
-    ++issued;
-    return true;
+  uint32_t loaded = 0, stored = 0;  // pieces whose load / store was issued (lane 0)
+  // lane 0: issue the stores of pieces [stored, upto) in order
+  auto store_until = [&](uint32_t upto) {
+    for (; stored < upto; ++stored) {
+      const uint32_t q = stored % STAGES;
+      mbar_wait(&bars[q], (stored / STAGES) & 1u);
+      if (ring_bytes[q]) bulk_store(ring_dst[q], smem + (size_t)q * kSlot, ring_bytes[q]);
+      bulk_commit();
+    }
   };
 
-  for (int k = 0; k < STAGES; ++k)
-    if (!issue_load()) break;
-  uint32_t c, s;
-  for (uint32_t i = 0; st.next(&c, &s); ++i) {
-    mbar_wait(&bars[i % STAGES], (i / STAGES) & 1u);
-    const Piece p = bulk_piece<SHIFT>(t, c, s);
-    if (p.bytes) bulk_store(p.dst, smem + (size_t)(i % STAGES) * kSlot, p.bytes);
-    bulk_commit();
-    // Refill the slot of piece i-1 once its store has finished reading smem
-    // (only the newest group, piece i's store, may still be reading).
-    if (i >= 1 && issued == i - 1 + STAGES) {
-      bulk_wait_read1();
-      issue_load();
+  Cursor<CAP> cur(t, blockIdx.x + lane * gridDim.x, 32u * gridDim.x);
+  for (;;) {
+    uint32_t c, sd;
+    const bool v = cur.next(&c, &sd);
+    Piece mine{nullptr, nullptr, 0};
+    if (v) {
+      mine = bulk_piece<SHIFT>(t, c, sd);
+      if (c + 1 == t.first_chunk[sd + 1]) {  // last chunk of descriptor sd: its tail
+        const CopyDesc& d = t.d[sd];
+        for (uint64_t b = d.len & ~15ull; b < d.len; ++b)
+          static_cast<uint8_t*>(d.dst)[b] = static_cast<const uint8_t*>(d.src)[b];
+      }
+    }
+    // Lanes leave their cursor loops after different trip counts: reconverge
+    // explicitly before the ballot and the shuffles (without it the ballot was
+    // compiled without a warp sync and saw only the lanes already done).
+    __syncwarp();
+    uint32_t mask = __ballot_sync(0xffffffffu, v);
+    if (!mask) break;
+    while (mask) {
+      const int j = __ffs(mask) - 1;
+      mask &= mask - 1;
+      const uint8_t* src = reinterpret_cast<const uint8_t*>(shfl64(reinterpret_cast<uint64_t>(mine.src), j));
+      uint8_t* dst = reinterpret_cast<uint8_t*>(shfl64(reinterpret_cast<uint64_t>(mine.dst), j));
+      const uint32_t bytes = __shfl_sync(0xffffffffu, mine.bytes, j);
+      if (lane == 0) {
+        const uint32_t k = loaded;
+        if (k >= STAGES) {
+          store_until(k - STAGES + 2 <= k ? k - STAGES + 2 : k);  // stores through piece k-STAGES+1
+          bulk_wait_read1();  // all but the newest store have left smem: slot of k-STAGES is free
+        }
+        const uint32_t q = k % STAGES;
+        ring_dst[q] = dst;
+        ring_bytes[q] = bytes;
+        mbar_expect_tx(&bars[q], bytes);
+        if (bytes) bulk_load(smem + (size_t)q * kSlot, src, bytes, &bars[q]);
+        ++loaded;
+      }
+      __syncwarp();
     }
   }
-  bulk_wait_all();
+  if (lane == 0) {
+    store_until(loaded);
+    bulk_wait_all();
+  }
 }
 
 // ---------------------------------------------------------------- variants
@@ -373,13 +416,17 @@ struct Shape {
 // direct (threads, unroll, vector bytes): 0 (256,8,16) 1 (512,8,16)
 // 2 (256,16,16) 3 (1024,4,16) 4 (128,8,16) 5 (256,4,32) 6 (256,8,32)
 // 7 (128,4,32) 8 (256,4,32 + L2 evict-first loads) 9 (128,8,32)
-// bulk (piece, stages): 0 (32K,6) 1 (16K,12) 2 (64K,3)
+// bulk (piece, stages, CTAs/SM): 0 (32K,6,1) 1 (16K,12,1) 2 (64K,3,1) 3 (32K,3,1)
+// 4 (16K,4,3) 5 (8K,2,1) 6 (4K,3,1) -- 5 and 6 use 16 / 12 KB of shared
+// memory, small enough to sit beside a cuBLAS GEMM CTA (214 KB)
 constexpr Shape kDirect[kDirectVariants] = {
     {256, 15, 0, 2, 16, 0}, {512, 16, 0, 1, 16, 1}, {256, 16, 0, 2, 16, 2}, {1024, 16, 0, 1, 16, 3},
     {128, 14, 0, 4, 16, 4}, {256, 15, 0, 2, 32, 0}, {256, 16, 0, 2, 32, 2}, {128, 14, 0, 4, 32, 4},
     {256, 15, 0, 2, 32, 0}, {128, 15, 0, 4, 32, 4}};
 constexpr Shape kBulk[kBulkVariants] = {
-    {32, 15, 6u << 15, 1, 16, 0}, {32, 14, 12u << 14, 1, 16, 1}, {32, 16, 3u << 16, 1, 16, 2}};
+    {32, 15, 6u << 15, 1, 16, 0}, {32, 14, 12u << 14, 1, 16, 1}, {32, 16, 3u << 16, 1, 16, 2},
+    {32, 15, 3u << 15, 1, 16, 3}, {32, 14, 4u << 14, 3, 16, 4}, {32, 13, 2u << 13, 1, 16, 5},
+    {32, 12, 3u << 12, 1, 16, 6}};
 
 template <int CAP>
 using KernelFn = void (*)(CopyTable<CAP>);
@@ -391,6 +438,10 @@ KernelFn<CAP> kernel_for(int path, int variant, int dir, bool pf) {
     switch (variant) {
       case 1: return o ? mp_swap_bulk<kDirOut, 14, 12, CAP> : mp_swap_bulk<kDirIn, 14, 12, CAP>;
       case 2: return o ? mp_swap_bulk<kDirOut, 16, 3, CAP> : mp_swap_bulk<kDirIn, 16, 3, CAP>;
+      case 3: return o ? mp_swap_bulk<kDirOut, 15, 3, CAP> : mp_swap_bulk<kDirIn, 15, 3, CAP>;
+      case 4: return o ? mp_swap_bulk<kDirOut, 14, 4, CAP> : mp_swap_bulk<kDirIn, 14, 4, CAP>;
+      case 5: return o ? mp_swap_bulk<kDirOut, 13, 2, CAP> : mp_swap_bulk<kDirIn, 13, 2, CAP>;
+      case 6: return o ? mp_swap_bulk<kDirOut, 12, 3, CAP> : mp_swap_bulk<kDirIn, 12, 3, CAP>;
       default: return o ? mp_swap_bulk<kDirOut, 15, 6, CAP> : mp_swap_bulk<kDirIn, 15, 6, CAP>;
     }
   }
@@ -542,11 +593,12 @@ int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* gr
     // co-reside instead of taking SMs away from it; full grid: 2 x 256-thread
     // CTAs per SM saturate HBM (profiles/r01 sweeps).  Both use 32-byte
     // vectors (LDG/STG .256, +1% over 16-byte ones; 16-byte fallback when the
-    // data is only 16-byte aligned).  bulk: 6 x 32 KiB.
+    // data is only 16-byte aligned).  bulk: 3 x 32 KiB, one CTA per SM
+    // (profiles/r01/sweep_bulk_variants.jsonl).
     if (path == MPRESS_PATH_DIRECT)
       variant = (max_ctas > 0 && max_ctas <= sms) ? 7 : 5;
     else
-      variant = 0;
+      variant = 3;
   }
   const int nvar = path == MPRESS_PATH_BULK ? kBulkVariants : kDirectVariants;
   if (variant < 0 || variant >= nvar) return fail(MPRESS_ERR_ARG, "kernel variant %d out of range", variant);
