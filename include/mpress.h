@@ -515,6 +515,10 @@ MPRESS_API int mpress_query(mpress_ctx_t* ctx, mpress_handle_t* handle);
 /* Current state (MPRESS_STATE_*) without querying the device. */
 MPRESS_API int mpress_handle_state(const mpress_handle_t* handle);
 
+/* 1 if the handle's swap-out was captured into a CUDA graph (a graph handle,
+ * see "CUDA graph capture" above), 0 if not, < 0 on error. */
+MPRESS_API int mpress_handle_is_graph(const mpress_handle_t* handle);
+
 /* Slice base of the handle inside this source's partition of each peer's
  * pool [world]; UINT64_MAX for peers the plan does not use (tests). */
 MPRESS_API int mpress_handle_slices(const mpress_handle_t* handle, uint64_t* slice_off);

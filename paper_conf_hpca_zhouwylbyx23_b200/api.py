@@ -42,6 +42,7 @@ EXPORTED = [
     "mpress_init_local",
     "mpress_finalize", "mpress_stash_free", "mpress_set_option", "mpress_get_option",
     "mpress_swap_out", "mpress_swap_in", "mpress_wait", "mpress_query", "mpress_handle_state",
+    "mpress_handle_is_graph",
     "mpress_handle_slices", "mpress_handle_free", "mpress_peer_read", "mpress_last_launches",
     "mpress_share_fds", "mpress_last_error", "mpress_version",
 ]
@@ -124,6 +125,7 @@ def _load():
         "mpress_wait": (c_int, [P, P, P]),
         "mpress_query": (c_int, [P, P]),
         "mpress_handle_state": (c_int, [P]),
+        "mpress_handle_is_graph": (c_int, [P]),
         "mpress_handle_slices": (c_int, [P, P]),
         "mpress_handle_free": (c_int, [P, P, c_int]),
         "mpress_peer_read": (c_int, [P, c_int, c_uint64, c_uint64, P]),
@@ -367,13 +369,19 @@ def share_fds(world, rank, my_fd, want, exchange_cb):
 
 class Handle:
     """An mpress_handle_t (one swapped batch).  Released by free(), by the
-    garbage collector (forced), or when its context is finalized."""
+    garbage collector (forced), or when its context is finalized.  A graph
+    handle (swap-out captured into a CUDA graph) is owned by its graph's
+    replays, so the context keeps it alive until free() is called explicitly
+    -- dropping the Python object must not release slices a replay uses."""
 
     def __init__(self, ctx, h, plan):
         self._ctx = ctx
         self._h = h
         self.plan = plan  # keeps the Plan alive while the handle exists
         ctx._handles.add(self)
+        self.graph = _check(lib.mpress_handle_is_graph(h)) == 1
+        if self.graph:
+            ctx._graph_handles.add(self)
 
     def __del__(self):
         try:
@@ -396,6 +404,7 @@ class Handle:
         if self._h is not None and self._h.value:
             _check(lib.mpress_handle_free(self._ctx._h, self._h, 1 if force else 0))
         self._h = None
+        self._ctx._graph_handles.discard(self)
 
 
 class Executor:
@@ -447,6 +456,7 @@ class Context:
         self.device = device
         self._exchange = exchange_cb  # keep the ctypes callback alive
         self._handles = weakref.WeakSet()
+        self._graph_handles = set()   # strong refs: released only by Handle.free()
 
     def __del__(self):
         # A local context can be released here; a distributed one must be
@@ -480,8 +490,14 @@ class Context:
         if self._h is not None:
             for hd in list(self._handles):   # the library frees them with the context
                 hd._h = None
+            self._graph_handles.clear()
             h, self._h = self._h, None
             _check(lib.mpress_finalize(h))
+
+    @property
+    def graph_handles(self):
+        """Graph handles not yet freed (kept alive for their graphs' replays)."""
+        return list(self._graph_handles)
 
     def set_option(self, key, value):
         _check(lib.mpress_set_option(self._h, key, int(value)))

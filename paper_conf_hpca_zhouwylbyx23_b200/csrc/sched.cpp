@@ -416,6 +416,11 @@ extern "C" int mpress_query(mpress_ctx_t* c, mpress_handle_t* h) {
 
 extern "C" int mpress_handle_state(const mpress_handle_t* h) { return h ? h->state : MPRESS_ERR_ARG; }
 
+extern "C" int mpress_handle_is_graph(const mpress_handle_t* h) {
+  if (!h) return fail(MPRESS_ERR_ARG, "mpress_handle_is_graph: null handle");
+  return h->graph ? 1 : 0;
+}
+
 extern "C" int mpress_handle_slices(const mpress_handle_t* h, uint64_t* slice_off) {
   if (!h || !slice_off) return fail(MPRESS_ERR_ARG, "mpress_handle_slices: null argument");
   std::copy(h->slice_off.begin(), h->slice_off.end(), slice_off);

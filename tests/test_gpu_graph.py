@@ -163,3 +163,34 @@ def test_graph_misuse():
         h3.free()
     finally:
         ctx.finalize()
+
+
+def test_graph_handle_survives_python_gc():
+    """Dropping the Python handle of a captured swap must not release the
+    slices its graph replays into; Context.graph_handles gives it back."""
+    import gc
+    sizes, o, pl, ctx = _setup(mp.PATH_DIRECT)
+    try:
+        src = [torch.empty(n, dtype=torch.uint8, device="cuda") for n in sizes]
+        dst = [torch.zeros(n, dtype=torch.uint8, device="cuda") for n in sizes]
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=torch.cuda.Stream()):
+            h = ctx.swap_out(pl, src)
+            ctx.swap_in(h, dst)
+        assert h.graph
+        held = ctx.stash_free()
+        del h
+        gc.collect()
+        assert ctx.stash_free() == held                 # still reserved
+        _refill(src, 321)
+        g.replay()
+        torch.cuda.synchronize()
+        for i, d in enumerate(dst):
+            assert synth_dev.check(d, 321, i) == 0
+        (hg,) = ctx.graph_handles
+        del g
+        hg.free()
+        assert ctx.graph_handles == []
+        assert ctx.stash_free() != held
+    finally:
+        ctx.finalize()
