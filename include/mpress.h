@@ -320,6 +320,9 @@ MPRESS_API int mpress_schedule_1f1b(const mpress_1f1b_params* params, mpress_1f1
  *       triggers on the swap-in stream, into the buffers given by
  *       mpress_executor_restore_to(x, m, dst) beforehand.
  * Enqueue-only.  One executor serves any number of steps.
+ * An executor step cannot be captured into a CUDA graph (MPRESS_ERR_STATE
+ * while any of its streams is capturing): it recycles stash slices between
+ * micro-batches, which a replayed graph would share with eager swaps.
  * Free executors before mpress_finalize of their context.
  * Errors: MPRESS_ERR_ARG, MPRESS_ERR_STATE (op order violated, no restore
  * buffers), plus those of swap_out / swap_in.

@@ -11,6 +11,7 @@
 //     m on the swap-in stream into the buffers registered for m;
 //   * before B(m): makes the compute stream wait for that swap-in.
 // Everything is enqueue-only (no blocking of the main thread).
+#include <initializer_list>
 #include <new>
 #include <vector>
 
@@ -82,9 +83,29 @@ extern "C" int mpress_executor_restore_to(mpress_executor_t* x, uint32_t micro_b
   return MPRESS_OK;
 }
 
+namespace {
+// The executor frees each micro-batch's handle at its backward and reuses the
+// slices for later micro-batches; under graph capture those slices would be
+// handed back to eager swaps while the graph still replays into them, so an
+// executor step is not capturable (capture individual swap pairs instead).
+bool any_capturing(std::initializer_list<cudaStream_t> ss) {
+  for (cudaStream_t s : ss) {
+    cudaStreamCaptureStatus st = cudaStreamCaptureStatusNone;
+    if (cudaStreamIsCapturing(s, &st) != cudaSuccess) {
+      cudaGetLastError();
+      continue;
+    }
+    if (st != cudaStreamCaptureStatusNone) return true;
+  }
+  return false;
+}
+}  // namespace
+
 extern "C" int mpress_executor_before(mpress_executor_t* x, uint32_t op, void* compute_stream, uint32_t* kind,
                                       uint32_t* micro_batch) {
   if (!x || op >= x->kind.size()) return fail(MPRESS_ERR_ARG, "mpress_executor_before: bad op");
+  if (any_capturing({static_cast<cudaStream_t>(compute_stream), x->out_stream, x->in_stream}))
+    return fail(MPRESS_ERR_STATE, "mpress_executor_before: executor steps cannot be captured into a CUDA graph");
   const int m = x->mb[op];
   if (kind) *kind = (uint32_t)x->kind[op];
   if (micro_batch) *micro_batch = (uint32_t)m;
@@ -102,6 +123,8 @@ extern "C" int mpress_executor_before(mpress_executor_t* x, uint32_t op, void* c
 extern "C" int mpress_executor_after(mpress_executor_t* x, uint32_t op, void* compute_stream,
                                      void* const* activations) {
   if (!x || op >= x->kind.size()) return fail(MPRESS_ERR_ARG, "mpress_executor_after: bad op");
+  if (any_capturing({static_cast<cudaStream_t>(compute_stream), x->out_stream, x->in_stream}))
+    return fail(MPRESS_ERR_STATE, "mpress_executor_after: executor steps cannot be captured into a CUDA graph");
   mpress_ctx_s* c = x->ctx;
   DeviceGuard g(c->device);
   EvRef done = take_event(c);

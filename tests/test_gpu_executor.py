@@ -72,3 +72,22 @@ def test_executor_missing_restore_buffers():
         ex.free()
     finally:
         ctx.finalize()
+
+
+def test_executor_refuses_graph_capture():
+    """An executor step recycles stash slices between micro-batches, so it
+    must refuse to run while one of its streams is being captured."""
+    M = 2
+    ctx, pl, sizes = _setup(M)
+    s_out, s_in = torch.cuda.Stream(), torch.cuda.Stream()
+    try:
+        ex = mp.Executor(ctx, pl, 2, 0, M, 10_000, 20_000, 5_000, 5_000, s_out, s_in)
+        src = [torch.empty(n, dtype=torch.uint8, device="cuda") for n in sizes]
+        g = torch.cuda.CUDAGraph()
+        with pytest.raises(mp.MPressError) as ei:
+            with torch.cuda.graph(g, stream=torch.cuda.Stream()):
+                ex.after(0, torch.cuda.current_stream(), src)
+        assert ei.value.code == mp.ERR_STATE
+        ex.free()
+    finally:
+        ctx.finalize()
