@@ -49,7 +49,8 @@ def parse():
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="mpress", choices=["mpress", "reference"])
-    ap.add_argument("--path", default="direct", choices=["direct", "bulk", "ce"])
+    ap.add_argument("--path", default="auto", choices=["auto", "direct", "bulk", "ce"],
+                    help="auto = the library default: bulk (TMA) at a full grid, direct when capped")
     ap.add_argument("--max-ctas", type=int, default=0)
     ap.add_argument("--variant", type=int, default=-1, help="kernel shape within --path (-1 = auto)")
     ap.add_argument("--micro-batches", type=int, default=MICRO_BATCHES)
@@ -264,7 +265,7 @@ def main():
     sizes = workloads.cfg2_sizes(1)
     mb = args.micro_batches
     G = mp.DEFAULT_GRANULE
-    path = {"direct": mp.PATH_DIRECT, "bulk": mp.PATH_BULK, "ce": mp.PATH_CE}[args.path]
+    path = {"direct": mp.PATH_DIRECT, "bulk": mp.PATH_BULK, "ce": mp.PATH_CE, "auto": mp.PATH_AUTO}[args.path]
 
     if n == 1:
         world, source = 4, 0
@@ -374,6 +375,8 @@ def main():
     if int(bad_t.item()) != 0:
         raise SystemExit("round trip mismatch: %d bytes" % int(bad_t.item()))
 
+    ran = {mp.PATH_DIRECT: "direct", mp.PATH_BULK: "bulk", mp.PATH_CE: "ce"}.get(
+        ctx.get_option(mp.OPT_LAST_PATH), "?")
     # per-kernel durations (each swap call here is exactly one kernel launch)
     dur = {k: [a.elapsed_time(b) for a, b in v] for k, v in timing.items()}
     tot = {k: sum(v) for k, v in dur.items()}
@@ -385,8 +388,8 @@ def main():
         achieved = algo_bytes / (avg_ms / 1e3) / 1e9
         peak = float(peaks.get("hbm_gbs", FALLBACK_HBM))
         roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                "frac": achieved / peak, "traffic": traffic_from_profile(),
-                "kernel": "mp_swap_%s<%s>" % (args.path, "kDirIn" if dom == "in" else "kDirOut"),
+                "frac": achieved / peak, "traffic": traffic_from_profile(ran),
+                "kernel": "mp_swap_%s<%s>" % (ran, "kDirIn" if dom == "in" else "kDirOut"),
                 "algorithmic_bytes_per_launch": algo_bytes,
                 "avg_launch_ms": avg_ms, "peak_source": "%s hbm_gbs (MEASURED_PEAKS.json)" % peaks_src,
                 "share_of_step": (tot["in"] + tot["out"]) / ms * 1.0 if ms > 0 else None}
@@ -396,7 +399,7 @@ def main():
         roof = {"bound": "nvlink", "achieved": achieved, "peak": NVLINK_MEASURED, "unit": "GB/s",
                 "frac": achieved / NVLINK_MEASURED, "traffic": None,
                 "nominal_peak": NVLINK_NOMINAL, "frac_of_nominal": achieved / NVLINK_NOMINAL,
-                "kernel": "mp_swap_%s<%s>" % (args.path, "kDirIn" if dom == "in" else "kDirOut"),
+                "kernel": "mp_swap_%s<%s>" % (ran, "kDirIn" if dom == "in" else "kDirOut"),
                 "algorithmic_bytes_per_launch": algo_bytes, "avg_launch_ms": avg_ms,
                 "peak_source": "B200_PROFILING.md measured peer copy per direction"}
     per_dir = {k: bytes_per_mb / (statistics.mean(v) / 1e3) / 1e9 for k, v in dur.items()}
@@ -434,6 +437,7 @@ def main():
             "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
             "config": workload_config(args, n),
+            "swap_path_ran": ran,
             "per_direction_gbs": per_dir,
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": launches[0], "clocks": clk, "gemm_slowdown": gemm,
@@ -466,7 +470,7 @@ def other_configs(args, mp, device):
     import torch
     from synth import device as synth_dev
     from synth import workloads
-    path = {"direct": mp.PATH_DIRECT, "bulk": mp.PATH_BULK, "ce": mp.PATH_CE}[args.path]
+    path = {"direct": mp.PATH_DIRECT, "bulk": mp.PATH_BULK, "ce": mp.PATH_CE, "auto": mp.PATH_AUTO}[args.path]
     c3 = workloads.CONFIGS[3]
     cases = [
         ("cfg1 16 x 4 MiB fp16 activations -> 1 peer", 2, [1], [0, 1 << 30], workloads.cfg1_sizes()),
@@ -571,14 +575,14 @@ def planner_timing(mp, world, source, spare, bw, sizes):
             "stripes": len(o["stripes"]), "note": "cpp includes the ctypes call; identical plans"}
 
 
-def traffic_from_profile():
-    """dram read+write bytes per launch of the dominant kernel from the
-    committed ncu --set full summary, if one exists for this round."""
+def traffic_from_profile(path):
+    """dram read+write bytes per launch of the dominant kernel (the swap
+    kernel of `path`) from the committed ncu --set full summary, if any."""
     p = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(p):
         try:
             with open(p) as f:
-                return json.load(f).get("dram_bytes_per_launch")
+                return json.load(f)["per_path"][path]["dram_bytes_per_launch"]
         except Exception:
             return None
     return None
@@ -670,6 +674,7 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
     L(setup)
     for _ in range(4):
         L(round_)
+    st["ran"] = ctx.get_option(mp.OPT_LAST_PATH)
     if "old_cap" in st:
         L(ctx.set_option, mp.OPT_MAX_CTAS, st["old_cap"])
     t = torch.tensor([statistics.median(alone) if alone else float("nan"),
@@ -682,7 +687,8 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
     a_ms, d_ms = float(t[0]), float(t[1])
     return {"gemm": "bf16 8192x8192x8192 torch.matmul (cuBLAS) on the compute stream",
             "alone_ms": a_ms, "with_swap_ms": d_ms, "slowdown": d_ms / a_ms - 1,
-            "swap_path": args.path, "swap_max_ctas": args.gemm_cap,
+            "swap_path": {mp.PATH_DIRECT: "direct", mp.PATH_BULK: "bulk", mp.PATH_CE: "ce"}.get(
+                st.get("ran"), args.path), "swap_max_ctas": args.gemm_cap,
             "swap_gbs_during": statistics.median(swap_gbs),
             "gemms_counted": len(during),
             "note": ("N=1 loopback: the swap's bytes also load the GEMM's HBM (2 B per swapped "

@@ -392,11 +392,17 @@ MPRESS_API int mpress_finalize(mpress_ctx_t* ctx);
  * [world] -> the spare_bytes argument of mpress_plan for the next batch. */
 MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
 
-/* Tunables.  MPRESS_OPT_PATH: 0 = SM kernel, direct 16-B loads/stores
- * (default); 1 = SM kernel, bulk-async copies (the SM's TMA engine,
- * cp.async.bulk) staged through shared memory; 2 = copy engines
- * (cudaMemcpyAsync per stripe on per-peer streams, the measured comparator).
- * Setting the path resets the variant to MPRESS_VARIANT_AUTO.
+/* Tunables.  MPRESS_OPT_PATH: 0 = SM kernel, direct 16/32-B loads/stores;
+ * 1 = SM kernel, bulk-async copies (the SM's TMA engine, cp.async.bulk)
+ * staged through shared memory; 2 = copy engines (cudaMemcpyAsync per stripe
+ * on per-peer streams, the measured comparator); 3 = MPRESS_PATH_AUTO
+ * (default): per launch, bulk at a full grid (max_ctas 0 or above the SM
+ * count: +0.8% over direct, profiles/r01), direct when the grid is capped to
+ * <= one CTA per SM (its 128-thread CTAs co-reside with a GEMM, bulk CTAs'
+ * shared memory does not) or when a peer is a host pool.
+ * MPRESS_OPT_LAST_PATH (read-only) reports the path the last swap call ran.
+ * Setting the path resets the variant to MPRESS_VARIANT_AUTO; under
+ * MPRESS_PATH_AUTO only MPRESS_VARIANT_AUTO is accepted.
  * MPRESS_OPT_MAX_CTAS: cap on the kernel grid (0 = the variant's default
  * grid, a multiple of the SM count); CTAs spread one per SM first, so this is
  * the SM-count cap that protects a concurrent GEMM.
@@ -431,6 +437,7 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
  * shared with CUDA IPC handles through the all-gather; used when the fd path
  * fails on any rank, or forced with the environment variable MPRESS_IPC=legacy). */
 #define MPRESS_OPT_TRANSPORT 5
+#define MPRESS_OPT_LAST_PATH 6   /* read-only: path of the last swap call */
 #define MPRESS_TRANSPORT_LOCAL      0
 #define MPRESS_TRANSPORT_VMM_FD     1
 #define MPRESS_TRANSPORT_LEGACY_IPC 2
@@ -440,6 +447,7 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
 #define MPRESS_PATH_DIRECT   0
 #define MPRESS_PATH_BULK     1
 #define MPRESS_PATH_CE       2
+#define MPRESS_PATH_AUTO     3
 MPRESS_API int mpress_set_option(mpress_ctx_t* ctx, int key, int64_t value);
 MPRESS_API int mpress_get_option(const mpress_ctx_t* ctx, int key, int64_t* value);
 

@@ -23,9 +23,10 @@ OPT_PATH, OPT_MAX_CTAS, OPT_VARIANT, OPT_ORDER = 1, 2, 3, 4
 ORDER_INTERLEAVE, ORDER_PLAN = 0, 1
 DEVICE_HOST = -1   # mpress_init_local: a pinned host pool as a peer (NEXT-4)
 OPT_TRANSPORT = 5  # read-only
+OPT_LAST_PATH = 6  # read-only: path of the last swap call
 TRANSPORT_LOCAL, TRANSPORT_VMM_FD, TRANSPORT_LEGACY_IPC = 0, 1, 2
 VARIANT_AUTO = -1
-PATH_DIRECT, PATH_BULK, PATH_CE = 0, 1, 2
+PATH_DIRECT, PATH_BULK, PATH_CE, PATH_AUTO = 0, 1, 2, 3
 STATE_OUT_PENDING, STATE_OUT, STATE_IN_PENDING, STATE_IN = 1, 2, 3, 4
 
 _ERR_NAMES = {ERR_ARG: "ERR_ARG", ERR_NO_SPACE: "ERR_NO_SPACE", ERR_ALIGN: "ERR_ALIGN",

@@ -97,7 +97,9 @@ struct mpress_ctx_s {
   mpress::Mapping own;                // multi-process: this rank's exported pool
   std::vector<mpress::Mapping> maps;  // [world] pool mappings used by this source
   std::vector<mpress::Partition> parts;  // [world]
-  int path = MPRESS_PATH_DIRECT;
+  int path = MPRESS_PATH_AUTO;
+  int last_path = -1;                 // path the last swap call ran (MPRESS_OPT_LAST_PATH)
+  bool host_peer = false;             // a peer pool is pinned host memory (NEXT-4)
   int max_ctas = 0;
   int variant = MPRESS_VARIANT_AUTO;
   int order = MPRESS_ORDER_INTERLEAVE;

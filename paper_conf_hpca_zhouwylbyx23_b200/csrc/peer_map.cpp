@@ -198,6 +198,7 @@ extern "C" int mpress_init_local(int world, int source, const int* devices,
     if (p == source || want == 0) continue;
     if (devices[p] == MPRESS_DEVICE_HOST) {
       const int rc = map_host_pool(&c->maps[p], want);
+      c->host_peer = true;
       if (rc != MPRESS_OK) {
         destroy(c);
         return rc;
@@ -458,7 +459,8 @@ extern "C" int mpress_set_option(mpress_ctx_t* c, int key, int64_t value) {
   std::lock_guard<std::mutex> lk(c->mu);
   switch (key) {
     case MPRESS_OPT_PATH:
-      if (value != MPRESS_PATH_DIRECT && value != MPRESS_PATH_BULK && value != MPRESS_PATH_CE)
+      if (value != MPRESS_PATH_DIRECT && value != MPRESS_PATH_BULK && value != MPRESS_PATH_CE &&
+          value != MPRESS_PATH_AUTO)
         return fail(MPRESS_ERR_ARG, "unknown path %lld", (long long)value);
       c->path = (int)value;
       c->variant = MPRESS_VARIANT_AUTO;  // variants are per path
@@ -474,7 +476,8 @@ extern "C" int mpress_set_option(mpress_ctx_t* c, int key, int64_t value) {
       return MPRESS_OK;
     case MPRESS_OPT_VARIANT: {
       const int nvar = c->path == MPRESS_PATH_BULK ? kBulkVariants
-                       : c->path == MPRESS_PATH_CE ? kCeVariants : kDirectVariants;
+                       : c->path == MPRESS_PATH_CE ? kCeVariants
+                       : c->path == MPRESS_PATH_AUTO ? 0 : kDirectVariants;
       if (value != MPRESS_VARIANT_AUTO && (value < 0 || value >= nvar))
         return fail(MPRESS_ERR_ARG, "variant %lld out of range for path %d", (long long)value, c->path);
       c->variant = (int)value;
@@ -492,6 +495,7 @@ extern "C" int mpress_get_option(const mpress_ctx_t* c, int key, int64_t* value)
     case MPRESS_OPT_VARIANT: *value = c->variant; return MPRESS_OK;
     case MPRESS_OPT_ORDER: *value = c->order; return MPRESS_OK;
     case MPRESS_OPT_TRANSPORT: *value = c->transport; return MPRESS_OK;
+    case MPRESS_OPT_LAST_PATH: *value = c->last_path; return MPRESS_OK;
   }
   return fail(MPRESS_ERR_ARG, "unknown option %d", key);
 }

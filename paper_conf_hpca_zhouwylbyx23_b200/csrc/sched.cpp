@@ -142,8 +142,20 @@ int record_done(mpress_ctx_s* c, cudaStream_t s, bool graph, EvRef* ev, EvRef* e
 int run_copy(mpress_ctx_s* c, int dir, const std::vector<CopyDesc>& d,
              const std::vector<int>& desc_peer, cudaStream_t stream) {
   c->last_launches = 0;
-  if (c->path != MPRESS_PATH_CE)
-    return launch_copy(c->path, c->variant, dir, d.data(),
+  int path = c->path;
+  if (path == MPRESS_PATH_AUTO) {
+    // bulk at a full grid (TMA, +0.8% over direct on B200, profiles/r01);
+    // direct when the grid is capped to <= one CTA per SM (small CTAs that
+    // co-reside with a GEMM) or a peer is pinned host memory
+    int dev = 0, sms = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const bool capped = c->max_ctas > 0 && c->max_ctas <= sms;
+    path = (capped || c->host_peer) ? MPRESS_PATH_DIRECT : MPRESS_PATH_BULK;
+  }
+  c->last_path = path;
+  if (path != MPRESS_PATH_CE)
+    return launch_copy(path, c->variant, dir, d.data(),
                        c->order == MPRESS_ORDER_INTERLEAVE ? desc_peer.data() : nullptr, d.size(), c->max_ctas,
                        stream, &c->last_launches);
 

@@ -194,3 +194,21 @@ def test_plan_overflow_and_zero_size_rejected():
     with pytest.raises(mp.MPressError) as ei:
         mp.plan(2, 0, [0, 1 << 40], [0, 1], [5, 0])
     assert ei.value.code == mp.ERR_ARG
+
+
+def test_header_constants_match_the_binding():
+    """Every integer constant include/mpress.h defines (options, paths,
+    orders, transports, states, errors, choices) has a twin with the same
+    value in the package namespace (MPRESS_X -> mp.X), so a constant added to
+    the ABI cannot be missing from the binding the bench and tests use."""
+    src = open(os.path.join(ROOT, "include", "mpress.h")).read()
+    defs = dict(re.findall(r"#define\s+MPRESS_(\w+)\s+\(?(-?\d+)u?\)?", src))
+    skip = {"VERSION"}
+    checked = 0
+    for name, val in defs.items():
+        if name in skip:
+            continue
+        assert hasattr(mp, name), "mp.%s missing (MPRESS_%s in mpress.h)" % (name, name)
+        assert getattr(mp, name) == int(val), name
+        checked += 1
+    assert checked >= 30
