@@ -650,10 +650,13 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
         torch.cuda.synchronize()
         st["per_swap_ms"] = e0.elapsed_time(e1)
 
+    ratios = []
+
     def round_():
         evs = gemms()
         torch.cuda.synchronize()
-        alone.extend(x.elapsed_time(y) for x, y in evs[4:])
+        a_r = [x.elapsed_time(y) for x, y in evs[4:]]
+        alone.extend(a_r)
         gemm_ms = statistics.median(alone)
         n_swap = int(2.0 * G * gemm_ms / st["per_swap_ms"]) + 2
         s0 = torch.cuda.Event(enable_timing=True)
@@ -667,26 +670,36 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
         evs = gemms()
         torch.cuda.synchronize()
         win = s0.elapsed_time(s1)
-        during.extend(x.elapsed_time(y) for x, y in evs[4:]
-                      if s0.elapsed_time(x) >= 0 and s0.elapsed_time(y) <= win)
+        d_r = [x.elapsed_time(y) for x, y in evs[4:]
+               if s0.elapsed_time(x) >= 0 and s0.elapsed_time(y) <= win]
+        during.extend(d_r)
+        if d_r:
+            ratios.append(statistics.median(d_r) / statistics.median(a_r))
         swap_gbs.append(2 * n_swap * sum(sizes) / win / 1e6)
 
     L(setup)
-    for _ in range(4):
+    for _ in range(8):
         L(round_)
     st["ran"] = ctx.get_option(mp.OPT_LAST_PATH)
     if "old_cap" in st:
         L(ctx.set_option, mp.OPT_MAX_CTAS, st["old_cap"])
     t = torch.tensor([statistics.median(alone) if alone else float("nan"),
                       statistics.median(during) if during else float("nan"),
-                      1.0 if L.err is not None else 0.0], dtype=torch.float64)
+                      1.0 if L.err is not None else 0.0,
+                      statistics.median(ratios) - 1 if ratios else float("nan")], dtype=torch.float64)
     if n > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     if float(t[2]) > 0:
         return {"error": L.err or "another rank failed"}
     a_ms, d_ms = float(t[0]), float(t[1])
     return {"gemm": "bf16 8192x8192x8192 torch.matmul (cuBLAS) on the compute stream",
-            "alone_ms": a_ms, "with_swap_ms": d_ms, "slowdown": d_ms / a_ms - 1,
+            "alone_ms": a_ms, "with_swap_ms": d_ms,
+            # each round pairs an alone and a with-swap run back to back, so
+            # clock / power drift between rounds cancels in the round's ratio
+            "slowdown": float(t[3]),
+            "slowdown_pooled": d_ms / a_ms - 1,
+            "rounds": len(ratios),
+            "slowdown_per_round": [r - 1 for r in ratios],
             "swap_path": {mp.PATH_DIRECT: "direct", mp.PATH_BULK: "bulk", mp.PATH_CE: "ce"}.get(
                 st.get("ran"), args.path), "swap_max_ctas": args.gemm_cap,
             "swap_gbs_during": statistics.median(swap_gbs),
@@ -773,12 +786,13 @@ def cfg5_leg(args, mp, rank, n, device, dist):
             evs.append((e0, e1))
         return evs
 
-    alone, during, gbs = [], [], []
+    alone, during, gbs, ratios = [], [], [], []
 
     def run_alone():
         evs = gemms()
         torch.cuda.synchronize()
-        alone.extend(x.elapsed_time(y) for x, y in evs[4:])
+        st["a_r"] = [x.elapsed_time(y) for x, y in evs[4:]]
+        alone.extend(st["a_r"])
 
     def run_with_swap():
         s0 = s1 = None
@@ -795,11 +809,14 @@ def cfg5_leg(args, mp, rank, n, device, dist):
         torch.cuda.synchronize()
         if is_src:
             win = s0.elapsed_time(s1)
-            during.extend(x.elapsed_time(y) for x, y in evs[4:]
-                          if s0.elapsed_time(x) >= 0 and s0.elapsed_time(y) <= win)
+            d_r = [x.elapsed_time(y) for x, y in evs[4:]
+                   if s0.elapsed_time(x) >= 0 and s0.elapsed_time(y) <= win]
             gbs.append(2 * n_swap * sum(sizes) / win / 1e6)
         else:   # importers: the middle of the run, inside every source's window
-            during.extend(x.elapsed_time(y) for x, y in evs[4:G - 4])
+            d_r = [x.elapsed_time(y) for x, y in evs[4:G - 4]]
+        during.extend(d_r)
+        if d_r:
+            ratios.append(statistics.median(d_r) / statistics.median(st["a_r"]))
 
     guard(setup)
     for _ in range(4):
@@ -810,16 +827,17 @@ def cfg5_leg(args, mp, rank, n, device, dist):
     bad = 0
     if is_src and not err:
         bad = guard(lambda: sum(synth_dev.check(t, 5000 + rank, i) for i, t in enumerate(st["dst"]))) or 0
-    row = torch.zeros(n, 5, dtype=torch.float64)
+    row = torch.zeros(n, 6, dtype=torch.float64)
     row[rank] = torch.tensor([statistics.median(alone) if alone else float("nan"),
                               statistics.median(during) if during else float("nan"),
-                              statistics.median(gbs) if gbs else 0.0, float(bad), float(len(err))],
+                              statistics.median(gbs) if gbs else 0.0, float(bad), float(len(err)),
+                              statistics.median(ratios) - 1 if ratios else float("nan")],
                              dtype=torch.float64)
     dist.all_reduce(row)
     ctx.finalize()
     if float(row[:, 4].sum()) > 0:
         return {"error": err[0] if err else "a rank failed (see its stderr)"}
-    slow = [float(row[r, 1] / row[r, 0] - 1) for r in range(n)]
+    slow = [float(row[r, 5]) for r in range(n)]   # median over rounds of paired ratios
     return {"config": "cfg5 imbalanced all-stage swap: sources %s -> importers %s, source s swaps %s micro-batch "
                       "sets (900 MiB each, one plan), bf16 %dx%dx%d GEMMs on every rank" %
                       (sources, peers, [H - s for s in sources], M, M, M),
