@@ -426,11 +426,16 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
  * peers by a weighted round robin, so every peer link carries its share of
  * the swap at every moment (default; needed when several sources share
  * peers); 1 = plan order (peer by peer).
+ * MPRESS_OPT_PDL: 1 (default) = launch the SM kernels with programmatic
+ * dependent launch, so a swap kernel's launch and CTA ramp-up overlap the
+ * tail of the previous kernel on its stream (each kernel still waits for that
+ * grid to complete before touching memory); 0 = plain launches.
  * Invalid values -> MPRESS_ERR_ARG. */
 #define MPRESS_OPT_PATH      1
 #define MPRESS_OPT_MAX_CTAS  2
 #define MPRESS_OPT_VARIANT   3
 #define MPRESS_OPT_ORDER     4
+#define MPRESS_OPT_PDL       7
 /* Read-only (mpress_get_option): how the peer pools were mapped --
  * MPRESS_TRANSPORT_LOCAL (mpress_init_local), _VMM_FD (cuMem pools exported
  * as POSIX fds, passed over Unix sockets), or _LEGACY_IPC (cudaMalloc pools

@@ -24,6 +24,7 @@ ORDER_INTERLEAVE, ORDER_PLAN = 0, 1
 DEVICE_HOST = -1   # mpress_init_local: a pinned host pool as a peer (NEXT-4)
 OPT_TRANSPORT = 5  # read-only
 OPT_LAST_PATH = 6  # read-only: path of the last swap call
+OPT_PDL = 7
 TRANSPORT_LOCAL, TRANSPORT_VMM_FD, TRANSPORT_LEGACY_IPC = 0, 1, 2
 VARIANT_AUTO = -1
 PATH_DIRECT, PATH_BULK, PATH_CE, PATH_AUTO = 0, 1, 2, 3

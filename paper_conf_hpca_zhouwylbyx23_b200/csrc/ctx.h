@@ -103,6 +103,7 @@ struct mpress_ctx_s {
   int max_ctas = 0;
   int variant = MPRESS_VARIANT_AUTO;
   int order = MPRESS_ORDER_INTERLEAVE;
+  int pdl = 1;                        // MPRESS_OPT_PDL
   int transport = MPRESS_TRANSPORT_LOCAL;
   int last_launches = 0;
   std::vector<cudaStream_t> ce_streams;  // copy-engine comparator, one per peer

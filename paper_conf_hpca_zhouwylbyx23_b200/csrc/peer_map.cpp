@@ -469,6 +469,10 @@ extern "C" int mpress_set_option(mpress_ctx_t* c, int key, int64_t value) {
       if (value < 0 || value > (1 << 20)) return fail(MPRESS_ERR_ARG, "bad max_ctas %lld", (long long)value);
       c->max_ctas = (int)value;
       return MPRESS_OK;
+    case MPRESS_OPT_PDL:
+      if (value != 0 && value != 1) return fail(MPRESS_ERR_ARG, "MPRESS_OPT_PDL is 0 or 1, not %lld", (long long)value);
+      c->pdl = (int)value;
+      return MPRESS_OK;
     case MPRESS_OPT_ORDER:
       if (value != MPRESS_ORDER_INTERLEAVE && value != MPRESS_ORDER_PLAN)
         return fail(MPRESS_ERR_ARG, "unknown chunk order %lld", (long long)value);
@@ -494,6 +498,7 @@ extern "C" int mpress_get_option(const mpress_ctx_t* c, int key, int64_t* value)
     case MPRESS_OPT_MAX_CTAS: *value = c->max_ctas; return MPRESS_OK;
     case MPRESS_OPT_VARIANT: *value = c->variant; return MPRESS_OK;
     case MPRESS_OPT_ORDER: *value = c->order; return MPRESS_OK;
+    case MPRESS_OPT_PDL: *value = c->pdl; return MPRESS_OK;
     case MPRESS_OPT_TRANSPORT: *value = c->transport; return MPRESS_OK;
     case MPRESS_OPT_LAST_PATH: *value = c->last_path; return MPRESS_OK;
   }

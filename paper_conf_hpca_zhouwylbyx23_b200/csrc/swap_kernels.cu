@@ -170,6 +170,18 @@ struct Vec<32, HINT> {
   static __device__ __forceinline__ T ld(const T* p) { return ld_stream<HINT>(p); }
 };
 
+// Programmatic dependent launch (PDL): a swap kernel is launched with
+// programmatic stream serialization, so it may start while the previous
+// kernel of its stream is still draining.  It first waits for that grid to
+// complete and flush (griddepcontrol.wait: a no-op without a programmatic
+// predecessor), then lets its own successor launch early.  Only launch
+// latency and CTA ramp-up overlap, never data: ordering stays exact for any
+// predecessor (a producing GEMM, the matching swap-out, a user kernel).
+__device__ __forceinline__ void pdl_enter() {
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+
 // ---------------------------------------------------------------- direct path
 
 struct Span {
@@ -201,6 +213,7 @@ mp_swap_direct(const __grid_constant__ CopyTable<CAP> t) {
   // critical path of a latency-bound CTA (<= 1 CTA per SM: +50% at 32 CTAs).
   // With >= 2 CTAs per SM the memory system is saturated anyway and issuing
   // the stores first measured ~6% faster (tools/ab.py), so PF is off there.
+  pdl_enter();
   Cursor<CAP> cur(t);
   uint32_t c, s;
   if (!cur.next(&c, &s)) return;
@@ -338,6 +351,7 @@ mp_swap_bulk(const __grid_constant__ CopyTable<CAP> t) {
   __shared__ uint32_t ring_bytes[STAGES];
   const uint32_t lane = threadIdx.x;
 
+  pdl_enter();
   if (lane == 0) {
     for (int k = 0; k < STAGES; ++k) mbar_init(&bars[k], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -494,7 +508,7 @@ int prepare(KernelFn<CAP> k, const Shape& sh) {
 // CTAs between the groups in proportion to their chunks, launch.
 template <int CAP>
 int launch_batch(int path, int variant, int dir, const CopyDesc* d, const int* gid, uint32_t n,
-                 uint32_t shift, int cap, int sms, cudaStream_t stream, bool* launched) {
+                 uint32_t shift, int cap, int sms, bool pdl, cudaStream_t stream, bool* launched) {
   CopyTable<CAP> t;
   t.n = n;
   t.pad = 0;
@@ -525,8 +539,18 @@ int launch_batch(int path, int variant, int dir, const CopyDesc* d, const int* g
   const Shape& sh = shape_of(path, variant);
   KernelFn<CAP> k = kernel_for<CAP>(path, variant, dir, (int)grid <= sms);
   MP_TRY(prepare<CAP>(k, sh));
-  k<<<grid, sh.threads, sh.smem, stream>>>(t);
-  cudaError_t e = cudaGetLastError();
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(sh.threads);
+  cfg.dynamicSmemBytes = sh.smem;
+  cfg.stream = stream;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = pdl ? 1 : 0;
+  cudaError_t e = cudaLaunchKernelEx(&cfg, k, t);
+  if (e == cudaSuccess) e = cudaGetLastError();
   if (e != cudaSuccess) return fail(MPRESS_ERR_CUDA, "swap kernel launch: %s", cudaGetErrorString(e));
   *launched = true;
   return MPRESS_OK;
@@ -582,7 +606,7 @@ int preload_kernels() {
 }
 
 int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* group, size_t n,
-                int max_ctas, cudaStream_t stream, int* launches) {
+                int max_ctas, bool pdl, cudaStream_t stream, int* launches) {
   int dev = 0, sms = 0;
   if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess)
     return fail(MPRESS_ERR_CUDA, "cannot query the SM count");
@@ -618,11 +642,11 @@ int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* gr
     const int* g = group ? group + base : nullptr;
     bool launched = false;
     if (m <= 16)
-      MP_TRY(launch_batch<16>(path, variant, dir, d + base, g, m, shift, cap, sms, stream, &launched));
+      MP_TRY(launch_batch<16>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, stream, &launched));
     else if (m <= 128)
-      MP_TRY(launch_batch<128>(path, variant, dir, d + base, g, m, shift, cap, sms, stream, &launched));
+      MP_TRY(launch_batch<128>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, stream, &launched));
     else
-      MP_TRY(launch_batch<kMaxDescPerLaunch>(path, variant, dir, d + base, g, m, shift, cap, sms, stream, &launched));
+      MP_TRY(launch_batch<kMaxDescPerLaunch>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, stream, &launched));
     if (launched && launches) ++*launches;
   }
   return MPRESS_OK;

@@ -34,6 +34,7 @@ def setup(sizes, peers_n, copies=1):
     part = [[0] * world for _ in range(world)]
     part[0] = [copies * u * mp.DEFAULT_GRANULE for u in pl.units]
     ctx = mp.Context.local(world, 0, [0] * world, part)
+    ctx.set_option(mp.OPT_PDL, int(os.environ.get("SWEEP_PDL", "1")))
     src = [torch.empty(s, dtype=torch.uint8, device="cuda") for s in sizes]
     for i, t in enumerate(src):
         synth_dev.fill(t, 77, i)
@@ -98,7 +99,7 @@ def sizes_sweep():
     for peers_n in (1, 3, 7):
         for size in workloads.cfg4_sizes():
             ctx, pl, src, dst = setup([size], peers_n, copies=2)
-            for name in ("direct", "bulk", "ce", "ce_batch"):
+            for name in os.environ.get("SWEEP_SIZE_PATHS", "direct,bulk,ce,ce_batch").split(","):
                 ctx.set_option(mp.OPT_PATH, PATHS[name.split("_")[0]])
                 if name == "ce_batch":
                     ctx.set_option(mp.OPT_VARIANT, 1)   # one cudaMemcpyBatchAsync
