@@ -54,6 +54,8 @@ def parse():
     ap.add_argument("--max-ctas", type=int, default=0)
     ap.add_argument("--variant", type=int, default=-1, help="kernel shape within --path (-1 = auto)")
     ap.add_argument("--no-pdl", action="store_true", help="plain launches instead of programmatic dependent launch")
+    ap.add_argument("--pdl", type=int, default=1, choices=[0, 1, 2],
+                    help="MPRESS_OPT_PDL: 0 never, 1 uncapped grids only (default), 2 always")
     ap.add_argument("--micro-batches", type=int, default=MICRO_BATCHES)
     ap.add_argument("--e2e-steps", type=int, default=16)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -228,7 +230,7 @@ def workload_config(args, n):
              "ranks over NVLink (every rank a source and an importer)" % (args.micro_batches, n - 1)
     return {"workload": wl, "tensors_per_micro_batch": 47, "micro_batch_bytes": 900 << 20,
             "micro_batches": args.micro_batches, "peers": 3 if n == 1 else n - 1,
-            "path": args.path, "variant": args.variant, "max_ctas": args.max_ctas, "pdl": not args.no_pdl,
+            "path": args.path, "variant": args.variant, "max_ctas": args.max_ctas, "pdl": 0 if args.no_pdl else args.pdl,
             "l2": "inputs %.2f GiB per rank > 126 MB L2: no flush needed" %
                   (args.micro_batches * 900 / 1024)}
 
@@ -297,7 +299,7 @@ def main():
     ctx.set_option(mp.OPT_PATH, path)
     ctx.set_option(mp.OPT_VARIANT, args.variant)
     ctx.set_option(mp.OPT_MAX_CTAS, args.max_ctas)
-    ctx.set_option(mp.OPT_PDL, 0 if args.no_pdl else 1)
+    ctx.set_option(mp.OPT_PDL, 0 if args.no_pdl else args.pdl)
 
     seed0 = 2000 + 100 * rank
     src = [[torch.empty(s, dtype=torch.uint8, device="cuda") for s in sizes] for _ in range(mb)]
@@ -716,6 +718,8 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
             "slowdown_per_round": [r - 1 for r in ratios],
             "swap_path": {mp.PATH_DIRECT: "direct", mp.PATH_BULK: "bulk", mp.PATH_CE: "ce"}.get(
                 st.get("ran"), args.path), "swap_max_ctas": args.gemm_cap,
+            # MPRESS_OPT_PDL 1 (default) launches a capped grid without PDL
+            "swap_pdl_mode": ctx.get_option(mp.OPT_PDL),
             "swap_gbs_during": statistics.median(swap_gbs),
             "gemms_counted": len(during),
             "note": ("N=1 loopback: the swap's bytes also load the GEMM's HBM (2 B per swapped "

@@ -426,10 +426,13 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
  * peers by a weighted round robin, so every peer link carries its share of
  * the swap at every moment (default; needed when several sources share
  * peers); 1 = plan order (peer by peer).
- * MPRESS_OPT_PDL: 1 (default) = launch the SM kernels with programmatic
- * dependent launch, so a swap kernel's launch and CTA ramp-up overlap the
- * tail of the previous kernel on its stream (each kernel still waits for that
- * grid to complete before touching memory); 0 = plain launches.
+ * MPRESS_OPT_PDL: programmatic dependent launch of the SM kernels, so a swap
+ * kernel's launch and CTA ramp-up overlap the tail of the previous kernel on
+ * its stream (each kernel still waits for that grid to complete before
+ * touching memory).  1 (default) = only for an uncapped grid (MAX_CTAS 0 or
+ * above the SM count); a capped swap runs beside a GEMM, and there PDL chains
+ * of swap kernels cost the bf16 8192^3 cuBLAS GEMM +60% instead of +6-9%
+ * (profiles/r01/pdl_gemm_ab.txt); 2 = always; 0 = never.
  * Invalid values -> MPRESS_ERR_ARG. */
 #define MPRESS_OPT_PATH      1
 #define MPRESS_OPT_MAX_CTAS  2

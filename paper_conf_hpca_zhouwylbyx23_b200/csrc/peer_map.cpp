@@ -470,7 +470,7 @@ extern "C" int mpress_set_option(mpress_ctx_t* c, int key, int64_t value) {
       c->max_ctas = (int)value;
       return MPRESS_OK;
     case MPRESS_OPT_PDL:
-      if (value != 0 && value != 1) return fail(MPRESS_ERR_ARG, "MPRESS_OPT_PDL is 0 or 1, not %lld", (long long)value);
+      if (value < 0 || value > 2) return fail(MPRESS_ERR_ARG, "MPRESS_OPT_PDL is 0, 1 or 2, not %lld", (long long)value);
       c->pdl = (int)value;
       return MPRESS_OK;
     case MPRESS_OPT_ORDER:

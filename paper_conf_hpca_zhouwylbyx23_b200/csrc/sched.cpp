@@ -157,7 +157,7 @@ int run_copy(mpress_ctx_s* c, int dir, const std::vector<CopyDesc>& d,
   if (path != MPRESS_PATH_CE)
     return launch_copy(path, c->variant, dir, d.data(),
                        c->order == MPRESS_ORDER_INTERLEAVE ? desc_peer.data() : nullptr, d.size(), c->max_ctas,
-                       c->pdl != 0, stream, &c->last_launches);
+                       c->pdl, stream, &c->last_launches);
 
   // Copy-engine comparator, variant 1: the whole swap as one
   // cudaMemcpyBatchAsync on `stream` (CUDA 12.8+); the driver spreads the

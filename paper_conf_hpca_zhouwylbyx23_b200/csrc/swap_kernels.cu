@@ -606,10 +606,16 @@ int preload_kernels() {
 }
 
 int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* group, size_t n,
-                int max_ctas, bool pdl, cudaStream_t stream, int* launches) {
+                int max_ctas, int pdl_mode, cudaStream_t stream, int* launches) {
   int dev = 0, sms = 0;
   if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess)
     return fail(MPRESS_ERR_CUDA, "cannot query the SM count");
+  // PDL (MPRESS_OPT_PDL): mode 1 only for an uncapped grid.  A capped swap
+  // runs beside a GEMM, and there a PDL chain of swap kernels (the next one
+  // launched early, parked in griddepcontrol.wait) cost the concurrent cuBLAS
+  // GEMM +60% instead of +6-9% (profiles/r01/pdl_gemm_ab.txt).
+  const bool capped = max_ctas > 0 && max_ctas <= sms;
+  const bool pdl = pdl_mode == 2 || (pdl_mode == 1 && !capped);
   if (variant == MPRESS_VARIANT_AUTO) {
     // direct, capped grid (<= one CTA per SM, i.e. beside a GEMM): 128-thread
     // CTAs fit in the registers and shared memory a cuBLAS GEMM CTA leaves

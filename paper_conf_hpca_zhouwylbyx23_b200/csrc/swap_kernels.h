@@ -26,11 +26,12 @@ enum CopyDir { kDirOut = 0, kDirIn = 1 };
 
 // Enqueue kernels moving every descriptor on `stream`; `path` is
 // MPRESS_PATH_DIRECT or MPRESS_PATH_BULK, `variant` its kernel shape;
-// `max_ctas` caps the grid (0 = the variant's default grid); `pdl` launches
-// with programmatic stream serialization.  Adds the number
+// `max_ctas` caps the grid (0 = the variant's default grid); `pdl_mode`
+// (MPRESS_OPT_PDL: 0 never, 1 uncapped grids only, 2 always) launches with
+// programmatic stream serialization.  Adds the number
 // of kernel launches to *launches.  Returns MPRESS_OK or MPRESS_ERR_*.
 int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* group, size_t n,
-                int max_ctas, bool pdl,
+                int max_ctas, int pdl_mode,
                 cudaStream_t stream, int* launches);
 
 // Default grid of a path/variant on the current device (SMs x CTAs per SM).
