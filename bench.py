@@ -63,6 +63,8 @@ def parse():
     ap.add_argument("--gemm-cap", type=int, default=64,
                     help="swap grid cap (CTAs = SMs touched) while the concurrent GEMM runs")
     ap.add_argument("--no-gemm", action="store_true")
+    ap.add_argument("--gemm-settle-s", type=float, default=2.0,
+                    help="back-to-back GEMMs before the GEMM-slowdown rounds (power state)")
     ap.add_argument("--gemm-n", type=int, default=8192, help="GEMM size of the N>1 config-5 leg")
     ap.add_argument("--no-cfg5", action="store_true",
                     help="N>1: skip the config-5 leg (imbalanced swap + GEMM on every rank)")
@@ -665,6 +667,13 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
         gemms()
         torch.cuda.synchronize()
         st["per_swap_ms"] = e0.elapsed_time(e1)
+        # Settle the power state first: a B200 runs this GEMM at ~1670 TFLOP/s
+        # in a burst and ~1400 sustained (MEASURED_PEAKS.json), and rounds that
+        # straddle the drop mix the two regimes into the ratio.
+        t0 = time.time()
+        while time.time() - t0 < args.gemm_settle_s:
+            gemms()
+            torch.cuda.synchronize()
 
     ratios = []
 
@@ -710,6 +719,8 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
     a_ms, d_ms = float(t[0]), float(t[1])
     return {"gemm": "bf16 8192x8192x8192 torch.matmul (cuBLAS) on the compute stream",
             "alone_ms": a_ms, "with_swap_ms": d_ms,
+            "alone_tflops": 2 * M * N * K / (a_ms / 1e3) / 1e12,
+            "settle_s": args.gemm_settle_s,
             # each round pairs an alone and a with-swap run back to back, so
             # clock / power drift between rounds cancels in the round's ratio
             "slowdown": float(t[3]),
@@ -793,6 +804,10 @@ def cfg5_leg(args, mp, rank, n, device, dist):
             torch.cuda.synchronize()
             st["per_swap_ms"] = e0.elapsed_time(e1)
         torch.cuda.synchronize()
+        t0 = time.time()   # settle the power state (see gemm_interference)
+        while time.time() - t0 < args.gemm_settle_s:
+            gemms()
+            torch.cuda.synchronize()
 
     def gemms():
         evs = []
