@@ -7,6 +7,7 @@ keeps the driver's contract; this explains it.
   python tools/sweep.py paths        # cfg2 micro-batch, every path x cap
   python tools/sweep.py sizes        # cfg4 sizes 4 KiB .. 4 GiB, 1/3/7 peers
   python tools/sweep.py gemm         # GEMM slowdown vs swap path x cap
+  python tools/sweep.py power        # GEMM slowdown vs SM clock and board power
 """
 import json
 import os
@@ -245,6 +246,111 @@ def gemm():
     ctx.finalize()
 
 
+def power():
+    """Where the concurrent GEMM's slowdown comes from: for each swap setting,
+    SECONDS of back-to-back bf16 8192^3 GEMMs with the swap looping beside
+    them for the whole window, NVML sampling the SM clock and board power
+    every 20 ms; alone windows alternate with the swap windows.  If the GEMM
+    loses time in proportion to the SM clock drop, the interference is the
+    power cap (moving bytes costs watts), not SMs taken by the swap."""
+    import threading
+    import time
+
+    import pynvml
+    pynvml.nvmlInit()
+    nv = pynvml.nvmlDeviceGetHandleByIndex(torch.cuda.current_device())
+    seconds = float(os.environ.get("POWER_SECONDS", "3"))
+    sizes = workloads.cfg2_sizes(1)
+    nbytes = sum(sizes)
+    ctx, pl, src, dst = setup(sizes, 3)
+    comp = torch.cuda.current_stream()
+    swap = torch.cuda.Stream()
+    M = 8192
+    a = torch.randn(M, M, dtype=torch.bfloat16, device="cuda")
+    b = torch.randn(M, M, dtype=torch.bfloat16, device="cuda")
+    c = torch.empty(M, M, dtype=torch.bfloat16, device="cuda")
+
+    def sample(stop, out):
+        while not stop.is_set():
+            out.append((pynvml.nvmlDeviceGetClockInfo(nv, pynvml.NVML_CLOCK_SM),
+                        pynvml.nvmlDeviceGetPowerUsage(nv) / 1000.0))
+            time.sleep(0.02)
+
+    def window(setting):
+        if setting:
+            name, var, cap = setting
+            ctx.set_option(mp.OPT_PATH, PATHS[name])
+            if name != "ce":
+                ctx.set_option(mp.OPT_VARIANT, var)
+            ctx.set_option(mp.OPT_MAX_CTAS, cap)
+        per_pair = 0.0
+        if setting:   # one pair alone sizes the swap batch that covers 20 GEMMs
+            torch.cuda.synchronize()
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(swap)
+            h = ctx.swap_out(pl, src, stream=swap)
+            ctx.swap_in(h, dst, stream=swap)
+            e1.record(swap)
+            h.free()
+            torch.cuda.synchronize()
+            per_pair = e0.elapsed_time(e1)
+        torch.cuda.synchronize()
+        stop, smp = threading.Event(), []
+        th = threading.Thread(target=sample, args=(stop, smp))
+        th.start()
+        t0 = time.time()
+        n_gemm = n_swap = 0
+        gms = sms = 0.0
+        while time.time() - t0 < seconds:
+            g0 = torch.cuda.Event(enable_timing=True)
+            g1 = torch.cuda.Event(enable_timing=True)
+            s0 = torch.cuda.Event(enable_timing=True)
+            s1 = torch.cuda.Event(enable_timing=True)
+            k = 0
+            if setting:   # under contention a pair is slower: 1.1x alone-time cover is enough
+                k = max(1, int(1.1 * 20 * 0.75 / per_pair) + 1)
+                s0.record(swap)
+                for _ in range(k):
+                    h = ctx.swap_out(pl, src, stream=swap)
+                    ctx.swap_in(h, dst, stream=swap)
+                    h.free()
+                s1.record(swap)
+            g0.record(comp)
+            for _ in range(20):
+                torch.matmul(a, b, out=c)
+            g1.record(comp)
+            torch.cuda.synchronize()
+            n_gemm += 20
+            n_swap += k
+            gms += g0.elapsed_time(g1)
+            if setting:
+                sms += s0.elapsed_time(s1)
+        stop.set()
+        th.join()
+        keep = smp[len(smp) // 5:] or smp   # drop the ramp
+        row = {"sweep": "power", "setting": "alone" if not setting else "%s var=%d cap=%d" % setting,
+               "gemm_tflops": 2 * M ** 3 * n_gemm / (gms / 1e3) / 1e12,
+               "sm_mhz_median": statistics.median(x for x, _ in keep),
+               "power_w_median": statistics.median(w for _, w in keep), "samples": len(keep)}
+        if setting:
+            row["swap_gbs"] = 2 * n_swap * nbytes / sms / 1e6
+            row["swap_busy_over_gemm_busy"] = sms / gms
+        print(json.dumps(row), flush=True)
+        return row
+
+    window(None)   # warm to the sustained power state
+    settings = [("direct", 7, 32), ("direct", 7, 64), ("direct", 9, 64), ("direct", 7, 148), ("ce", 0, 0)]
+    for st in settings:
+        al = window(None)
+        wi = window(st)
+        print(json.dumps({"sweep": "power_pair", "setting": wi["setting"],
+                          "slowdown": al["gemm_tflops"] / wi["gemm_tflops"] - 1,
+                          "sm_clock_ratio": wi["sm_mhz_median"] / al["sm_mhz_median"],
+                          "swap_gbs": wi["swap_gbs"]}), flush=True)
+    ctx.finalize()
+
+
 if __name__ == "__main__":
     what = sys.argv[1] if len(sys.argv) > 1 else "paths"
-    {"paths": paths, "sizes": sizes_sweep, "gemm": gemm, "host": host}[what]()
+    {"paths": paths, "sizes": sizes_sweep, "gemm": gemm, "host": host, "power": power}[what]()
