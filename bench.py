@@ -53,6 +53,8 @@ def parse():
                     help="auto = the library default: bulk (TMA) at a full grid, direct when capped")
     ap.add_argument("--max-ctas", type=int, default=0)
     ap.add_argument("--variant", type=int, default=-1, help="kernel shape within --path (-1 = auto)")
+    ap.add_argument("--no-autotune", action="store_true",
+                    help="skip mpress_autotune (AUTO keeps the bulk kernel for uncapped grids)")
     ap.add_argument("--no-pdl", action="store_true", help="plain launches instead of programmatic dependent launch")
     ap.add_argument("--pdl", type=int, default=1, choices=[0, 1, 2],
                     help="MPRESS_OPT_PDL: 0 never, 1 uncapped grids only (default), 2 always")
@@ -302,6 +304,14 @@ def main():
     ctx.set_option(mp.OPT_VARIANT, args.variant)
     ctx.set_option(mp.OPT_MAX_CTAS, args.max_ctas)
     ctx.set_option(mp.OPT_PDL, 0 if args.no_pdl else args.pdl)
+    autotune = None
+    if path == mp.PATH_AUTO and not args.no_autotune:
+        # which SM kernel an uncapped AUTO swap runs on THIS run's links
+        # (loopback HBM at N=1, NVLink at N>1), measured before the timed steps
+        res = ctx.autotune(probe_bytes=256 << 20, trials=5)
+        nm = {mp.PATH_DIRECT: "direct", mp.PATH_BULK: "bulk"}
+        autotune = {"out": nm[res["out"]], "in": nm[res["in"]], "probe_bytes": 256 << 20, "trials": 5,
+                    "median_ms": res["ms"]}
 
     seed0 = 2000 + 100 * rank
     src = [[torch.empty(s, dtype=torch.uint8, device="cuda") for s in sizes] for _ in range(mb)]
@@ -321,7 +331,9 @@ def main():
     # swap-in per step (micro-batch k % mb in step k): a timing event between
     # two kernels serialises them, which would switch off the programmatic
     # dependent launch (PDL) overlap of every other launch boundary.
-    def step(record=False, k=0):
+    ran_dir = {}   # path each direction ran (MPRESS_OPT_LAST_PATH), from the first warm-up step
+
+    def step(record=False, k=0, probe_path=False):
         pl = mp.plan(world, source, per_copy, bw, sizes)              # a1
         hs = []
         tm = k % mb
@@ -331,6 +343,8 @@ def main():
                 e0 = torch.cuda.Event(enable_timing=True); e0.record(swap_stream)
             hs.append(ctx.swap_out(pl, src[m], stream=swap_stream))
             launches[0] += ctx.last_launches
+            if probe_path and m == 0:
+                ran_dir["out"] = ctx.get_option(mp.OPT_LAST_PATH)
             if rec:
                 e1 = torch.cuda.Event(enable_timing=True); e1.record(swap_stream)
                 timing["out"].append((e0, e1))
@@ -340,6 +354,8 @@ def main():
                 e0 = torch.cuda.Event(enable_timing=True); e0.record(swap_stream)
             ctx.swap_in(hs[m], dst[m], stream=swap_stream)
             launches[0] += ctx.last_launches
+            if probe_path and m == 0:
+                ran_dir["in"] = ctx.get_option(mp.OPT_LAST_PATH)
             if rec:
                 e1 = torch.cuda.Event(enable_timing=True); e1.record(swap_stream)
                 timing["in"].append((e0, e1))
@@ -347,8 +363,8 @@ def main():
         for h in hs:
             h.free()
 
-    for _ in range(args.warmup):
-        step()
+    for w in range(args.warmup):
+        step(probe_path=w == 0)
     torch.cuda.synchronize()
     if n > 1:
         dist.barrier()
@@ -388,12 +404,13 @@ def main():
     if int(bad_t.item()) != 0:
         raise SystemExit("round trip mismatch: %d bytes" % int(bad_t.item()))
 
-    ran = {mp.PATH_DIRECT: "direct", mp.PATH_BULK: "bulk", mp.PATH_CE: "ce"}.get(
-        ctx.get_option(mp.OPT_LAST_PATH), "?")
+    names = {mp.PATH_DIRECT: "direct", mp.PATH_BULK: "bulk", mp.PATH_CE: "ce"}
+    ran_by_dir = {k: names.get(v, "?") for k, v in ran_dir.items()}
     # per-kernel durations (each swap call here is exactly one kernel launch)
     dur = {k: [a.elapsed_time(b) for a, b in v] for k, v in timing.items()}
     tot = {k: sum(v) for k, v in dur.items()}
     dom = max(tot, key=tot.get)
+    ran = ran_by_dir.get(dom, "?")   # the dominant kernel's path
     avg_ms = statistics.mean(dur[dom])
     peaks, peaks_src = measured_peaks()
     if n == 1:
@@ -455,7 +472,7 @@ def main():
             "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
             "config": workload_config(args, n),
-            "swap_path_ran": ran,
+            "swap_path_ran": ran_by_dir, "autotune": autotune,
             "per_direction_gbs": per_dir,
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": launches[0], "clocks": clk, "gemm_slowdown": gemm,

@@ -446,6 +446,10 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
  * fails on any rank, or forced with the environment variable MPRESS_IPC=legacy). */
 #define MPRESS_OPT_TRANSPORT 5
 #define MPRESS_OPT_LAST_PATH 6   /* read-only: path of the last swap call */
+/* Read-only: the SM path MPRESS_PATH_AUTO takes for an uncapped grid, per
+ * direction (MPRESS_PATH_BULK until mpress_autotune measures direct faster). */
+#define MPRESS_OPT_AUTO_OUT  8
+#define MPRESS_OPT_AUTO_IN   9
 #define MPRESS_TRANSPORT_LOCAL      0
 #define MPRESS_TRANSPORT_VMM_FD     1
 #define MPRESS_TRANSPORT_LEGACY_IPC 2
@@ -457,6 +461,32 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
 #define MPRESS_PATH_CE       2
 #define MPRESS_PATH_AUTO     3
 MPRESS_API int mpress_set_option(mpress_ctx_t* ctx, int key, int64_t value);
+
+/* Measure, don't guess: which SM kernel MPRESS_PATH_AUTO should run for an
+ * uncapped grid on THIS context's links (HBM loopback on one GPU, NVLink /
+ * NVSwitch on several -- the two were only ever compared on loopback, +0.8%
+ * for bulk).  Moves `probe_bytes` (split equally over the
+ * mapped device peers, each share a multiple of 256 and at most that
+ * partition's largest free block) out of a library-owned scratch buffer into
+ * the stash partitions and back, with the direct kernel (shape 5) and the
+ * bulk kernel (shape 3), one warm-up round and then `trials` (1..64) rounds
+ * alternating which path goes first; per direction the median times decide,
+ * and bulk stays unless direct is at least 1% faster.  The result is read
+ * back with MPRESS_OPT_AUTO_OUT / _IN and used by every later AUTO swap of
+ * this context with an uncapped grid (a capped grid or a host peer still
+ * takes the direct kernel).  Runs synchronously on `stream` (NULL = legacy
+ * default stream).
+ * Collective for an mpress_init context: every rank calls it with the same
+ * `trials` (a rank without device peers only takes part in the barriers),
+ * and each probe starts on all ranks together (barriers through the
+ * exchange callback), so the probe sees the all-to-all load of a real swap.
+ * ms (may be NULL): [4] = median ms of direct out, direct in, bulk out,
+ * bulk in (0 when this rank probed nothing).
+ * Errors: MPRESS_ERR_ARG (null ctx, trials out of range, probe_bytes 0),
+ * MPRESS_ERR_STATE (a live handle: the probe uses the stash as scratch),
+ * MPRESS_ERR_CUDA, MPRESS_ERR_SYS / _PEER (exchange failed, another rank
+ * failed). */
+MPRESS_API int mpress_autotune(mpress_ctx_t* ctx, uint64_t probe_bytes, int trials, void* stream, float* ms);
 MPRESS_API int mpress_get_option(const mpress_ctx_t* ctx, int key, int64_t* value);
 
 /* ---- the swap --------------------------------------------------------------- */

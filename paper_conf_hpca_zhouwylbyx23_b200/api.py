@@ -25,6 +25,7 @@ DEVICE_HOST = -1   # mpress_init_local: a pinned host pool as a peer (NEXT-4)
 OPT_TRANSPORT = 5  # read-only
 OPT_LAST_PATH = 6  # read-only: path of the last swap call
 OPT_PDL = 7
+OPT_AUTO_OUT, OPT_AUTO_IN = 8, 9   # read-only: AUTO's uncapped-grid path per direction
 TRANSPORT_LOCAL, TRANSPORT_VMM_FD, TRANSPORT_LEGACY_IPC = 0, 1, 2
 VARIANT_AUTO = -1
 PATH_DIRECT, PATH_BULK, PATH_CE, PATH_AUTO = 0, 1, 2, 3
@@ -42,7 +43,7 @@ EXPORTED = [
     "mpress_executor_slot", "mpress_executor_restore_to", "mpress_executor_before",
     "mpress_executor_after", "mpress_executor_free", "mpress_init",
     "mpress_init_local",
-    "mpress_finalize", "mpress_stash_free", "mpress_set_option", "mpress_get_option",
+    "mpress_finalize", "mpress_stash_free", "mpress_set_option", "mpress_get_option", "mpress_autotune",
     "mpress_swap_out", "mpress_swap_in", "mpress_wait", "mpress_query", "mpress_handle_state",
     "mpress_handle_is_graph",
     "mpress_handle_slices", "mpress_handle_free", "mpress_peer_read", "mpress_last_launches",
@@ -122,6 +123,7 @@ def _load():
         "mpress_stash_free": (c_int, [P, P]),
         "mpress_set_option": (c_int, [P, c_int, c_int64]),
         "mpress_get_option": (c_int, [P, c_int, POINTER(c_int64)]),
+        "mpress_autotune": (c_int, [P, c_uint64, c_int, P, P]),
         "mpress_swap_out": (c_int, [P, P, P, P, P, POINTER(P)]),
         "mpress_swap_in": (c_int, [P, P, P, P]),
         "mpress_wait": (c_int, [P, P, P]),
@@ -508,6 +510,16 @@ class Context:
         v = c_int64()
         _check(lib.mpress_get_option(self._h, key, byref(v)))
         return v.value
+
+    def autotune(self, probe_bytes=256 << 20, trials=5, stream=None):
+        """mpress_autotune: time the direct and bulk kernels on this
+        context's links and let MPRESS_PATH_AUTO keep the faster per
+        direction (collective for a distributed context).  Returns the
+        chosen paths and the median probe times in ms."""
+        ms = (ctypes.c_float * 4)()
+        _check(lib.mpress_autotune(self._h, probe_bytes, trials, _stream(stream, self.device), ms))
+        return {"out": self.get_option(OPT_AUTO_OUT), "in": self.get_option(OPT_AUTO_IN),
+                "ms": {"direct_out": ms[0], "direct_in": ms[1], "bulk_out": ms[2], "bulk_in": ms[3]}}
 
     def stash_free(self):
         out = (c_uint64 * self.world)()

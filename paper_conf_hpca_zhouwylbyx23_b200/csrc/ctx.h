@@ -104,6 +104,9 @@ struct mpress_ctx_s {
   int variant = MPRESS_VARIANT_AUTO;
   int order = MPRESS_ORDER_INTERLEAVE;
   int pdl = 1;                        // MPRESS_OPT_PDL
+  // SM path MPRESS_PATH_AUTO takes for an uncapped grid, per direction
+  // (kDirOut, kDirIn); bulk until mpress_autotune measures otherwise
+  int auto_path[2] = {MPRESS_PATH_BULK, MPRESS_PATH_BULK};
   int transport = MPRESS_TRANSPORT_LOCAL;
   int last_launches = 0;
   std::vector<cudaStream_t> ce_streams;  // copy-engine comparator, one per peer

@@ -144,14 +144,15 @@ int run_copy(mpress_ctx_s* c, int dir, const std::vector<CopyDesc>& d,
   c->last_launches = 0;
   int path = c->path;
   if (path == MPRESS_PATH_AUTO) {
-    // bulk at a full grid (TMA, +0.8% over direct on B200, profiles/r01);
+    // full grid: bulk (TMA, +0.8% over direct on B200 loopback, profiles/r01)
+    // unless mpress_autotune measured direct faster on this context's links;
     // direct when the grid is capped to <= one CTA per SM (small CTAs that
     // co-reside with a GEMM) or a peer is pinned host memory
     int dev = 0, sms = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     const bool capped = c->max_ctas > 0 && c->max_ctas <= sms;
-    path = (capped || c->host_peer) ? MPRESS_PATH_DIRECT : MPRESS_PATH_BULK;
+    path = (capped || c->host_peer) ? MPRESS_PATH_DIRECT : c->auto_path[dir];
   }
   c->last_path = path;
   if (path != MPRESS_PATH_CE)
@@ -468,5 +469,129 @@ extern "C" int mpress_handle_free(mpress_ctx_t* c, mpress_handle_t* h, int force
   // An IN_PENDING handle's slices stay fenced: the fences share its event.
   c->handles.erase(h);
   delete h;
+  return MPRESS_OK;
+}
+
+namespace mpress {
+namespace {
+
+// Collective step of mpress_autotune: all ranks learn whether every rank is
+// still fine (and start the next probe together).  Local contexts: no-op.
+int autotune_barrier(mpress_ctx_t* c, int rc) {
+  if (c->local) return rc;
+  int32_t ok = rc == MPRESS_OK;
+  std::vector<int32_t> all(c->world);
+  if (c->exchange(c->exchange_user, &ok, sizeof ok, all.data()) != 0)
+    return rc != MPRESS_OK ? rc : fail(MPRESS_ERR_SYS, "mpress_autotune: exchange failed");
+  for (int r = 0; r < c->world; ++r)
+    if (!all[r]) return rc != MPRESS_OK ? rc : fail(MPRESS_ERR_PEER, "mpress_autotune: rank %d failed", r);
+  return rc;
+}
+
+float median(std::vector<float> v) {
+  if (v.empty()) return 0.f;
+  std::sort(v.begin(), v.end());
+  return v[v.size() / 2];
+}
+
+}  // namespace
+}  // namespace mpress
+
+// Runtime choice of the SM path MPRESS_PATH_AUTO takes for an uncapped grid:
+// time both SM kernels on this context's own peers and keep the faster per
+// direction (include/mpress.h).  The stash partitions serve as the probe's
+// scratch, so no handle may be live.
+extern "C" int mpress_autotune(mpress_ctx_t* c, uint64_t probe_bytes, int trials, void* stream_, float* ms_out) {
+  if (!c || trials < 1 || trials > 64 || probe_bytes == 0)
+    return fail(MPRESS_ERR_ARG, "mpress_autotune: bad argument");
+  std::lock_guard<std::mutex> lk(c->mu);
+  DeviceGuard g(c->device);
+  cudaStream_t stream = static_cast<cudaStream_t>(stream_);
+  int rc = c->handles.empty() ? MPRESS_OK
+                              : fail(MPRESS_ERR_STATE, "mpress_autotune: %zu live handle(s); the probe uses the "
+                                                       "stash as scratch", c->handles.size());
+  // probe layout: an equal share of probe_bytes on every mapped device peer
+  std::vector<int> peers;
+  if (rc == MPRESS_OK)
+    for (int p = 0; p < c->world; ++p)
+      if (p != c->source && c->parts[p].base && !(c->host_peer && c->maps[p].host)) peers.push_back(p);
+  std::vector<uint64_t> off(c->world, UINT64_MAX), len(c->world, 0);
+  uint64_t total = 0;
+  if (rc == MPRESS_OK && !peers.empty()) {
+    const uint64_t share = probe_bytes / peers.size() / MPRESS_ALIGN * MPRESS_ALIGN;
+    for (int p : peers) {
+      uint64_t best = 0;
+      for (auto& kv : c->parts[p].free) best = std::max(best, kv.second);
+      len[p] = std::min(share, best / MPRESS_ALIGN * MPRESS_ALIGN);
+      if (len[p] == 0 || !alloc_slice(&c->parts[p], len[p], &off[p])) { len[p] = 0; continue; }
+      total += len[p];
+    }
+  }
+  uint8_t *src = nullptr, *dst = nullptr;
+  cudaEvent_t ev[3] = {nullptr, nullptr, nullptr};
+  if (rc == MPRESS_OK && total) {
+    cudaError_t e = cudaMalloc(&src, total);
+    if (e == cudaSuccess) e = cudaMalloc(&dst, total);
+    if (e == cudaSuccess) e = cudaMemsetAsync(src, 0, total, stream);
+    for (int i = 0; i < 3 && e == cudaSuccess; ++i) e = cudaEventCreate(&ev[i]);
+    if (e != cudaSuccess) rc = cuda_fail(e, "mpress_autotune: probe buffers");
+  }
+  std::vector<CopyDesc> dout, din;
+  std::vector<int> grp;
+  uint64_t at = 0;
+  for (int p : peers) {
+    if (!len[p]) continue;
+    dout.push_back({src + at, c->parts[p].base + off[p], len[p]});
+    din.push_back({c->parts[p].base + off[p], dst + at, len[p]});
+    grp.push_back(p);
+    at += len[p];
+  }
+  // warm-up round (-1), then `trials` rounds alternating which path goes first
+  const int paths[2] = {MPRESS_PATH_DIRECT, MPRESS_PATH_BULK};
+  std::vector<float> t[2][2];  // [path][dir]
+  for (int r = -1; r < trials; ++r) {
+    for (int k = 0; k < 2; ++k) {
+      const int pi = (r & 1) ? 1 - k : k;
+      rc = autotune_barrier(c, rc);
+      if (rc != MPRESS_OK || dout.empty()) continue;
+      int launches = 0;
+      cudaEventRecord(ev[0], stream);
+      rc = launch_copy(paths[pi], MPRESS_VARIANT_AUTO, kDirOut, dout.data(), grp.data(), dout.size(), 0, c->pdl,
+                       stream, &launches);
+      cudaEventRecord(ev[1], stream);
+      if (rc == MPRESS_OK)
+        rc = launch_copy(paths[pi], MPRESS_VARIANT_AUTO, kDirIn, din.data(), grp.data(), din.size(), 0, c->pdl,
+                         stream, &launches);
+      cudaEventRecord(ev[2], stream);
+      cudaError_t e = cudaEventSynchronize(ev[2]);
+      float a = 0, b = 0;
+      if (e == cudaSuccess) e = cudaEventElapsedTime(&a, ev[0], ev[1]);
+      if (e == cudaSuccess) e = cudaEventElapsedTime(&b, ev[1], ev[2]);
+      if (e != cudaSuccess && rc == MPRESS_OK) rc = cuda_fail(e, "mpress_autotune: probe timing");
+      if (r >= 0) {
+        t[pi][kDirOut].push_back(a);
+        t[pi][kDirIn].push_back(b);
+      }
+    }
+  }
+  rc = autotune_barrier(c, rc);
+  for (int p : peers)
+    if (len[p]) free_slice(&c->parts[p], off[p], len[p]);
+  cudaFree(src);
+  cudaFree(dst);
+  for (auto e : ev) if (e) cudaEventDestroy(e);
+  if (rc != MPRESS_OK) return rc;
+  float m[2][2];
+  for (int pi = 0; pi < 2; ++pi)
+    for (int d = 0; d < 2; ++d) m[pi][d] = median(t[pi][d]);
+  if (!dout.empty())
+    for (int d = 0; d < 2; ++d)  // bulk stays unless direct is >= 1% faster
+      c->auto_path[d] = m[0][d] < 0.99f * m[1][d] ? MPRESS_PATH_DIRECT : MPRESS_PATH_BULK;
+  if (ms_out) {
+    ms_out[0] = m[0][kDirOut];
+    ms_out[1] = m[0][kDirIn];
+    ms_out[2] = m[1][kDirOut];
+    ms_out[3] = m[1][kDirIn];
+  }
   return MPRESS_OK;
 }

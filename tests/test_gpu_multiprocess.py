@@ -47,6 +47,10 @@ def _worker(rank, world, port, outdir, path, transport="fd"):
         ctx.set_option(mp.OPT_PATH, path)
         want = mp.TRANSPORT_LEGACY_IPC if transport == "legacy" else mp.TRANSPORT_VMM_FD
         assert ctx.get_option(mp.OPT_TRANSPORT) == want
+        if path == mp.PATH_AUTO:   # collective probe on the real (here: loopback) peers
+            res = ctx.autotune(probe_bytes=8 << 20, trials=2)
+            assert res["out"] in (mp.PATH_DIRECT, mp.PATH_BULK) and res["in"] in (mp.PATH_DIRECT, mp.PATH_BULK)
+            assert all(v > 0 for v in res["ms"].values()), res
         per_copy = [r // 2 for r in spare]
         pl = mp.plan(world, rank, per_copy, bwm[rank], sizes, 4096)
         o = oracle.plan(world, rank, per_copy, bwm[rank], sizes, 4096)
@@ -84,7 +88,7 @@ def _worker(rank, world, port, outdir, path, transport="fd"):
     dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("path,transport", [(0, "fd"), (1, "fd"), (0, "legacy")])
+@pytest.mark.parametrize("path,transport", [(0, "fd"), (1, "fd"), (0, "legacy"), (3, "fd")])
 def test_two_processes_one_gpu(path, transport):
     with tempfile.TemporaryDirectory() as d:
         tmp.spawn(_worker, args=(2, _free_port(), d, path, transport), nprocs=2, join=True)
@@ -120,6 +124,13 @@ def _cfg5_worker(rank, world, port, outdir):
     err = "" if part == opart else "partition differs from the oracle"
     ctx = mp.Context.distributed(0, world, rank, part)
     try:
+        # collective: the importers (no peers of their own) only join the barriers
+        res = ctx.autotune(probe_bytes=4 << 20, trials=1)
+        if rank in peers:
+            assert all(v == 0 for v in res["ms"].values()), res
+            assert res["out"] == res["in"] == mp.PATH_BULK
+        else:
+            assert all(v > 0 for v in res["ms"].values()), res
         if rank in sources and not err:
             sizes = sizes_of(rank)
             rem = list(spare)

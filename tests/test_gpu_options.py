@@ -120,3 +120,47 @@ def test_pdl_modes():
                     h.free()
     finally:
         ctx.finalize()
+
+
+def test_autotune_local():
+    """mpress_autotune on a loopback context: both kernels timed per
+    direction, the choice is one of them, later AUTO swaps with an uncapped
+    grid run the chosen path per direction (capped ones stay direct), and
+    everything round-trips bit-exactly.  A live handle refuses the probe."""
+    from synth import device as synth_dev
+    world = 4
+    sizes = [(7 << 20) + 3, 1 << 20, 33]
+    pl = mp.plan(world, 0, [0] + [1 << 30] * 3, [0, 1, 1, 1], sizes)
+    part = [[0] + [2 * u * 65536 for u in pl.units[1:]]] + [[0] * world for _ in range(3)]
+    ctx = mp.Context.local(world, 0, [0] * world, part)
+    try:
+        assert ctx.get_option(mp.OPT_AUTO_OUT) == ctx.get_option(mp.OPT_AUTO_IN) == mp.PATH_BULK
+        for bad in ((0, 3), (1 << 20, 0), (1 << 20, 65)):
+            with pytest.raises(mp.MPressError) as ei:
+                ctx.autotune(probe_bytes=bad[0], trials=bad[1])
+            assert ei.value.code == mp.ERR_ARG
+        free0 = ctx.stash_free()
+        res = ctx.autotune(probe_bytes=64 << 20, trials=3)
+        assert ctx.stash_free() == free0   # the probe's slices went back
+        assert res["out"] in (mp.PATH_DIRECT, mp.PATH_BULK) and res["in"] in (mp.PATH_DIRECT, mp.PATH_BULK)
+        assert all(v > 0 for v in res["ms"].values()), res
+        src = [torch.empty(n, dtype=torch.uint8, device="cuda") for n in sizes]
+        for i, t in enumerate(src):
+            synth_dev.fill(t, 61, i)
+        torch.cuda.synchronize()
+        for cap in (0, 16):
+            ctx.set_option(mp.OPT_MAX_CTAS, cap)
+            dst = [torch.zeros(n, dtype=torch.uint8, device="cuda") for n in sizes]
+            h = ctx.swap_out(pl, src)
+            assert ctx.get_option(mp.OPT_LAST_PATH) == (res["out"] if cap == 0 else mp.PATH_DIRECT)
+            if cap == 0:
+                with pytest.raises(mp.MPressError) as ei:
+                    ctx.autotune()
+                assert ei.value.code == mp.ERR_STATE
+            ctx.swap_in(h, dst)
+            assert ctx.get_option(mp.OPT_LAST_PATH) == (res["in"] if cap == 0 else mp.PATH_DIRECT)
+            torch.cuda.synchronize()
+            assert all(synth_dev.check(d, 61, i) == 0 for i, d in enumerate(dst)), cap
+            h.free()
+    finally:
+        ctx.finalize()
