@@ -396,10 +396,12 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
  * 1 = SM kernel, bulk-async copies (the SM's TMA engine, cp.async.bulk)
  * staged through shared memory; 2 = copy engines (cudaMemcpyAsync per stripe
  * on per-peer streams, the measured comparator); 3 = MPRESS_PATH_AUTO
- * (default): per launch, bulk at a full grid (max_ctas 0 or above the SM
- * count: +0.8% over direct, profiles/r01), direct when the grid is capped to
- * <= one CTA per SM (its 128-thread CTAs co-reside with a GEMM, bulk CTAs'
- * shared memory does not) or when a peer is a host pool.
+ * (default): per launch, at a full grid (max_ctas 0 or above the SM count)
+ * the kernel mpress_autotune measured faster on this context's links for
+ * that direction (bulk until then: +0.8% over direct on one B200,
+ * profiles/r01), direct when the grid is capped to <= one CTA per SM (its
+ * 128-thread CTAs co-reside with a GEMM, bulk CTAs' shared memory does not)
+ * or when a peer is a host pool.
  * MPRESS_OPT_LAST_PATH (read-only) reports the path the last swap call ran.
  * Setting the path resets the variant to MPRESS_VARIANT_AUTO; under
  * MPRESS_PATH_AUTO only MPRESS_VARIANT_AUTO is accepted.
