@@ -182,6 +182,9 @@ def test_init_argument_errors_without_gpu():
     assert mp.lib.mpress_init_local(2, 0, devs, bad_align, ctypes.byref(h)) == mp.ERR_ARG
     assert mp.lib.mpress_init_local(2, 2, devs, bad_align, ctypes.byref(h)) == mp.ERR_ARG
     assert mp.lib.mpress_finalize(None) == 0
+    assert mp.lib.mpress_autotune(None, 1 << 20, 3, None, None) == mp.ERR_ARG
+    v = ctypes.c_int64()
+    assert mp.lib.mpress_get_option(None, mp.OPT_AUTO_OUT, ctypes.byref(v)) == mp.ERR_ARG
     with pytest.raises(mp.MPressError) as ei:
         mp.plan(3, 0, [0, 1], [0, 1, 1], [10])
     assert ei.value.code == mp.ERR_ARG
