@@ -1,5 +1,6 @@
-"""Full-size parity at BASELINE.json's sizes, in the launch configuration
-bench.py times (default path and grid): sampled stash windows against the
+"""Full-size parity at BASELINE.json's sizes, in the launch configurations
+bench.py times (default grid; AUTO's default kernel and the direct kernel,
+the two mpress_autotune chooses between): sampled stash windows against the
 oracle's plan + the generator (the oracle computes each window one by one),
 and the round trip checked on the device against the generator for every
 byte.  Plus compute-sanitizer memcheck of the smoke path."""
@@ -22,7 +23,7 @@ pytestmark = pytest.mark.gpu
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
-def _sampled_roundtrip(world, source, spare, bw, sizes, seed, samples=64):
+def _sampled_roundtrip(world, source, spare, bw, sizes, seed, samples=64, path=None):
     o = oracle.plan(world, source, spare, bw, sizes)
     pl = mp.plan(world, source, spare, bw, sizes)
     assert pl.stripes == [tuple(s) for s in o["stripes"]]
@@ -31,6 +32,8 @@ def _sampled_roundtrip(world, source, spare, bw, sizes, seed, samples=64):
     part[source] = [u * o["G"] for u in pl.units]
     ctx = mp.Context.local(world, source, [0] * world, part)
     try:
+        if path is not None:
+            ctx.set_option(mp.OPT_PATH, path)
         src = []
         for i, n in enumerate(sizes):
             t = torch.empty(n, dtype=torch.uint8, device="cuda")
@@ -70,31 +73,34 @@ def _sampled_roundtrip(world, source, spare, bw, sizes, seed, samples=64):
     return o
 
 
-def test_config3_gpt_adam_states_full_size():
+@pytest.mark.parametrize("path", [None, mp.PATH_DIRECT], ids=["auto", "direct"])
+def test_config3_gpt_adam_states_full_size(path):
     """BJ:9: 100 fp32 Adam m/v tensors (12.21 GB) -> peers 5,6,7 with 8/8/2 GiB
     spare: the cap binds on peer 7 (water-fill)."""
     c = workloads.CONFIGS[3]
     spare = workloads.spare_vector(8, 0, c["peers"], spare_by_peer=c["spare_by_peer"])
     bw = workloads.bw_vector(8, 0, c["peers"])
-    o = _sampled_roundtrip(8, 0, spare, bw, workloads.cfg3_sizes(), seed=3000)
+    o = _sampled_roundtrip(8, 0, spare, bw, workloads.cfg3_sizes(), seed=3000, path=path)
     assert o["units"][7] * o["G"] == 2 << 30
 
 
-def test_config4_largest_size_seven_peers():
+@pytest.mark.parametrize("path", [None, mp.PATH_DIRECT], ids=["auto", "direct"])
+def test_config4_largest_size_seven_peers(path):
     """BJ:10: one 4 GiB uint8 tensor striped over 7 peers."""
     peers = list(range(1, 8))
     spare = workloads.spare_vector(8, 0, peers, spare=8 << 30)
     bw = workloads.bw_vector(8, 0, peers)
-    _sampled_roundtrip(8, 0, spare, bw, [4 << 30], seed=4000)
+    _sampled_roundtrip(8, 0, spare, bw, [4 << 30], seed=4000, path=path)
 
 
-def test_config2_x8_single_batch_full_size():
+@pytest.mark.parametrize("path", [None, mp.PATH_DIRECT], ids=["auto", "direct"])
+def test_config2_x8_single_batch_full_size(path):
     """BJ:8: the 8 in-flight micro-batches (376 tensors, 7.03 GiB) as one plan
     over 3 peers."""
     peers = [1, 2, 3]
     spare = workloads.spare_vector(4, 0, peers, spare=24 << 30)
     bw = workloads.bw_vector(4, 0, peers)
-    _sampled_roundtrip(4, 0, spare, bw, workloads.cfg2_sizes(8), seed=2000)
+    _sampled_roundtrip(4, 0, spare, bw, workloads.cfg2_sizes(8), seed=2000, path=path)
 
 
 @pytest.mark.skipif(shutil.which("compute-sanitizer") is None and
