@@ -310,8 +310,9 @@ def main():
         # (loopback HBM at N=1, NVLink at N>1), measured before the timed steps
         res = ctx.autotune(probe_bytes=256 << 20, trials=5)
         nm = {mp.PATH_DIRECT: "direct", mp.PATH_BULK: "bulk"}
-        autotune = {"out": nm[res["out"]], "in": nm[res["in"]], "probe_bytes": 256 << 20, "trials": 5,
-                    "median_ms": res["ms"]}
+        autotune = {"out": nm[res["out"]], "in": nm[res["in"]], "out_small": nm[res["out_small"]],
+                    "in_small": nm[res["in_small"]], "small_below_bytes": mp.AUTO_SMALL_BYTES,
+                    "probe_bytes": 256 << 20, "trials": 5, "median_ms_per_launch": res["ms"]}
 
     seed0 = 2000 + 100 * rank
     src = [[torch.empty(s, dtype=torch.uint8, device="cuda") for s in sizes] for _ in range(mb)]

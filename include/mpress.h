@@ -398,8 +398,9 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
  * on per-peer streams, the measured comparator); 3 = MPRESS_PATH_AUTO
  * (default): per launch, at a full grid (max_ctas 0 or above the SM count)
  * the kernel mpress_autotune measured faster on this context's links for
- * that direction (bulk until then: +0.8% over direct on one B200,
- * profiles/r01), direct when the grid is capped to <= one CTA per SM (its
+ * that direction and size class (until then direct below
+ * MPRESS_AUTO_SMALL_BYTES per launch, bulk above), direct when the grid is
+ * capped to <= one CTA per SM (its
  * 128-thread CTAs co-reside with a GEMM, bulk CTAs' shared memory does not)
  * or when a peer is a host pool.
  * MPRESS_OPT_LAST_PATH (read-only) reports the path the last swap call ran.
@@ -449,9 +450,17 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
 #define MPRESS_OPT_TRANSPORT 5
 #define MPRESS_OPT_LAST_PATH 6   /* read-only: path of the last swap call */
 /* Read-only: the SM path MPRESS_PATH_AUTO takes for an uncapped grid, per
- * direction (MPRESS_PATH_BULK until mpress_autotune measures direct faster). */
+ * direction, for a launch moving >= MPRESS_AUTO_SMALL_BYTES (_OUT / _IN) or
+ * fewer (_OUT_SMALL / _IN_SMALL).  Until mpress_autotune measures otherwise:
+ * bulk for large launches, direct for small ones (one B200, CUDA-graph-
+ * replayed swap pairs, 4 KiB - 4 GiB x 1/3/7 peers: direct 5-25% faster up
+ * to 16 MiB over 3 or 7 peers, the two even at 64 MiB, bulk 3-8% faster from
+ * 256 MiB; profiles/r01/sweep_sizes_v2.jsonl). */
 #define MPRESS_OPT_AUTO_OUT  8
 #define MPRESS_OPT_AUTO_IN   9
+#define MPRESS_OPT_AUTO_OUT_SMALL 10
+#define MPRESS_OPT_AUTO_IN_SMALL  11
+#define MPRESS_AUTO_SMALL_BYTES   33554432u  /* 32 MiB */
 #define MPRESS_TRANSPORT_LOCAL      0
 #define MPRESS_TRANSPORT_VMM_FD     1
 #define MPRESS_TRANSPORT_LEGACY_IPC 2
@@ -466,24 +475,31 @@ MPRESS_API int mpress_set_option(mpress_ctx_t* ctx, int key, int64_t value);
 
 /* Measure, don't guess: which SM kernel MPRESS_PATH_AUTO should run for an
  * uncapped grid on THIS context's links (HBM loopback on one GPU, NVLink /
- * NVSwitch on several -- the two were only ever compared on loopback, +0.8%
- * for bulk).  Moves `probe_bytes` (split equally over the
- * mapped device peers, each share a multiple of 256 and at most that
- * partition's largest free block) out of a library-owned scratch buffer into
- * the stash partitions and back, with the direct kernel (shape 5) and the
- * bulk kernel (shape 3), one warm-up round and then `trials` (1..64) rounds
- * alternating which path goes first; per direction the median times decide,
- * and bulk stays unless direct is at least 1% faster.  The result is read
- * back with MPRESS_OPT_AUTO_OUT / _IN and used by every later AUTO swap of
- * this context with an uncapped grid (a capped grid or a host peer still
- * takes the direct kernel).  Runs synchronously on `stream` (NULL = legacy
- * default stream).
+ * NVSwitch on several -- the kernels were only ever compared on loopback,
+ * DESIGN.md §7), per direction and size class.  Class "large": one launch
+ * each way of `probe_bytes` (split equally over the mapped device peers,
+ * each share a multiple of 256 and at most that partition's largest free
+ * block; use >= MPRESS_AUTO_SMALL_BYTES for a meaningful large-class
+ * decision).  Class "small": 16 launches of 16 MiB (same split) back to back
+ * each way, each on the next 16 MiB window of the probe, so that with
+ * probe_bytes >= 256 MiB the working set exceeds the 126 MB L2 as a
+ * pipeline's stream of fresh tensors does.  Both from a library-owned
+ * scratch buffer into the
+ * stash partitions and back, with the direct kernel (shape 5) and the bulk
+ * kernel (shape 3); one warm-up round then `trials` (1..64) rounds
+ * alternating which kernel goes first; per direction and class the median
+ * times decide, and the class's current choice stays unless the other
+ * kernel is at least 1% faster.  Read the result back with
+ * MPRESS_OPT_AUTO_OUT / _IN / _OUT_SMALL / _IN_SMALL; every later AUTO swap of
+ * this context with an uncapped grid uses it (a capped grid or a host peer
+ * still takes the direct kernel).  Runs synchronously on `stream` (NULL =
+ * legacy default stream).
  * Collective for an mpress_init context: every rank calls it with the same
  * `trials` (a rank without device peers only takes part in the barriers),
  * and each probe starts on all ranks together (barriers through the
  * exchange callback), so the probe sees the all-to-all load of a real swap.
- * ms (may be NULL): [4] = median ms of direct out, direct in, bulk out,
- * bulk in (0 when this rank probed nothing).
+ * ms (may be NULL): [8] = median ms per launch of {small class, large class}
+ * x {direct, bulk} x {out, in} (0 when this rank probed nothing).
  * Errors: MPRESS_ERR_ARG (null ctx, trials out of range, probe_bytes 0),
  * MPRESS_ERR_STATE (a live handle: the probe uses the stash as scratch),
  * MPRESS_ERR_CUDA, MPRESS_ERR_SYS / _PEER (exchange failed, another rank

@@ -25,7 +25,9 @@ DEVICE_HOST = -1   # mpress_init_local: a pinned host pool as a peer (NEXT-4)
 OPT_TRANSPORT = 5  # read-only
 OPT_LAST_PATH = 6  # read-only: path of the last swap call
 OPT_PDL = 7
-OPT_AUTO_OUT, OPT_AUTO_IN = 8, 9   # read-only: AUTO's uncapped-grid path per direction
+OPT_AUTO_OUT, OPT_AUTO_IN = 8, 9   # read-only: AUTO's uncapped-grid path per direction (large launches)
+OPT_AUTO_OUT_SMALL, OPT_AUTO_IN_SMALL = 10, 11   # ... for launches < AUTO_SMALL_BYTES
+AUTO_SMALL_BYTES = 32 << 20
 TRANSPORT_LOCAL, TRANSPORT_VMM_FD, TRANSPORT_LEGACY_IPC = 0, 1, 2
 VARIANT_AUTO = -1
 PATH_DIRECT, PATH_BULK, PATH_CE, PATH_AUTO = 0, 1, 2, 3
@@ -516,10 +518,12 @@ class Context:
         context's links and let MPRESS_PATH_AUTO keep the faster per
         direction (collective for a distributed context).  Returns the
         chosen paths and the median probe times in ms."""
-        ms = (ctypes.c_float * 4)()
+        ms = (ctypes.c_float * 8)()
         _check(lib.mpress_autotune(self._h, probe_bytes, trials, _stream(stream, self.device), ms))
+        names = [c + "_" + k + "_" + d for c in ("small", "large") for k in ("direct", "bulk") for d in ("out", "in")]
         return {"out": self.get_option(OPT_AUTO_OUT), "in": self.get_option(OPT_AUTO_IN),
-                "ms": {"direct_out": ms[0], "direct_in": ms[1], "bulk_out": ms[2], "bulk_in": ms[3]}}
+                "out_small": self.get_option(OPT_AUTO_OUT_SMALL), "in_small": self.get_option(OPT_AUTO_IN_SMALL),
+                "ms": dict(zip(names, ms))}
 
     def stash_free(self):
         out = (c_uint64 * self.world)()

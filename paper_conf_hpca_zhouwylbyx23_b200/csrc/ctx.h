@@ -105,8 +105,10 @@ struct mpress_ctx_s {
   int order = MPRESS_ORDER_INTERLEAVE;
   int pdl = 1;                        // MPRESS_OPT_PDL
   // SM path MPRESS_PATH_AUTO takes for an uncapped grid, per direction
-  // (kDirOut, kDirIn); bulk until mpress_autotune measures otherwise
-  int auto_path[2] = {MPRESS_PATH_BULK, MPRESS_PATH_BULK};
+  // (kDirOut, kDirIn) and size class (a launch moving < MPRESS_AUTO_SMALL_BYTES,
+  // or more); until mpress_autotune measures otherwise: direct for small
+  // launches, bulk for large ones (profiles/r01/sweep_sizes_v2.jsonl)
+  int auto_path[2][2] = {{MPRESS_PATH_DIRECT, MPRESS_PATH_BULK}, {MPRESS_PATH_DIRECT, MPRESS_PATH_BULK}};
   int transport = MPRESS_TRANSPORT_LOCAL;
   int last_launches = 0;
   std::vector<cudaStream_t> ce_streams;  // copy-engine comparator, one per peer

@@ -501,8 +501,10 @@ extern "C" int mpress_get_option(const mpress_ctx_t* c, int key, int64_t* value)
     case MPRESS_OPT_PDL: *value = c->pdl; return MPRESS_OK;
     case MPRESS_OPT_TRANSPORT: *value = c->transport; return MPRESS_OK;
     case MPRESS_OPT_LAST_PATH: *value = c->last_path; return MPRESS_OK;
-    case MPRESS_OPT_AUTO_OUT: *value = c->auto_path[mpress::kDirOut]; return MPRESS_OK;
-    case MPRESS_OPT_AUTO_IN: *value = c->auto_path[mpress::kDirIn]; return MPRESS_OK;
+    case MPRESS_OPT_AUTO_OUT: *value = c->auto_path[mpress::kDirOut][1]; return MPRESS_OK;
+    case MPRESS_OPT_AUTO_IN: *value = c->auto_path[mpress::kDirIn][1]; return MPRESS_OK;
+    case MPRESS_OPT_AUTO_OUT_SMALL: *value = c->auto_path[mpress::kDirOut][0]; return MPRESS_OK;
+    case MPRESS_OPT_AUTO_IN_SMALL: *value = c->auto_path[mpress::kDirIn][0]; return MPRESS_OK;
   }
   return fail(MPRESS_ERR_ARG, "unknown option %d", key);
 }

@@ -144,15 +144,18 @@ int run_copy(mpress_ctx_s* c, int dir, const std::vector<CopyDesc>& d,
   c->last_launches = 0;
   int path = c->path;
   if (path == MPRESS_PATH_AUTO) {
-    // full grid: bulk (TMA, +0.8% over direct on B200 loopback, profiles/r01)
-    // unless mpress_autotune measured direct faster on this context's links;
+    // full grid: per direction and size class, the kernel mpress_autotune
+    // measured faster on this context's links (before it runs: direct below
+    // MPRESS_AUTO_SMALL_BYTES, bulk above -- TMA, +0.8% on B200 loopback);
     // direct when the grid is capped to <= one CTA per SM (small CTAs that
     // co-reside with a GEMM) or a peer is pinned host memory
     int dev = 0, sms = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     const bool capped = c->max_ctas > 0 && c->max_ctas <= sms;
-    path = (capped || c->host_peer) ? MPRESS_PATH_DIRECT : c->auto_path[dir];
+    uint64_t total = 0;
+    for (const CopyDesc& x : d) total += x.len;
+    path = (capped || c->host_peer) ? MPRESS_PATH_DIRECT : c->auto_path[dir][total >= MPRESS_AUTO_SMALL_BYTES];
   }
   c->last_path = path;
   if (path != MPRESS_PATH_CE)
@@ -498,9 +501,10 @@ float median(std::vector<float> v) {
 }  // namespace mpress
 
 // Runtime choice of the SM path MPRESS_PATH_AUTO takes for an uncapped grid:
-// time both SM kernels on this context's own peers and keep the faster per
-// direction (include/mpress.h).  The stash partitions serve as the probe's
-// scratch, so no handle may be live.
+// time both SM kernels on this context's own peers, for a small and a large
+// launch, and keep the faster per direction and size class
+// (include/mpress.h).  The stash partitions serve as the probe's scratch, so
+// no handle may be live.
 extern "C" int mpress_autotune(mpress_ctx_t* c, uint64_t probe_bytes, int trials, void* stream_, float* ms_out) {
   if (!c || trials < 1 || trials > 64 || probe_bytes == 0)
     return fail(MPRESS_ERR_ARG, "mpress_autotune: bad argument");
@@ -536,41 +540,62 @@ extern "C" int mpress_autotune(mpress_ctx_t* c, uint64_t probe_bytes, int trials
     for (int i = 0; i < 3 && e == cudaSuccess; ++i) e = cudaEventCreate(&ev[i]);
     if (e != cudaSuccess) rc = cuda_fail(e, "mpress_autotune: probe buffers");
   }
-  std::vector<CopyDesc> dout, din;
+  // Two probes per path.  Class 1 ("large"): the whole probe, one launch
+  // each way.  Class 0 ("small"): launches of kSmallProbe (split over the
+  // peers), kSmallReps back to back each way, each on the next window of the
+  // probe buffers, so the working set (the whole probe) exceeds L2 as a
+  // pipeline's stream of fresh tensors does -- repeating one 16 MiB window
+  // would time L2, not HBM / NVLink.
+  constexpr uint64_t kSmallProbe = 16ull << 20;
+  constexpr int kSmallReps = 16;
+  std::vector<CopyDesc> dout[2][kSmallReps], din[2][kSmallReps];
   std::vector<int> grp;
   uint64_t at = 0;
+  const uint64_t small_share =
+      peers.empty() ? 0 : std::max<uint64_t>(MPRESS_ALIGN, kSmallProbe / peers.size() / MPRESS_ALIGN * MPRESS_ALIGN);
   for (int p : peers) {
     if (!len[p]) continue;
-    dout.push_back({src + at, c->parts[p].base + off[p], len[p]});
-    din.push_back({c->parts[p].base + off[p], dst + at, len[p]});
     grp.push_back(p);
+    dout[1][0].push_back({src + at, c->parts[p].base + off[p], len[p]});
+    din[1][0].push_back({c->parts[p].base + off[p], dst + at, len[p]});
+    const uint64_t n = std::min(len[p], small_share);
+    const uint64_t windows = std::max<uint64_t>(1, len[p] / n);
+    for (int w = 0; w < kSmallReps; ++w) {
+      const uint64_t o = (w % windows) * n;
+      dout[0][w].push_back({src + at + o, c->parts[p].base + off[p] + o, n});
+      din[0][w].push_back({c->parts[p].base + off[p] + o, dst + at + o, n});
+    }
     at += len[p];
   }
   // warm-up round (-1), then `trials` rounds alternating which path goes first
   const int paths[2] = {MPRESS_PATH_DIRECT, MPRESS_PATH_BULK};
-  std::vector<float> t[2][2];  // [path][dir]
+  std::vector<float> t[2][2][2];  // [class][path][dir], ms per launch
   for (int r = -1; r < trials; ++r) {
-    for (int k = 0; k < 2; ++k) {
-      const int pi = (r & 1) ? 1 - k : k;
-      rc = autotune_barrier(c, rc);
-      if (rc != MPRESS_OK || dout.empty()) continue;
-      int launches = 0;
-      cudaEventRecord(ev[0], stream);
-      rc = launch_copy(paths[pi], MPRESS_VARIANT_AUTO, kDirOut, dout.data(), grp.data(), dout.size(), 0, c->pdl,
-                       stream, &launches);
-      cudaEventRecord(ev[1], stream);
-      if (rc == MPRESS_OK)
-        rc = launch_copy(paths[pi], MPRESS_VARIANT_AUTO, kDirIn, din.data(), grp.data(), din.size(), 0, c->pdl,
-                         stream, &launches);
-      cudaEventRecord(ev[2], stream);
-      cudaError_t e = cudaEventSynchronize(ev[2]);
-      float a = 0, b = 0;
-      if (e == cudaSuccess) e = cudaEventElapsedTime(&a, ev[0], ev[1]);
-      if (e == cudaSuccess) e = cudaEventElapsedTime(&b, ev[1], ev[2]);
-      if (e != cudaSuccess && rc == MPRESS_OK) rc = cuda_fail(e, "mpress_autotune: probe timing");
-      if (r >= 0) {
-        t[pi][kDirOut].push_back(a);
-        t[pi][kDirIn].push_back(b);
+    for (int cls = 0; cls < 2; ++cls) {
+      const int reps = cls ? 1 : kSmallReps;
+      for (int k = 0; k < 2; ++k) {
+        const int pi = (r & 1) ? 1 - k : k;
+        rc = autotune_barrier(c, rc);
+        if (rc != MPRESS_OK || grp.empty()) continue;
+        int launches = 0;
+        cudaEventRecord(ev[0], stream);
+        for (int i = 0; i < reps && rc == MPRESS_OK; ++i)
+          rc = launch_copy(paths[pi], MPRESS_VARIANT_AUTO, kDirOut, dout[cls][i].data(), grp.data(),
+                           dout[cls][i].size(), 0, c->pdl, stream, &launches);
+        cudaEventRecord(ev[1], stream);
+        for (int i = 0; i < reps && rc == MPRESS_OK; ++i)
+          rc = launch_copy(paths[pi], MPRESS_VARIANT_AUTO, kDirIn, din[cls][i].data(), grp.data(),
+                           din[cls][i].size(), 0, c->pdl, stream, &launches);
+        cudaEventRecord(ev[2], stream);
+        cudaError_t e = cudaEventSynchronize(ev[2]);
+        float a = 0, b = 0;
+        if (e == cudaSuccess) e = cudaEventElapsedTime(&a, ev[0], ev[1]);
+        if (e == cudaSuccess) e = cudaEventElapsedTime(&b, ev[1], ev[2]);
+        if (e != cudaSuccess && rc == MPRESS_OK) rc = cuda_fail(e, "mpress_autotune: probe timing");
+        if (r >= 0) {
+          t[cls][pi][kDirOut].push_back(a / reps);
+          t[cls][pi][kDirIn].push_back(b / reps);
+        }
       }
     }
   }
@@ -581,17 +606,20 @@ extern "C" int mpress_autotune(mpress_ctx_t* c, uint64_t probe_bytes, int trials
   cudaFree(dst);
   for (auto e : ev) if (e) cudaEventDestroy(e);
   if (rc != MPRESS_OK) return rc;
-  float m[2][2];
-  for (int pi = 0; pi < 2; ++pi)
-    for (int d = 0; d < 2; ++d) m[pi][d] = median(t[pi][d]);
-  if (!dout.empty())
-    for (int d = 0; d < 2; ++d)  // bulk stays unless direct is >= 1% faster
-      c->auto_path[d] = m[0][d] < 0.99f * m[1][d] ? MPRESS_PATH_DIRECT : MPRESS_PATH_BULK;
-  if (ms_out) {
-    ms_out[0] = m[0][kDirOut];
-    ms_out[1] = m[0][kDirIn];
-    ms_out[2] = m[1][kDirOut];
-    ms_out[3] = m[1][kDirIn];
+  for (int cls = 0; cls < 2; ++cls) {
+    float m[2][2];
+    for (int pi = 0; pi < 2; ++pi)
+      for (int d = 0; d < 2; ++d) m[pi][d] = median(t[cls][pi][d]);
+    if (!grp.empty())
+      for (int d = 0; d < 2; ++d) {  // the class default stays unless the other kernel is >= 1% faster
+        const int def = c->auto_path[d][cls];
+        const int other = def == MPRESS_PATH_DIRECT ? MPRESS_PATH_BULK : MPRESS_PATH_DIRECT;
+        const float t_def = m[def == MPRESS_PATH_BULK][d], t_other = m[other == MPRESS_PATH_BULK][d];
+        c->auto_path[d][cls] = t_other < 0.99f * t_def ? other : def;
+      }
+    if (ms_out)
+      for (int pi = 0; pi < 2; ++pi)
+        for (int d = 0; d < 2; ++d) ms_out[cls * 4 + pi * 2 + d] = m[pi][d];
   }
   return MPRESS_OK;
 }

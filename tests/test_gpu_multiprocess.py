@@ -129,6 +129,7 @@ def _cfg5_worker(rank, world, port, outdir):
         if rank in peers:
             assert all(v == 0 for v in res["ms"].values()), res
             assert res["out"] == res["in"] == mp.PATH_BULK
+            assert res["out_small"] == res["in_small"] == mp.PATH_DIRECT
         else:
             assert all(v > 0 for v in res["ms"].values()), res
         if rank in sources and not err:

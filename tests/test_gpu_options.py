@@ -42,9 +42,10 @@ def test_options_and_stash_free():
 
 
 def test_auto_path_resolution():
-    """MPRESS_PATH_AUTO: bulk (TMA) at a full grid, direct when the grid is
-    capped to <= one CTA per SM; variants cannot be forced under AUTO; every
-    resolution round-trips bit-exactly."""
+    """MPRESS_PATH_AUTO: at a full grid the size class's kernel (direct for a
+    small launch before any autotune), direct when the grid is capped to <=
+    one CTA per SM; variants cannot be forced under AUTO; every resolution
+    round-trips bit-exactly."""
     from synth import device as synth_dev
     world = 3
     sizes = [(3 << 20) + 5, 4096]
@@ -60,7 +61,11 @@ def test_auto_path_resolution():
         for i, t in enumerate(src):
             synth_dev.fill(t, 4, i)
         sms = torch.cuda.get_device_properties(0).multi_processor_count
-        for cap, want in ((0, mp.PATH_BULK), (sms + 1, mp.PATH_BULK), (sms, mp.PATH_DIRECT), (16, mp.PATH_DIRECT)):
+        # a ~3 MiB launch is in the small class: direct before any autotune
+        assert sum(sizes) < mp.AUTO_SMALL_BYTES
+        small = ctx.get_option(mp.OPT_AUTO_OUT_SMALL)
+        assert small == ctx.get_option(mp.OPT_AUTO_IN_SMALL) == mp.PATH_DIRECT
+        for cap, want in ((0, small), (sms + 1, small), (sms, mp.PATH_DIRECT), (16, mp.PATH_DIRECT)):
             ctx.set_option(mp.OPT_MAX_CTAS, cap)
             dst = [torch.zeros(n, dtype=torch.uint8, device="cuda") for n in sizes]
             h = ctx.swap_out(pl, src)
@@ -124,17 +129,22 @@ def test_pdl_modes():
 
 def test_autotune_local():
     """mpress_autotune on a loopback context: both kernels timed per
-    direction, the choice is one of them, later AUTO swaps with an uncapped
-    grid run the chosen path per direction (capped ones stay direct), and
-    everything round-trips bit-exactly.  A live handle refuses the probe."""
+    direction and size class, each choice is one of them, later AUTO swaps
+    with an uncapped grid run the chosen kernel for their direction and size
+    class (capped ones stay direct), and everything round-trips bit-exactly.
+    A live handle refuses the probe."""
     from synth import device as synth_dev
     world = 4
-    sizes = [(7 << 20) + 3, 1 << 20, 33]
-    pl = mp.plan(world, 0, [0] + [1 << 30] * 3, [0, 1, 1, 1], sizes)
-    part = [[0] + [2 * u * 65536 for u in pl.units[1:]]] + [[0] * world for _ in range(3)]
+    small = [(7 << 20) + 3, 1 << 20, 33]          # < AUTO_SMALL_BYTES per launch
+    large = [48 << 20, 5]                          # >= AUTO_SMALL_BYTES
+    assert sum(small) < mp.AUTO_SMALL_BYTES <= sum(large)
+    spare, bw = [0] + [1 << 30] * 3, [0, 1, 1, 1]
+    pls = {"small": mp.plan(world, 0, spare, bw, small), "large": mp.plan(world, 0, spare, bw, large)}
+    part = [[0] + [2 * u * 65536 for u in pls["large"].units[1:]]] + [[0] * world for _ in range(3)]
     ctx = mp.Context.local(world, 0, [0] * world, part)
     try:
         assert ctx.get_option(mp.OPT_AUTO_OUT) == ctx.get_option(mp.OPT_AUTO_IN) == mp.PATH_BULK
+        assert ctx.get_option(mp.OPT_AUTO_OUT_SMALL) == ctx.get_option(mp.OPT_AUTO_IN_SMALL) == mp.PATH_DIRECT
         for bad in ((0, 3), (1 << 20, 0), (1 << 20, 65)):
             with pytest.raises(mp.MPressError) as ei:
                 ctx.autotune(probe_bytes=bad[0], trials=bad[1])
@@ -142,25 +152,29 @@ def test_autotune_local():
         free0 = ctx.stash_free()
         res = ctx.autotune(probe_bytes=64 << 20, trials=3)
         assert ctx.stash_free() == free0   # the probe's slices went back
-        assert res["out"] in (mp.PATH_DIRECT, mp.PATH_BULK) and res["in"] in (mp.PATH_DIRECT, mp.PATH_BULK)
-        assert all(v > 0 for v in res["ms"].values()), res
-        src = [torch.empty(n, dtype=torch.uint8, device="cuda") for n in sizes]
-        for i, t in enumerate(src):
-            synth_dev.fill(t, 61, i)
-        torch.cuda.synchronize()
-        for cap in (0, 16):
-            ctx.set_option(mp.OPT_MAX_CTAS, cap)
-            dst = [torch.zeros(n, dtype=torch.uint8, device="cuda") for n in sizes]
-            h = ctx.swap_out(pl, src)
-            assert ctx.get_option(mp.OPT_LAST_PATH) == (res["out"] if cap == 0 else mp.PATH_DIRECT)
-            if cap == 0:
-                with pytest.raises(mp.MPressError) as ei:
-                    ctx.autotune()
-                assert ei.value.code == mp.ERR_STATE
-            ctx.swap_in(h, dst)
-            assert ctx.get_option(mp.OPT_LAST_PATH) == (res["in"] if cap == 0 else mp.PATH_DIRECT)
+        for k in ("out", "in", "out_small", "in_small"):
+            assert res[k] in (mp.PATH_DIRECT, mp.PATH_BULK), res
+        assert len(res["ms"]) == 8 and all(v > 0 for v in res["ms"].values()), res
+        for cls, sizes in (("small", small), ("large", large)):
+            pl = pls[cls]
+            src = [torch.empty(n, dtype=torch.uint8, device="cuda") for n in sizes]
+            for i, t in enumerate(src):
+                synth_dev.fill(t, 61, i)
             torch.cuda.synchronize()
-            assert all(synth_dev.check(d, 61, i) == 0 for i, d in enumerate(dst)), cap
-            h.free()
+            suffix = "" if cls == "large" else "_small"
+            for cap in (0, 16):
+                ctx.set_option(mp.OPT_MAX_CTAS, cap)
+                dst = [torch.zeros(n, dtype=torch.uint8, device="cuda") for n in sizes]
+                h = ctx.swap_out(pl, src)
+                assert ctx.get_option(mp.OPT_LAST_PATH) == (res["out" + suffix] if cap == 0 else mp.PATH_DIRECT)
+                if cap == 0:
+                    with pytest.raises(mp.MPressError) as ei:
+                        ctx.autotune()
+                    assert ei.value.code == mp.ERR_STATE
+                ctx.swap_in(h, dst)
+                assert ctx.get_option(mp.OPT_LAST_PATH) == (res["in" + suffix] if cap == 0 else mp.PATH_DIRECT)
+                torch.cuda.synchronize()
+                assert all(synth_dev.check(d, 61, i) == 0 for i, d in enumerate(dst)), (cls, cap)
+                h.free()
     finally:
         ctx.finalize()
