@@ -112,6 +112,7 @@ struct mpress_ctx_s {
   int transport = MPRESS_TRANSPORT_LOCAL;
   int last_launches = 0;
   std::vector<cudaStream_t> ce_streams;  // copy-engine comparator, one per peer
+  mpress::TableRing* ring = nullptr;  // device-resident tables of large launches (lazy)
   mpress::EvPool ev_pool = std::make_shared<std::vector<cudaEvent_t>>();
   std::set<mpress_handle_s*> handles;
   std::vector<mpress::CopyDesc> scratch_desc;  // per-call buffers, reused

@@ -144,6 +144,7 @@ void destroy(mpress_ctx_s* c) {
   for (auto e : *c->ev_pool) cudaEventDestroy(e);
   c->ev_pool->clear();
   for (auto s : c->ce_streams) if (s) cudaStreamDestroy(s);
+  table_ring_destroy(c->ring);
   delete c;
 }
 

@@ -20,6 +20,7 @@
 #include <cstring>
 
 #include "ctx.h"
+#include "hostprof.h"
 #include "swap_kernels.h"
 
 namespace mpress {
@@ -140,7 +141,7 @@ int record_done(mpress_ctx_s* c, cudaStream_t s, bool graph, EvRef* ev, EvRef* e
 
 // Move every descriptor on `stream` with the context's path.
 int run_copy(mpress_ctx_s* c, int dir, const std::vector<CopyDesc>& d,
-             const std::vector<int>& desc_peer, cudaStream_t stream) {
+             const std::vector<int>& desc_peer, cudaStream_t stream, bool graph) {
   c->last_launches = 0;
   int path = c->path;
   if (path == MPRESS_PATH_AUTO) {
@@ -158,10 +159,14 @@ int run_copy(mpress_ctx_s* c, int dir, const std::vector<CopyDesc>& d,
     path = (capped || c->host_peer) ? MPRESS_PATH_DIRECT : c->auto_path[dir][total >= MPRESS_AUTO_SMALL_BYTES];
   }
   c->last_path = path;
-  if (path != MPRESS_PATH_CE)
+  if (path != MPRESS_PATH_CE) {
+    // Large tables live in device memory (TableRing), except under graph
+    // capture: a replay would re-read a staging slot later launches reused.
+    if (!graph && d.size() > (size_t)kParamDescMax && !c->ring) MP_TRY(table_ring_create(c->device, &c->ring));
     return launch_copy(path, c->variant, dir, d.data(),
                        c->order == MPRESS_ORDER_INTERLEAVE ? desc_peer.data() : nullptr, d.size(), c->max_ctas,
-                       c->pdl, stream, &c->last_launches);
+                       c->pdl, stream, &c->last_launches, graph ? nullptr : c->ring);
+  }
 
   // Copy-engine comparator, variant 1: the whole swap as one
   // cudaMemcpyBatchAsync on `stream` (CUDA 12.8+); the driver spreads the
@@ -243,6 +248,7 @@ using namespace mpress;
 extern "C" int mpress_swap_out(mpress_ctx_t* c, const mpress_plan_t* plan_, void* const* tensors,
                                void* stream_, void* after, mpress_handle_t** out) {
   if (!c || !plan_ || !out) return fail(MPRESS_ERR_ARG, "mpress_swap_out: null argument");
+  HP_START();
   *out = nullptr;
   std::lock_guard<std::mutex> lk(c->mu);
   const uint64_t *units, *peer_bytes;
@@ -259,6 +265,7 @@ extern "C" int mpress_swap_out(mpress_ctx_t* c, const mpress_plan_t* plan_, void
   DeviceGuard g(c->device);
   cudaStream_t stream = static_cast<cudaStream_t>(stream_);
   const bool graph = capturing(stream);
+  HP_LAP(0, "out: plan/ptrs/capture query");
 
   auto* h = new mpress_handle_s();
   h->ctx = c;
@@ -297,6 +304,7 @@ extern "C" int mpress_swap_out(mpress_ctx_t* c, const mpress_plan_t* plan_, void
     delete h;
     return rc;
   }
+  HP_LAP(1, "out: handle + slices + fences");
   h->slices_held = true;
   h->stripes.assign(st, st + n_st);
   h->n_tensors = info.n_tensors;
@@ -313,8 +321,11 @@ extern "C" int mpress_swap_out(mpress_ctx_t* c, const mpress_plan_t* plan_, void
     dp[i] = (int)s.peer;
   }
   if (after) cudaStreamWaitEvent(stream, static_cast<cudaEvent_t>(after), 0);
-  rc = run_copy(c, kDirOut, d, dp, stream);
+  HP_LAP(2, "out: descriptors");
+  rc = run_copy(c, kDirOut, d, dp, stream, graph);
+  HP_LAP(3, "out: run_copy (launch)");
   if (rc == MPRESS_OK) rc = record_done(c, stream, graph, &h->out_done, &h->out_ext, "cudaEventRecord(out_done)");
+  HP_LAP(4, "out: event record");
   if (rc != MPRESS_OK) {
     // Kernels may already be queued: keep the slices fenced by a sync (a
     // failed capture is invalidated anyway: nothing was enqueued for real).
@@ -333,6 +344,7 @@ extern "C" int mpress_swap_out(mpress_ctx_t* c, const mpress_plan_t* plan_, void
 
 extern "C" int mpress_swap_in(mpress_ctx_t* c, mpress_handle_t* h, void* const* dst, void* stream_) {
   if (!c || !h) return fail(MPRESS_ERR_ARG, "mpress_swap_in: null argument");
+  HP_START();
   std::lock_guard<std::mutex> lk(c->mu);
   if (h->ctx != c || !c->handles.count(h)) return fail(MPRESS_ERR_ARG, "mpress_swap_in: handle not of this context");
   if (h->state != MPRESS_STATE_OUT_PENDING && h->state != MPRESS_STATE_OUT)
@@ -360,10 +372,13 @@ extern "C" int mpress_swap_in(mpress_ctx_t* c, mpress_handle_t* h, void* const* 
     dp[i] = (int)s.peer;
   }
   if (h->graph || !same_stream(h->out_stream, stream)) cudaStreamWaitEvent(stream, h->out_done.get(), 0);
-  int rc = run_copy(c, kDirIn, d, dp, stream);
+  HP_LAP(5, "in: checks + capture query + desc");
+  int rc = run_copy(c, kDirIn, d, dp, stream, h->graph);
+  HP_LAP(6, "in: run_copy (launch)");
   if (rc != MPRESS_OK) return rc;
   EvRef in_done, in_ext;
   MP_TRY(record_done(c, stream, h->graph, &in_done, &in_ext, "cudaEventRecord(in_done)"));
+  HP_LAP(7, "in: event record");
   h->in_done = in_done;
   h->in_ext = in_ext;
   h->state = MPRESS_STATE_IN_PENDING;
@@ -387,6 +402,7 @@ extern "C" int mpress_swap_in(mpress_ctx_t* c, mpress_handle_t* h, void* const* 
     free_slice(&c->parts[p], h->slice_off[p], h->slice_len[p]);
   }
   h->slices_held = false;
+  HP_LAP(8, "in: fences + slice release");
   return MPRESS_OK;
 }
 
@@ -445,6 +461,7 @@ extern "C" int mpress_handle_slices(const mpress_handle_t* h, uint64_t* slice_of
 
 extern "C" int mpress_handle_free(mpress_ctx_t* c, mpress_handle_t* h, int force) {
   if (!c || !h) return fail(MPRESS_ERR_ARG, "mpress_handle_free: null argument");
+  HP_START();
   std::lock_guard<std::mutex> lk(c->mu);
   if (h->ctx != c || !c->handles.count(h)) return fail(MPRESS_ERR_ARG, "mpress_handle_free: handle not of this context");
   DeviceGuard g(c->device);
@@ -472,6 +489,7 @@ extern "C" int mpress_handle_free(mpress_ctx_t* c, mpress_handle_t* h, int force
   // An IN_PENDING handle's slices stay fenced: the fences share its event.
   c->handles.erase(h);
   delete h;
+  HP_LAP(9, "handle_free");
   return MPRESS_OK;
 }
 

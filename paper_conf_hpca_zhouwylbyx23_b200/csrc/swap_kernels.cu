@@ -36,12 +36,15 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstddef>
+#include <type_traits>
 #include <mutex>
 #include <set>
 #include <utility>
 #include <vector>
 
 #include "common.h"
+#include "hostprof.h"
 #include "swap_kernels.h"
 
 namespace mpress {
@@ -49,8 +52,11 @@ namespace {
 
 constexpr int kMaxGroups = 64;  // peers per launch (NVSwitch domains up to 64 GPUs)
 
-// Descriptor tables come in three capacities so a small swap does not ship a
-// 28 KB parameter block with its launch (launch latency grows with it).
+// Descriptor tables come in five capacities (16, 32, 64, 128, 1024) so a
+// small swap does not ship a 28 KB parameter block with its launch: the
+// host cost of cudaLaunchKernelEx grows ~0.75 us per KB of parameters
+// (16 -> 17 stripes, i.e. a 0.6 KB -> 4.1 KB table: +2.65 us per launch,
+// tools/hostcost.py).
 template <int CAP>
 struct CopyTable {
   // every group holds >= 1 descriptor, so a table needs <= CAP groups
@@ -202,8 +208,7 @@ __device__ __forceinline__ Span span_of(const CopyTable<CAP>& t, uint32_t c, uin
 // DIR only names the instantiation (swap-out vs swap-in in profiles): the
 // byte movement is the same, the descriptors say which side is the peer.
 template <int DIR, int THREADS, int UNROLL, int VB, bool HINT, bool PF, int CAP>
-__global__ void __launch_bounds__(THREADS)
-mp_swap_direct(const __grid_constant__ CopyTable<CAP> t) {
+__device__ __forceinline__ void direct_body(const CopyTable<CAP>& t) {
   using VT = typename Vec<VB, HINT>::T;
   constexpr uint32_t kChunk = THREADS * UNROLL * VB;
   static_assert((kChunk & (kChunk - 1)) == 0, "chunk must be a power of two");
@@ -252,6 +257,20 @@ mp_swap_direct(const __grid_constant__ CopyTable<CAP> t) {
     if (!more) break;
     sp = nx;
   }
+}
+
+// The table as a kernel parameter (constant bank) ...
+template <int DIR, int THREADS, int UNROLL, int VB, bool HINT, bool PF, int CAP>
+__global__ void __launch_bounds__(THREADS)
+mp_swap_direct(const __grid_constant__ CopyTable<CAP> t) {
+  direct_body<DIR, THREADS, UNROLL, VB, HINT, PF, CAP>(t);
+}
+
+// ... or device-resident (TableRing, large tables), read through a pointer.
+template <int DIR, int THREADS, int UNROLL, int VB, bool HINT, bool PF, int CAP>
+__global__ void __launch_bounds__(THREADS)
+mp_swap_direct_g(const CopyTable<CAP>* __restrict__ tp) {
+  direct_body<DIR, THREADS, UNROLL, VB, HINT, PF, CAP>(*tp);
 }
 
 // ---------------------------------------------------------------- bulk path
@@ -342,8 +361,7 @@ __device__ __forceinline__ uint64_t shfl64(uint64_t v, int lane) {
 // out of its slot, keeping one store in flight behind the newest
 // (wait_group.read 1).
 template <int DIR, int SHIFT, int STAGES, int CAP>
-__global__ void __launch_bounds__(32)
-mp_swap_bulk(const __grid_constant__ CopyTable<CAP> t) {
+__device__ __forceinline__ void bulk_body(const CopyTable<CAP>& t) {
   constexpr uint32_t kSlot = 1u << SHIFT;
   extern __shared__ __align__(128) uint8_t smem[];
   __shared__ __align__(8) uint64_t bars[STAGES];
@@ -416,6 +434,18 @@ mp_swap_bulk(const __grid_constant__ CopyTable<CAP> t) {
   }
 }
 
+template <int DIR, int SHIFT, int STAGES, int CAP>
+__global__ void __launch_bounds__(32)
+mp_swap_bulk(const __grid_constant__ CopyTable<CAP> t) {
+  bulk_body<DIR, SHIFT, STAGES, CAP>(t);
+}
+
+template <int DIR, int SHIFT, int STAGES, int CAP>
+__global__ void __launch_bounds__(32)
+mp_swap_bulk_g(const CopyTable<CAP>* __restrict__ tp) {
+  bulk_body<DIR, SHIFT, STAGES, CAP>(*tp);
+}
+
 // ---------------------------------------------------------------- variants
 
 struct Shape {
@@ -444,37 +474,60 @@ constexpr Shape kBulk[kBulkVariants] = {
 
 template <int CAP>
 using KernelFn = void (*)(CopyTable<CAP>);
-
 template <int CAP>
-KernelFn<CAP> kernel_for(int path, int variant, int dir, bool pf) {
+using KernelFnG = void (*)(const CopyTable<CAP>*);
+
+// Entry point of one instantiation; `if constexpr` keeps the pointer-table
+// (G) kernels from being instantiated for the capacities that never use them.
+template <int CAP, bool G, int D, int SH, int ST>
+void* bulk_ptr() {
+  if constexpr (G) return reinterpret_cast<void*>(mp_swap_bulk_g<D, SH, ST, CAP>);
+  else return reinterpret_cast<void*>(mp_swap_bulk<D, SH, ST, CAP>);
+}
+template <int CAP, bool G, int D, int T, int U, int VB, bool H, bool PF>
+void* direct_ptr() {
+  if constexpr (G) return reinterpret_cast<void*>(mp_swap_direct_g<D, T, U, VB, H, PF, CAP>);
+  else return reinterpret_cast<void*>(mp_swap_direct<D, T, U, VB, H, PF, CAP>);
+}
+
+// G = false: the table is a __grid_constant__ parameter; G = true: a pointer
+// to a device-resident table (TableRing).
+template <int CAP, bool G>
+std::conditional_t<G, KernelFnG<CAP>, KernelFn<CAP>> kernel_for(int path, int variant, int dir, bool pf) {
   const bool o = dir == kDirOut;
+#define MP_BULK(SH, ST) (o ? bulk_ptr<CAP, G, kDirOut, SH, ST>() : bulk_ptr<CAP, G, kDirIn, SH, ST>())
+#define MP_DIRECT1(D, T, U, VB, H) \
+  (pf ? direct_ptr<CAP, G, D, T, U, VB, H, true>() : direct_ptr<CAP, G, D, T, U, VB, H, false>())
+#define MP_DIRECT(T, U, VB, H) (o ? MP_DIRECT1(kDirOut, T, U, VB, H) : MP_DIRECT1(kDirIn, T, U, VB, H))
+  void* k;
   if (path == MPRESS_PATH_BULK) {
     switch (variant) {
-      case 1: return o ? mp_swap_bulk<kDirOut, 14, 12, CAP> : mp_swap_bulk<kDirIn, 14, 12, CAP>;
-      case 2: return o ? mp_swap_bulk<kDirOut, 16, 3, CAP> : mp_swap_bulk<kDirIn, 16, 3, CAP>;
-      case 3: return o ? mp_swap_bulk<kDirOut, 15, 3, CAP> : mp_swap_bulk<kDirIn, 15, 3, CAP>;
-      case 4: return o ? mp_swap_bulk<kDirOut, 14, 4, CAP> : mp_swap_bulk<kDirIn, 14, 4, CAP>;
-      case 5: return o ? mp_swap_bulk<kDirOut, 13, 2, CAP> : mp_swap_bulk<kDirIn, 13, 2, CAP>;
-      case 6: return o ? mp_swap_bulk<kDirOut, 12, 3, CAP> : mp_swap_bulk<kDirIn, 12, 3, CAP>;
-      default: return o ? mp_swap_bulk<kDirOut, 15, 6, CAP> : mp_swap_bulk<kDirIn, 15, 6, CAP>;
+      case 1: k = MP_BULK(14, 12); break;
+      case 2: k = MP_BULK(16, 3); break;
+      case 3: k = MP_BULK(15, 3); break;
+      case 4: k = MP_BULK(14, 4); break;
+      case 5: k = MP_BULK(13, 2); break;
+      case 6: k = MP_BULK(12, 3); break;
+      default: k = MP_BULK(15, 6); break;
+    }
+  } else {
+    switch (variant) {
+      case 1: k = MP_DIRECT(512, 8, 16, false); break;
+      case 2: k = MP_DIRECT(256, 16, 16, false); break;
+      case 3: k = MP_DIRECT(1024, 4, 16, false); break;
+      case 4: k = MP_DIRECT(128, 8, 16, false); break;
+      case 5: k = MP_DIRECT(256, 4, 32, false); break;
+      case 6: k = MP_DIRECT(256, 8, 32, false); break;
+      case 7: k = MP_DIRECT(128, 4, 32, false); break;
+      case 8: k = MP_DIRECT(256, 4, 32, true); break;
+      case 9: k = MP_DIRECT(128, 8, 32, false); break;
+      default: k = MP_DIRECT(256, 8, 16, false); break;
     }
   }
-#define MP_DIRECT(T, U, VB, H)                                                                        \
-  (o ? (pf ? mp_swap_direct<kDirOut, T, U, VB, H, true, CAP> : mp_swap_direct<kDirOut, T, U, VB, H, false, CAP>) \
-     : (pf ? mp_swap_direct<kDirIn, T, U, VB, H, true, CAP> : mp_swap_direct<kDirIn, T, U, VB, H, false, CAP>))
-  switch (variant) {
-    case 1: return MP_DIRECT(512, 8, 16, false);
-    case 2: return MP_DIRECT(256, 16, 16, false);
-    case 3: return MP_DIRECT(1024, 4, 16, false);
-    case 4: return MP_DIRECT(128, 8, 16, false);
-    case 5: return MP_DIRECT(256, 4, 32, false);
-    case 6: return MP_DIRECT(256, 8, 32, false);
-    case 7: return MP_DIRECT(128, 4, 32, false);
-    case 8: return MP_DIRECT(256, 4, 32, true);
-    case 9: return MP_DIRECT(128, 8, 32, false);
-    default: return MP_DIRECT(256, 8, 16, false);
-  }
 #undef MP_DIRECT
+#undef MP_DIRECT1
+#undef MP_BULK
+  return reinterpret_cast<std::conditional_t<G, KernelFnG<CAP>, KernelFn<CAP>>>(k);
 }
 
 const Shape& shape_of(int path, int variant) {
@@ -489,8 +542,8 @@ struct DevCache {
 DevCache g_cache;
 
 // Opt a kernel into > 48 KB of dynamic shared memory, once per device.
-template <int CAP>
-int prepare(KernelFn<CAP> k, const Shape& sh) {
+template <typename K>
+int prepare(K k, const Shape& sh) {
   if (sh.smem <= 48 * 1024) return MPRESS_OK;
   static std::mutex mu;
   static std::set<std::pair<int, const void*>> done;
@@ -504,12 +557,11 @@ int prepare(KernelFn<CAP> k, const Shape& sh) {
   return MPRESS_OK;
 }
 
-// Build the table for descriptors d[0..n) (group ids gid[]), split `cap`
-// CTAs between the groups in proportion to their chunks, launch.
+// Fill the table for descriptors d[0..n) (group ids gid[]); *chunks = the
+// launch's chunk count (0: nothing to move).
 template <int CAP>
-int launch_batch(int path, int variant, int dir, const CopyDesc* d, const int* gid, uint32_t n,
-                 uint32_t shift, int cap, int sms, bool pdl, cudaStream_t stream, bool* launched) {
-  CopyTable<CAP> t;
+int build_table(CopyTable<CAP>& t, const CopyDesc* d, const int* gid, uint32_t n, uint32_t shift,
+                uint64_t* chunks_out) {
   t.n = n;
   t.pad = 0;
   uint64_t chunks = 0;
@@ -529,16 +581,17 @@ int launch_batch(int path, int variant, int dir, const CopyDesc* d, const int* g
   t.g_chunk[ng] = (uint32_t)chunks;
   t.g_desc[ng] = n;
   t.n_groups = ng;
-  *launched = false;
-  if (chunks == 0) return MPRESS_OK;
   uint32_t largest = 0;
   for (uint32_t g = 0; g < ng; ++g) largest = std::max(largest, t.g_chunk[g + 1] - t.g_chunk[g]);
   t.rounds_log2 = 0;
   while ((1ull << t.rounds_log2) < largest) ++t.rounds_log2;
-  const unsigned grid = (unsigned)std::min<uint64_t>(chunks, (uint64_t)cap);
-  const Shape& sh = shape_of(path, variant);
-  KernelFn<CAP> k = kernel_for<CAP>(path, variant, dir, (int)grid <= sms);
-  MP_TRY(prepare<CAP>(k, sh));
+  *chunks_out = chunks;
+  return MPRESS_OK;
+}
+
+template <typename K, typename Arg>
+int launch_kernel(K k, const Shape& sh, unsigned grid, bool pdl, cudaStream_t stream, Arg arg) {
+  MP_TRY(prepare(k, sh));
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(grid);
   cfg.blockDim = dim3(sh.threads);
@@ -549,9 +602,60 @@ int launch_batch(int path, int variant, int dir, const CopyDesc* d, const int* g
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = pdl ? 1 : 0;
-  cudaError_t e = cudaLaunchKernelEx(&cfg, k, t);
+  HP_START();
+  cudaError_t e = cudaLaunchKernelEx(&cfg, k, arg);
+  HP_LAP(11, "launch: cudaLaunchKernelEx");
   if (e == cudaSuccess) e = cudaGetLastError();
   if (e != cudaSuccess) return fail(MPRESS_ERR_CUDA, "swap kernel launch: %s", cudaGetErrorString(e));
+  return MPRESS_OK;
+}
+
+// One launch with the table as a kernel parameter.
+template <int CAP>
+int launch_batch(int path, int variant, int dir, const CopyDesc* d, const int* gid, uint32_t n,
+                 uint32_t shift, int cap, int sms, bool pdl, cudaStream_t stream, bool* launched) {
+  CopyTable<CAP> t;
+  uint64_t chunks;
+  *launched = false;
+  MP_TRY(build_table(t, d, gid, n, shift, &chunks));
+  if (chunks == 0) return MPRESS_OK;
+  const unsigned grid = (unsigned)std::min<uint64_t>(chunks, (uint64_t)cap);
+  const Shape& sh = shape_of(path, variant);
+  MP_TRY(launch_kernel(kernel_for<CAP, false>(path, variant, dir, (int)grid <= sms), sh, grid, pdl, stream, t));
+  *launched = true;
+  return MPRESS_OK;
+}
+
+// One launch with the table device-resident (TableRing): built in a pinned
+// staging slot, copied to the device slot on `stream` (only the used prefix),
+// read by the kernel through a pointer; the slot's event, recorded after the
+// kernel, guards both slots' reuse.
+int launch_batch_ring(TableRing* r, int path, int variant, int dir, const CopyDesc* d, const int* gid, uint32_t n,
+                      uint32_t shift, int cap, int sms, bool pdl, cudaStream_t stream, bool* launched) {
+  using T = CopyTable<kMaxDescPerLaunch>;
+  *launched = false;
+  const int slot = r->next;
+  if (r->armed[slot]) {
+    const cudaError_t e = cudaEventSynchronize(r->ev[slot]);   // blocks only if the ring wrapped
+    if (e != cudaSuccess) return fail(MPRESS_ERR_CUDA, "descriptor ring: %s", cudaGetErrorString(e));
+    r->armed[slot] = false;
+  }
+  T* ht = reinterpret_cast<T*>(r->host + (size_t)slot * r->slot_bytes);
+  T* dt = reinterpret_cast<T*>(r->dev + (size_t)slot * r->slot_bytes);
+  uint64_t chunks;
+  MP_TRY(build_table(*ht, d, gid, n, shift, &chunks));
+  if (chunks == 0) return MPRESS_OK;
+  r->next = (slot + 1) % r->nslots;
+  const size_t bytes = offsetof(T, d) + (size_t)n * sizeof(CopyDesc);
+  cudaError_t e = cudaMemcpyAsync(dt, ht, bytes, cudaMemcpyHostToDevice, stream);
+  if (e != cudaSuccess) return fail(MPRESS_ERR_CUDA, "descriptor upload: %s", cudaGetErrorString(e));
+  const unsigned grid = (unsigned)std::min<uint64_t>(chunks, (uint64_t)cap);
+  const Shape& sh = shape_of(path, variant);
+  MP_TRY(launch_kernel(kernel_for<kMaxDescPerLaunch, true>(path, variant, dir, (int)grid <= sms), sh, grid, pdl,
+                       stream, static_cast<const T*>(dt)));
+  e = cudaEventRecord(r->ev[slot], stream);
+  if (e != cudaSuccess) return fail(MPRESS_ERR_CUDA, "descriptor ring event: %s", cudaGetErrorString(e));
+  r->armed[slot] = true;
   *launched = true;
   return MPRESS_OK;
 }
@@ -566,8 +670,8 @@ int copy_wave_ctas(int path, int variant) {
   int& w = g_cache.wave[pi][variant][dev];
   if (w == 0) {
     const Shape& sh = shape_of(path, variant);
-    KernelFn<kMaxDescPerLaunch> k = kernel_for<kMaxDescPerLaunch>(path, variant, kDirOut, false);
-    if (prepare<kMaxDescPerLaunch>(k, sh) != MPRESS_OK) return 0;
+    KernelFn<kMaxDescPerLaunch> k = kernel_for<kMaxDescPerLaunch, false>(path, variant, kDirOut, false);
+    if (prepare(k, sh) != MPRESS_OK) return 0;
     int sms = 0, per_sm = 0;
     if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) return 0;
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, (const void*)k, sh.threads, sh.smem) != cudaSuccess)
@@ -578,7 +682,7 @@ int copy_wave_ctas(int path, int variant) {
 }
 
 namespace {
-template <int CAP>
+template <int CAP, bool G>
 int preload_cap() {
   for (int path : {MPRESS_PATH_DIRECT, MPRESS_PATH_BULK}) {
     const int nvar = path == MPRESS_PATH_BULK ? kBulkVariants : kDirectVariants;
@@ -586,10 +690,10 @@ int preload_cap() {
       for (int dir : {kDirOut, kDirIn})
         for (bool pf : {false, true}) {
           cudaFuncAttributes a;
-          KernelFn<CAP> k = kernel_for<CAP>(path, v, dir, pf);
+          auto k = kernel_for<CAP, G>(path, v, dir, pf);
           if (cudaFuncGetAttributes(&a, (const void*)k) != cudaSuccess)
             return fail(MPRESS_ERR_CUDA, "cannot load the swap kernels");
-          MP_TRY(prepare<CAP>(k, shape_of(path, v)));
+          MP_TRY(prepare(k, shape_of(path, v)));
         }
   }
   return MPRESS_OK;
@@ -600,13 +704,49 @@ int preload_cap() {
 // wait for the whole device; loading every swap kernel at context creation
 // keeps that stall out of the training step.
 int preload_kernels() {
-  MP_TRY(preload_cap<16>());
-  MP_TRY(preload_cap<128>());
-  return preload_cap<kMaxDescPerLaunch>();
+  MP_TRY((preload_cap<16, false>()));
+  MP_TRY((preload_cap<32, false>()));
+  MP_TRY((preload_cap<64, false>()));
+  MP_TRY((preload_cap<128, false>()));
+  MP_TRY((preload_cap<kMaxDescPerLaunch, false>()));
+  return preload_cap<kMaxDescPerLaunch, true>();
+}
+
+int table_ring_create(int device, TableRing** out) {
+  *out = nullptr;
+  auto* r = new TableRing();
+  r->device = device;
+  r->slot_bytes = (sizeof(CopyTable<kMaxDescPerLaunch>) + 255) / 256 * 256;
+  r->nslots = 256;   // 7.4 MB device + 7.4 MB pinned: 256 large launches in flight before the host waits
+  r->ev = new cudaEvent_t[r->nslots]();
+  r->armed = new bool[r->nslots]();
+  const size_t bytes = r->slot_bytes * r->nslots;
+  cudaError_t e = cudaMalloc(&r->dev, bytes);
+  if (e == cudaSuccess) e = cudaHostAlloc(&r->host, bytes, cudaHostAllocDefault);
+  for (int i = 0; i < r->nslots && e == cudaSuccess; ++i) e = cudaEventCreateWithFlags(&r->ev[i], cudaEventDisableTiming);
+  if (e != cudaSuccess) {
+    table_ring_destroy(r);
+    return fail(MPRESS_ERR_CUDA, "descriptor ring (%zu B): %s", bytes, cudaGetErrorString(e));
+  }
+  *out = r;
+  return MPRESS_OK;
+}
+
+void table_ring_destroy(TableRing* r) {
+  if (!r) return;
+  for (int i = 0; i < r->nslots; ++i) {
+    if (r->armed[i]) cudaEventSynchronize(r->ev[i]);
+    if (r->ev[i]) cudaEventDestroy(r->ev[i]);
+  }
+  if (r->dev) cudaFree(r->dev);
+  if (r->host) cudaFreeHost(r->host);
+  delete[] r->ev;
+  delete[] r->armed;
+  delete r;
 }
 
 int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* group, size_t n,
-                int max_ctas, int pdl_mode, cudaStream_t stream, int* launches) {
+                int max_ctas, int pdl_mode, cudaStream_t stream, int* launches, TableRing* ring) {
   int dev = 0, sms = 0;
   if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess)
     return fail(MPRESS_ERR_CUDA, "cannot query the SM count");
@@ -647,8 +787,14 @@ int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* gr
     const uint32_t m = (uint32_t)std::min<size_t>(kMaxDescPerLaunch, n - base);
     const int* g = group ? group + base : nullptr;
     bool launched = false;
-    if (m <= 16)
+    if (ring && m > (uint32_t)kParamDescMax)
+      MP_TRY(launch_batch_ring(ring, path, variant, dir, d + base, g, m, shift, cap, sms, pdl, stream, &launched));
+    else if (m <= 16)
       MP_TRY(launch_batch<16>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, stream, &launched));
+    else if (m <= 32)
+      MP_TRY(launch_batch<32>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, stream, &launched));
+    else if (m <= 64)
+      MP_TRY(launch_batch<64>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, stream, &launched));
     else if (m <= 128)
       MP_TRY(launch_batch<128>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, stream, &launched));
     else

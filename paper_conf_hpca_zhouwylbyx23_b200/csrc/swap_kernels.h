@@ -24,15 +24,39 @@ constexpr int kCeVariants = 2;           // copy engines: 0 per-peer streams, 1 
 
 enum CopyDir { kDirOut = 0, kDirIn = 1 };
 
+// Device-resident descriptor tables for launches with more than
+// kParamDescMax descriptors: a 28 KB __grid_constant__ table costs ~20 us of
+// host time per launch and fills the driver's launch queue after ~60 queued
+// launches (tools/hostcost.py), so large tables are written into a pinned
+// staging slot, copied to a device slot on the launch's stream, and the
+// kernel reads them through a pointer.  A slot is reused once the event
+// recorded after its kernel has completed.  Not used under graph capture (a
+// replay would re-read a staging slot that later launches overwrote).
+struct TableRing {
+  int device = -1;
+  size_t slot_bytes = 0;
+  int nslots = 0;
+  uint8_t* dev = nullptr;     // nslots x slot_bytes, device memory
+  uint8_t* host = nullptr;    // nslots x slot_bytes, pinned staging
+  cudaEvent_t* ev = nullptr;  // per slot: recorded after the kernel reading it
+  bool* armed = nullptr;      // per slot: ev was recorded
+  int next = 0;
+};
+constexpr int kParamDescMax = 128;
+int table_ring_create(int device, TableRing** out);
+void table_ring_destroy(TableRing* r);
+
 // Enqueue kernels moving every descriptor on `stream`; `path` is
 // MPRESS_PATH_DIRECT or MPRESS_PATH_BULK, `variant` its kernel shape;
 // `max_ctas` caps the grid (0 = the variant's default grid); `pdl_mode`
 // (MPRESS_OPT_PDL: 0 never, 1 uncapped grids only, 2 always) launches with
 // programmatic stream serialization.  Adds the number
 // of kernel launches to *launches.  Returns MPRESS_OK or MPRESS_ERR_*.
+// `ring` (may be null): device-resident tables for launches of more than
+// kParamDescMax descriptors.
 int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* group, size_t n,
                 int max_ctas, int pdl_mode,
-                cudaStream_t stream, int* launches);
+                cudaStream_t stream, int* launches, TableRing* ring = nullptr);
 
 // Default grid of a path/variant on the current device (SMs x CTAs per SM).
 int copy_wave_ctas(int path, int variant);

@@ -21,6 +21,7 @@ from synth import device as synth_dev  # noqa: E402
 
 def main():
     n_tensors = int(sys.argv[1]) if len(sys.argv) > 1 else 4
+    pdl = int(sys.argv[2]) if len(sys.argv) > 2 else 1
     sizes = [4096] * n_tensors
     world = 4
     spare = [0, 1 << 30, 1 << 30, 1 << 30]
@@ -29,12 +30,15 @@ def main():
     part = [[0] * world for _ in range(world)]
     part[0] = [64 * u * mp.DEFAULT_GRANULE for u in pl.units]
     ctx = mp.Context.local(world, 0, [0] * world, part)
+    ctx.set_option(mp.OPT_PDL, pdl)
     src = [torch.empty(s, dtype=torch.uint8, device="cuda") for s in sizes]
     dst = [torch.empty(s, dtype=torch.uint8, device="cuda") for s in sizes]
     s = torch.cuda.Stream()
     base = torch.zeros(1, dtype=torch.int64, device="cuda")
     res = {}
-    R = 150   # stays below the stream's queue depth (the host would block)
+    # stays below the stream's queue depth (the host would block); large
+    # descriptor tables (28 KB of kernel parameters) fill the launch queue sooner
+    R = int(sys.argv[3]) if len(sys.argv) > 3 else 150
     for mode in ("python", "ctypes"):
         synth_dev.stamp(base, s)
         synth_dev.gate(base, 2_000_000_000, s)     # ~2 s of GPU work queued first
@@ -55,6 +59,8 @@ def main():
         res[mode + "_us_per_pair"] = (time.perf_counter() - t0) / R * 1e6
         torch.cuda.synchronize()
     res["n_tensors"] = n_tensors
+    res["stripes"] = len(pl.stripes)
+    res["pdl"] = pdl
     print(json.dumps(res))
     ctx.finalize()
 
