@@ -224,8 +224,8 @@ __device__ __forceinline__ void direct_body(const CopyTable<CAP>& t) {
   if (!cur.next(&c, &s)) return;
   Span sp = span_of<kShift>(t, c, s);
   for (;;) {
-    Span nx;
-    bool more;
+    Span nx{nullptr, nullptr, 0};
+    bool more = false;
     if (sp.rem >= kChunk) {
       const VT* sv = reinterpret_cast<const VT*>(sp.src) + threadIdx.x;
       VT* dv = reinterpret_cast<VT*>(sp.dst) + threadIdx.x;

@@ -142,6 +142,23 @@ for path, variant, cap in ((mp.PATH_BULK, 0, 2), (mp.PATH_BULK, 3, 3), (mp.PATH_
     assert all(synth_dev.check(d, 9, i) == 0 for i, d in enumerate(dst)), (path, variant, cap)
     h.free()
 ctx.finalize()
+# > 128 descriptors: device-resident tables (pinned staging -> device slot)
+sizes = [1 + (i * 7919) % 5000 for i in range(140)]
+pl = mp.plan(3, 0, [0, 1 << 30, 1 << 30], [0, 1, 1], sizes)
+assert len(pl.stripes) > 128
+ctx = mp.Context.local(3, 0, [0, 0, 0], [[0] + [u * 65536 for u in pl.units[1:]], [0] * 3, [0] * 3])
+src = [torch.empty(n, dtype=torch.uint8, device="cuda") for n in sizes]
+for i, t in enumerate(src):
+    synth_dev.fill(t, 10, i)
+for path in (mp.PATH_BULK, mp.PATH_DIRECT):
+    ctx.set_option(mp.OPT_PATH, path)
+    dst = [torch.zeros(n, dtype=torch.uint8, device="cuda") for n in sizes]
+    h = ctx.swap_out(pl, src)
+    ctx.swap_in(h, dst)
+    torch.cuda.synchronize()
+    assert all(synth_dev.check(d, 10, i) == 0 for i, d in enumerate(dst)), path
+    h.free()
+ctx.finalize()
 print("multi-piece ok")
 """
 
@@ -153,8 +170,9 @@ print("multi-piece ok")
 def test_sanitizer_multi_piece_ctas(tool):
     """Kernels whose CTAs move many pieces each (small grids), so the bulk
     path's slot ring wraps, its per-lane cursors finish at different times and
-    its shuffles/ballots run every batch: no memory error, shared-memory race
-    or illegal warp/barrier synchronisation."""
+    its shuffles/ballots run every batch; and launches with > 128 descriptors
+    (device-resident tables): no memory error, shared-memory race or illegal
+    warp/barrier synchronisation."""
     cs = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitizer"
     r = subprocess.run([cs, "--tool", tool, "--error-exitcode", "9", sys.executable, "-c", _MULTI_PIECE],
                        cwd=ROOT, capture_output=True, text=True, timeout=900)
