@@ -147,6 +147,7 @@ sizes = [1 + (i * 7919) % 5000 for i in range(140)]
 pl = mp.plan(3, 0, [0, 1 << 30, 1 << 30], [0, 1, 1], sizes)
 assert len(pl.stripes) > 128
 ctx = mp.Context.local(3, 0, [0, 0, 0], [[0] + [u * 65536 for u in pl.units[1:]], [0] * 3, [0] * 3])
+ctx.autotune(probe_bytes=256 << 10, trials=1)   # the probe kernels and scratch buffers too
 src = [torch.empty(n, dtype=torch.uint8, device="cuda") for n in sizes]
 for i, t in enumerate(src):
     synth_dev.fill(t, 10, i)
