@@ -169,8 +169,13 @@ def _ptr(x):
 
 def pointers(tensors):
     """A reusable C array of the tensors' device addresses (marshal once,
-    pass to swap_out / swap_in many times; the tensors must stay alive)."""
-    return (c_void_p * len(tensors))(*[_ptr(t) for t in tensors])
+    pass to swap_out / swap_in many times; the tensors must stay alive).
+    A uint64 array: the same bytes as `void* const*` on the 64-bit ABI, and
+    ~3x cheaper to build from a list of tensors than c_void_p items."""
+    try:
+        return (c_uint64 * len(tensors))(*[t.data_ptr() for t in tensors])
+    except AttributeError:   # int addresses mixed in
+        return (c_uint64 * len(tensors))(*[_ptr(t) for t in tensors])
 
 
 def _ptr_array(x):
