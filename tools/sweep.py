@@ -341,6 +341,11 @@ def power():
 
     window(None)   # warm to the sustained power state
     settings = [("direct", 7, 32), ("direct", 7, 64), ("direct", 9, 64), ("direct", 7, 148), ("ce", 0, 0)]
+    if os.environ.get("POWER_SETTINGS"):   # e.g. "direct:7:16,32,64;bulk:5:148;ce:0:0"
+        settings = []
+        for part in os.environ["POWER_SETTINGS"].split(";"):
+            nm, v, caps = part.split(":")
+            settings += [(nm, int(v), int(c)) for c in caps.split(",")]
     for st in settings:
         al = window(None)
         wi = window(st)
