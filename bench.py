@@ -65,6 +65,7 @@ def parse():
     ap.add_argument("--gemm-cap", type=int, default=64,
                     help="swap grid cap (CTAs = SMs touched) while the concurrent GEMM runs")
     ap.add_argument("--no-gemm", action="store_true")
+    ap.add_argument("--no-gemm-ce", action="store_true", help="skip the copy-engine pass of the GEMM leg")
     ap.add_argument("--gemm-settle-s", type=float, default=2.0,
                     help="back-to-back GEMMs before the GEMM-slowdown rounds (power state)")
     ap.add_argument("--gemm-n", type=int, default=8192, help="GEMM size of the N>1 config-5 leg")
@@ -451,6 +452,8 @@ def main():
     e2e = leg(run_e2e, args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap_stream, n, dist)
     gemm = None if args.no_gemm else leg(gemm_interference, args, ctx, mp, world, source, per_copy, bw,
                                          sizes, src, dst, swap_stream, n, dist)
+    gemm_ce = None if (args.no_gemm or args.no_gemm_ce) else leg(
+        gemm_interference, args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap_stream, n, dist, True)
     cfg5 = None
     if n > 1 and not args.no_gemm and not args.no_cfg5:
         cfg5 = leg(cfg5_leg, args, mp, rank, n, local_rank, dist)
@@ -476,7 +479,7 @@ def main():
             "swap_path_ran": ran_by_dir, "autotune": autotune,
             "per_direction_gbs": per_dir,
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
-            "gpu_launches": launches[0], "clocks": clk, "gemm_slowdown": gemm,
+            "gpu_launches": launches[0], "clocks": clk, "gemm_slowdown": gemm, "gemm_slowdown_ce": gemm_ce,
             "planner": planner, "other_configs": others, "cfg5": cfg5,
             "parity": "round trip bit-exact vs generator (all %d tensors x %d ranks)" % (47 * mb, n),
             "per_rank_gbs": value / n,
@@ -642,12 +645,13 @@ class _Local:
             return None
 
 
-def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap, n, dist):
+def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap, n, dist, ce=False):
     """Second half of the metric: slowdown of a bf16 GEMM (8192^3, the shape
     MEASURED_PEAKS.json is quoted on) on the compute stream while swaps loop on
     the side stream with the grid capped at --gemm-cap CTAs.  Alone and
     with-swap rounds alternate (so power-cap drift hits both), and only GEMMs
-    that ran entirely inside the swap window count."""
+    that ran entirely inside the swap window count.  ce=True: the same with
+    the copy-engine comparator (a7, no SMs) moving the swap."""
     import torch
     comp = torch.cuda.current_stream()
     M = K = N = 8192
@@ -674,6 +678,9 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
         st["pl"] = mp.plan(world, source, per_copy, bw, sizes)
         st["old_cap"] = ctx.get_option(mp.OPT_MAX_CTAS)
         ctx.set_option(mp.OPT_MAX_CTAS, args.gemm_cap)
+        if ce:
+            st["old_path"] = ctx.get_option(mp.OPT_PATH)
+            ctx.set_option(mp.OPT_PATH, mp.PATH_CE)
         # swap time at this cap, to size the loop that must cover the GEMM window
         e0 = torch.cuda.Event(enable_timing=True)
         e1 = torch.cuda.Event(enable_timing=True)
@@ -704,13 +711,21 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
         n_swap = int(2.0 * G * gemm_ms / st["per_swap_ms"]) + 2
         s0 = torch.cuda.Event(enable_timing=True)
         s1 = torch.cuda.Event(enable_timing=True)
+        # The SM paths enqueue in ~10 us per call, far ahead of the GPU, so
+        # their swaps go first and cover the whole GEMM run.  The copy-engine
+        # path costs ~3 us of host time per stripe (one cudaMemcpyAsync each):
+        # enqueued first, its swaps would run as fast as the host issues them
+        # and be over before the GEMMs start, so the GEMMs go first there.
+        if ce:
+            evs = gemms()
         s0.record(swap)
         for _ in range(n_swap):
             h = ctx.swap_out(st["pl"], src[0], stream=swap)
             ctx.swap_in(h, dst[0], stream=swap)
             h.free()
         s1.record(swap)
-        evs = gemms()
+        if not ce:
+            evs = gemms()
         torch.cuda.synchronize()
         win = s0.elapsed_time(s1)
         d_r = [x.elapsed_time(y) for x, y in evs[4:]
@@ -726,6 +741,8 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
     st["ran"] = ctx.get_option(mp.OPT_LAST_PATH)
     if "old_cap" in st:
         L(ctx.set_option, mp.OPT_MAX_CTAS, st["old_cap"])
+    if "old_path" in st:
+        L(ctx.set_option, mp.OPT_PATH, st["old_path"])
     t = torch.tensor([statistics.median(alone) if alone else float("nan"),
                       statistics.median(during) if during else float("nan"),
                       1.0 if L.err is not None else 0.0,
@@ -746,7 +763,7 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
             "rounds": len(ratios),
             "slowdown_per_round": [r - 1 for r in ratios],
             "swap_path": {mp.PATH_DIRECT: "direct", mp.PATH_BULK: "bulk", mp.PATH_CE: "ce"}.get(
-                st.get("ran"), args.path), "swap_max_ctas": args.gemm_cap,
+                st.get("ran"), args.path), "swap_max_ctas": None if ce else args.gemm_cap,
             # MPRESS_OPT_PDL 1 (default) launches a capped grid without PDL
             "swap_pdl_mode": ctx.get_option(mp.OPT_PDL),
             "swap_gbs_during": statistics.median(swap_gbs),
