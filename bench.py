@@ -76,6 +76,18 @@ def parse():
     return ap.parse_args()
 
 
+def _finite(x):
+    """The JSON line must be strict JSON: NaN / inf (e.g. a slowdown with no
+    GEMM inside the swap window) become null."""
+    if isinstance(x, float):
+        return x if x == x and x not in (float("inf"), float("-inf")) else None
+    if isinstance(x, dict):
+        return {k: _finite(v) for k, v in x.items()}
+    if isinstance(x, (list, tuple)):
+        return [_finite(v) for v in x]
+    return x
+
+
 def measured_peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
@@ -220,7 +232,7 @@ def run_reference(args):
             "data": "synthetic", "config": workload_config(args, args.gpus),
             "cpu_baseline": {"value": v, "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": sample},
             "e2e": {"value": v, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
-    print(json.dumps(line))
+    print(json.dumps(_finite(line), allow_nan=False))
     return 0
 
 
@@ -455,8 +467,11 @@ def main():
     gemm_ce = None if (args.no_gemm or args.no_gemm_ce) else leg(
         gemm_interference, args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap_stream, n, dist, True)
     cfg5 = None
+    cfg5_ce = None
     if n > 1 and not args.no_gemm and not args.no_cfg5:
         cfg5 = leg(cfg5_leg, args, mp, rank, n, local_rank, dist)
+        if not args.no_gemm_ce:
+            cfg5_ce = leg(cfg5_leg, args, mp, rank, n, local_rank, dist, True)
     others = None
     if n == 1 and not args.no_configs:
         del src, dst
@@ -480,7 +495,7 @@ def main():
             "per_direction_gbs": per_dir,
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": launches[0], "clocks": clk, "gemm_slowdown": gemm, "gemm_slowdown_ce": gemm_ce,
-            "planner": planner, "other_configs": others, "cfg5": cfg5,
+            "planner": planner, "other_configs": others, "cfg5": cfg5, "cfg5_ce": cfg5_ce,
             "parity": "round trip bit-exact vs generator (all %d tensors x %d ranks)" % (47 * mb, n),
             "per_rank_gbs": value / n,
             "transport": {mp.TRANSPORT_LOCAL: "local (mpress_init_local)",
@@ -494,7 +509,7 @@ def main():
             "note": "N=1 and N>1 cross different links, so value(N) / (N * value(1)) is not a "
                     "scaling efficiency; compare per_rank_gbs with the NVLink roofline",
         }
-        print(json.dumps(line))
+        print(json.dumps(_finite(line), allow_nan=False))
     ctx.finalize()
     if n > 1:
         dist.destroy_process_group()
@@ -773,7 +788,7 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
                     ("every rank swaps to all others while running the GEMM; max over ranks")}
 
 
-def cfg5_leg(args, mp, rank, n, device, dist):
+def cfg5_leg(args, mp, rank, n, device, dist, ce=False):
     """BASELINE config 5 (BJ:11, reading R20) at N GPUs: the
     first half of the ranks are the heavy stages (sources), the second half
     the light ones (pure importers).  Source s swaps (N/2 - s) Bert stage-0
@@ -782,7 +797,8 @@ def cfg5_leg(args, mp, rank, n, device, dist):
     sequential partition (R12), grid capped at --gemm-cap CTAs, while EVERY
     rank runs back-to-back bf16 GEMMs on its compute stream.  Reports each
     source's swap GB/s (out + in) under contention and the GEMM slowdown on
-    sources and importers.  Every collective is reached by all ranks even if
+    sources and importers.  ce=True: the same with the copy-engine
+    comparator moving the swaps (no SMs).  Every collective is reached by all ranks even if
     a rank's local work fails (the failure is reported, not hung on)."""
     import torch
     from synth import device as synth_dev
@@ -822,6 +838,8 @@ def cfg5_leg(args, mp, rank, n, device, dist):
             for p in range(n):
                 rem[p] -= part[s][p]
         ctx.set_option(mp.OPT_MAX_CTAS, args.gemm_cap)
+        if ce:
+            ctx.set_option(mp.OPT_PATH, mp.PATH_CE)
         st["a"] = torch.randn(M, M, dtype=torch.bfloat16, device="cuda")
         st["b"] = torch.randn(M, M, dtype=torch.bfloat16, device="cuda")
         st["c"] = torch.empty(M, M, dtype=torch.bfloat16, device="cuda")
@@ -864,6 +882,7 @@ def cfg5_leg(args, mp, rank, n, device, dist):
 
     def run_with_swap():
         s0 = s1 = None
+        evs = gemms() if ce else None   # copy engines: GEMMs first (see gemm_interference)
         if is_src:
             n_swap = int(2.0 * G * statistics.median(alone) / st["per_swap_ms"]) + 2
             s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -873,7 +892,8 @@ def cfg5_leg(args, mp, rank, n, device, dist):
                 ctx.swap_in(h, st["dst"], stream=swap)
                 h.free()
             s1.record(swap)
-        evs = gemms()
+        if not ce:
+            evs = gemms()
         torch.cuda.synchronize()
         if is_src:
             win = s0.elapsed_time(s1)
@@ -909,7 +929,8 @@ def cfg5_leg(args, mp, rank, n, device, dist):
     return {"config": "cfg5 imbalanced all-stage swap: sources %s -> importers %s, source s swaps %s micro-batch "
                       "sets (900 MiB each, one plan), bf16 %dx%dx%d GEMMs on every rank" %
                       (sources, peers, [H - s for s in sources], M, M, M),
-            "swap_max_ctas": args.gemm_cap,
+            "swap_path": "ce" if ce else "auto (capped -> direct)",
+            "swap_max_ctas": None if ce else args.gemm_cap,
             "per_source_gbs": [float(row[s, 2]) for s in sources],
             "per_source_bytes": [sum(workloads.cfg2_sizes(H - s)) for s in sources],
             "gemm_alone_ms": [float(row[r, 0]) for r in range(n)],

@@ -27,3 +27,14 @@ def test_reference_arm_non_zero_rank_is_silent():
     r = subprocess.run([sys.executable, "bench.py", "--impl", "reference", "--steps", "1", "--warmup", "1"],
                        cwd=ROOT, capture_output=True, text=True, timeout=300, env=env)
     assert r.returncode == 0 and r.stdout.strip() == ""
+
+
+def test_json_line_is_strict_json():
+    """NaN / inf never reach the JSON line (a strict parser would reject it)."""
+    import importlib.util
+    spec = importlib.util.spec_from_file_location("bench_mod", os.path.join(ROOT, "bench.py"))
+    b = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(b)
+    line = b._finite({"slowdown": float("nan"), "x": [1.5, float("inf")], "y": {"z": float("-inf"), "w": 2}})
+    assert line == {"slowdown": None, "x": [1.5, None], "y": {"z": None, "w": 2}}
+    json.dumps(line, allow_nan=False)
