@@ -128,7 +128,7 @@ extern "C" int mpress_schedule_1f1b(const mpress_1f1b_params* p, mpress_1f1b_slo
     return fail(MPRESS_ERR_ARG, "mpress_schedule_1f1b: bad stages/stage/micro_batches");
   try {
     // 1. the no-swap timeline
-    Pipeline base{S, M};
+    Pipeline base{S, M, {}, {}, {}, {}};
     base.build(p->t_fwd_ns, p->t_bwd_ns);
     std::vector<uint64_t> s0, e0;
     if (!base.g.longest(&s0, &e0)) return fail(MPRESS_ERR_ARG, "mpress_schedule_1f1b: cyclic model");
@@ -152,7 +152,7 @@ extern "C" int mpress_schedule_1f1b(const mpress_1f1b_params* p, mpress_1f1b_slo
       trig[m] = j;
     }
     // 3. the timeline with the swap ops of stage e, in executor enqueue order
-    Pipeline sw{S, M};
+    Pipeline sw{S, M, {}, {}, {}, {}};
     sw.build(p->t_fwd_ns, p->t_bwd_ns);
     std::vector<int> outn(M, -1), inn(M, -1);
     int last_out = -1, last_in = -1;  // stream order (duplex: two streams)

@@ -615,7 +615,7 @@ template <int CAP>
 int launch_batch(int path, int variant, int dir, const CopyDesc* d, const int* gid, uint32_t n,
                  uint32_t shift, int cap, int sms, bool pdl, cudaStream_t stream, bool* launched) {
   CopyTable<CAP> t;
-  uint64_t chunks;
+  uint64_t chunks = 0;
   *launched = false;
   MP_TRY(build_table(t, d, gid, n, shift, &chunks));
   if (chunks == 0) return MPRESS_OK;
@@ -642,7 +642,7 @@ int launch_batch_ring(TableRing* r, int path, int variant, int dir, const CopyDe
   }
   T* ht = reinterpret_cast<T*>(r->host + (size_t)slot * r->slot_bytes);
   T* dt = reinterpret_cast<T*>(r->dev + (size_t)slot * r->slot_bytes);
-  uint64_t chunks;
+  uint64_t chunks = 0;
   MP_TRY(build_table(*ht, d, gid, n, shift, &chunks));
   if (chunks == 0) return MPRESS_OK;
   r->next = (slot + 1) % r->nslots;
