@@ -23,7 +23,7 @@ SYNTH_LIB = os.path.join(ROOT, "synth", "libsynth.so")
 
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
-CFLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-fvisibility=hidden",
+CFLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-fvisibility=hidden,-Wall,-Wextra",
           "-I" + os.path.join(ROOT, "include")] + os.environ.get("MPRESS_NVCC_FLAGS", "").split()
 
 
