@@ -56,3 +56,35 @@ def test_mixed_nvlink_and_host_striping(path):
     o = _roundtrip(world, [0, 0, 0, 0, mp.DEVICE_HOST], [0] + [1 << 30] * 4, [0, 900, 900, 900, 55],
                    [1000, 70000, 3 << 20, 17], 12, path)
     assert 0 < o["units"][4] < o["units"][1]
+
+
+def test_autotune_skips_host_pools():
+    """mpress_autotune probes only device peers (a host pool is PCIe, and AUTO
+    sends any swap touching one to the direct kernel anyway): with a device
+    peer and a host peer it times the device peer, leaves the host pool's
+    free space untouched, and AUTO swaps still run direct and bit-exact."""
+    from synth import device as synth_dev
+    world = 3
+    spare, bw = [0, 1 << 30, 1 << 30], [0, 900, 55]
+    sizes = [3 << 20, 4097]
+    pl = mp.plan(world, 0, spare, bw, sizes)
+    part = [[0] + [2 * u * 65536 for u in pl.units[1:]], [0] * 3, [0] * 3]
+    ctx = mp.Context.local(world, 0, [0, 0, mp.DEVICE_HOST], part)
+    try:
+        free0 = ctx.stash_free()
+        res = ctx.autotune(probe_bytes=1 << 20, trials=1)
+        assert all(v > 0 for v in res["ms"].values()), res
+        assert ctx.stash_free() == free0
+        src = [torch.empty(n, dtype=torch.uint8, device="cuda") for n in sizes]
+        for i, t in enumerate(src):
+            synth_dev.fill(t, 81, i)
+        dst = [torch.zeros(n, dtype=torch.uint8, device="cuda") for n in sizes]
+        torch.cuda.synchronize()
+        h = ctx.swap_out(pl, src)
+        assert ctx.get_option(mp.OPT_LAST_PATH) == mp.PATH_DIRECT
+        ctx.swap_in(h, dst)
+        torch.cuda.synchronize()
+        assert all(synth_dev.check(d, 81, i) == 0 for i, d in enumerate(dst))
+        h.free()
+    finally:
+        ctx.finalize()
