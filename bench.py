@@ -62,8 +62,13 @@ def parse():
     ap.add_argument("--e2e-steps", type=int, default=16)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
-    ap.add_argument("--gemm-cap", type=int, default=64,
-                    help="swap grid cap (CTAs = SMs touched) while the concurrent GEMM runs")
+    ap.add_argument("--gemm-cap", type=int, default=0,
+                    help="swap grid cap (CTAs = SMs touched) while the concurrent GEMM runs; 0 = calibrate: "
+                         "the smallest of --gemm-cap-candidates whose swap rate on this run's links reaches "
+                         "--gemm-target-gbs / 0.85")
+    ap.add_argument("--gemm-cap-candidates", default="64,96,128,148")
+    ap.add_argument("--gemm-target-gbs", type=float, default=720.0,
+                    help="per-source swap rate the GEMM-concurrent swap should sustain (BJ:5: 80%% of 900)")
     ap.add_argument("--no-gemm", action="store_true")
     ap.add_argument("--no-gemm-ce", action="store_true", help="skip the copy-engine pass of the GEMM leg")
     ap.add_argument("--gemm-settle-s", type=float, default=2.0,
@@ -462,6 +467,11 @@ def main():
             return {"error": "%s: %s" % (type(exc).__name__, exc)}
 
     e2e = leg(run_e2e, args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap_stream, n, dist)
+    cap_cal = None
+    if not args.no_gemm and args.gemm_cap <= 0:
+        cap_cal = calibrate_gemm_cap(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap_stream, n,
+                                     dist)
+        args.gemm_cap = cap_cal["chosen"]
     gemm = None if args.no_gemm else leg(gemm_interference, args, ctx, mp, world, source, per_copy, bw,
                                          sizes, src, dst, swap_stream, n, dist)
     gemm_ce = None if (args.no_gemm or args.no_gemm_ce) else leg(
@@ -495,6 +505,7 @@ def main():
             "per_direction_gbs": per_dir,
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": launches[0], "clocks": clk, "gemm_slowdown": gemm, "gemm_slowdown_ce": gemm_ce,
+            "gemm_cap_calibration": cap_cal,
             "planner": planner, "other_configs": others, "cfg5": cfg5, "cfg5_ce": cfg5_ce,
             "parity": "round trip bit-exact vs generator (all %d tensors x %d ranks)" % (47 * mb, n),
             "per_rank_gbs": value / n,
@@ -658,6 +669,60 @@ class _Local:
         except Exception as exc:  # pragma: no cover - reported in the line
             self.err = "%s: %s" % (type(exc).__name__, exc)
             return None
+
+
+def calibrate_gemm_cap(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap, n, dist):
+    """Grid cap of the GEMM-concurrent swap, measured on this run's links
+    (HBM loopback at N = 1, NVLink at N > 1, where every remote access pays
+    ~2x the latency, so the same cap keeps fewer bytes in flight per µs):
+    for each candidate cap the capped swap (AUTO -> direct shape 7) runs
+    alone, out + in, on every rank at once; the smallest cap whose slowest
+    rank reaches --gemm-target-gbs / 0.85 (headroom for the GEMM's
+    contention) is chosen, else the largest candidate.  Collective: every rank
+    reaches every barrier and reduction even if its own work fails."""
+    import torch
+    caps = [int(c) for c in args.gemm_cap_candidates.split(",") if c.strip()]
+    old = ctx.get_option(mp.OPT_MAX_CTAS)
+    pl = mp.plan(world, source, per_copy, bw, sizes)
+    nbytes = sum(sizes)
+    reps = 3
+    table, err = {}, None
+    for cap in caps:
+        rate = 0.0
+        if n > 1:
+            dist.barrier()
+        if err is None:
+            try:
+                ctx.set_option(mp.OPT_MAX_CTAS, cap)
+                h = ctx.swap_out(pl, src[0], stream=swap)     # warm-up
+                ctx.swap_in(h, dst[0], stream=swap)
+                h.free()
+                torch.cuda.synchronize()
+                e0 = torch.cuda.Event(enable_timing=True)
+                e1 = torch.cuda.Event(enable_timing=True)
+                e0.record(swap)
+                for _ in range(reps):
+                    h = ctx.swap_out(pl, src[0], stream=swap)
+                    ctx.swap_in(h, dst[0], stream=swap)
+                    h.free()
+                e1.record(swap)
+                torch.cuda.synchronize()
+                rate = 2 * reps * nbytes / e0.elapsed_time(e1) / 1e6
+            except Exception as exc:  # pragma: no cover - reported in the line
+                err = "%s: %s" % (type(exc).__name__, exc)
+        t = torch.tensor([rate if err is None else 0.0], dtype=torch.float64)
+        if n > 1:
+            dist.all_reduce(t, op=dist.ReduceOp.MIN)
+        table[cap] = float(t.item())
+    try:
+        ctx.set_option(mp.OPT_MAX_CTAS, old)
+    except Exception:  # pragma: no cover
+        pass
+    need = args.gemm_target_gbs / 0.85
+    ok = [c for c in caps if table[c] >= need]
+    chosen = (min(ok) if ok else max(caps)) if err is None else 64
+    return {"chosen": chosen, "target_gbs": args.gemm_target_gbs, "needed_alone_gbs": need,
+            "alone_gbs_by_cap_min_over_ranks": {str(c): table[c] for c in caps}, "error": err}
 
 
 def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap, n, dist, ce=False):
