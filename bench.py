@@ -81,6 +81,11 @@ def parse():
     return ap.parse_args()
 
 
+# mpress_autotune probe: 4 back-to-back 256 MiB launches per direction (large
+# class), 16 x 16 MiB (small class), over a 1 GiB working set
+AUTOTUNE_PROBE = 1 << 30
+
+
 def _finite(x):
     """The JSON line must be strict JSON: NaN / inf (e.g. a slowdown with no
     GEMM inside the swap window) become null."""
@@ -326,11 +331,11 @@ def main():
     if path == mp.PATH_AUTO and not args.no_autotune:
         # which SM kernel an uncapped AUTO swap runs on THIS run's links
         # (loopback HBM at N=1, NVLink at N>1), measured before the timed steps
-        res = ctx.autotune(probe_bytes=256 << 20, trials=5)
+        res = ctx.autotune(probe_bytes=AUTOTUNE_PROBE, trials=5)
         nm = {mp.PATH_DIRECT: "direct", mp.PATH_BULK: "bulk"}
         autotune = {"out": nm[res["out"]], "in": nm[res["in"]], "out_small": nm[res["out_small"]],
                     "in_small": nm[res["in_small"]], "small_below_bytes": mp.AUTO_SMALL_BYTES,
-                    "probe_bytes": 256 << 20, "trials": 5, "median_ms_per_launch": res["ms"]}
+                    "probe_bytes": AUTOTUNE_PROBE, "trials": 5, "median_ms_per_launch": res["ms"]}
 
     seed0 = 2000 + 100 * rank
     src = [[torch.empty(s, dtype=torch.uint8, device="cuda") for s in sizes] for _ in range(mb)]

@@ -476,24 +476,23 @@ MPRESS_API int mpress_set_option(mpress_ctx_t* ctx, int key, int64_t value);
 /* Measure, don't guess: which SM kernel MPRESS_PATH_AUTO should run for an
  * uncapped grid on THIS context's links (HBM loopback on one GPU, NVLink /
  * NVSwitch on several -- the kernels were only ever compared on loopback,
- * DESIGN.md §7), per direction and size class.  Class "large": one launch
- * each way of `probe_bytes` (split equally over the mapped device peers,
- * each share a multiple of 256 and at most that partition's largest free
- * block; use >= MPRESS_AUTO_SMALL_BYTES for a meaningful large-class
- * decision).  Class "small": 16 launches of 16 MiB (same split) back to back
- * each way, each on the next 16 MiB window of the probe, so that with
- * probe_bytes >= 256 MiB the working set exceeds the 126 MB L2 as a
- * pipeline's stream of fresh tensors does.  Both from a library-owned
- * scratch buffer into the
- * stash partitions and back, with the direct kernel (shape 5) and the bulk
- * kernel (shape 3); one warm-up round then `trials` (1..64) rounds
- * alternating which kernel goes first; per direction and class the median
- * times decide, and the class's current choice stays unless the other
- * kernel is at least 1% faster.  Read the result back with
- * MPRESS_OPT_AUTO_OUT / _IN / _OUT_SMALL / _IN_SMALL; every later AUTO swap of
- * this context with an uncapped grid uses it (a capped grid or a host peer
- * still takes the direct kernel).  Runs synchronously on `stream` (NULL =
- * legacy default stream).
+ * DESIGN.md §7), per direction and size class.  The probe is `probe_bytes`
+ * split equally over the mapped device peers (each share a multiple of 256
+ * and at most that partition's largest free block), moved out of a
+ * library-owned scratch buffer into the stash partitions and back as runs of
+ * back-to-back launches over successive windows of it, as a pipeline streams
+ * fresh tensors: class "large" = 4 launches of probe_bytes / 4, class
+ * "small" = 16 launches of 16 MiB.  Use probe_bytes >= 256 MiB so the
+ * working set exceeds the 126 MB L2 and each large launch is at least
+ * MPRESS_AUTO_SMALL_BYTES.  Both kernels are timed -- direct (shape 5) and
+ * bulk (shape 3) -- one warm-up round then `trials` (1..64) rounds
+ * alternating which goes first; per direction and class the median time per
+ * launch decides, and the class's current choice stays unless the other
+ * kernel is at least 2% faster (the probe's run-to-run noise is ~1%).  Read
+ * the result back with MPRESS_OPT_AUTO_OUT / _IN / _OUT_SMALL / _IN_SMALL;
+ * every later AUTO swap of this context with an uncapped grid uses it (a
+ * capped grid or a host peer still takes the direct kernel).  Runs
+ * synchronously on `stream` (NULL = legacy default stream).
  * Collective for an mpress_init context: every rank calls it with the same
  * `trials` (a rank without device peers only takes part in the barriers),
  * and each probe starts on all ranks together (barriers through the

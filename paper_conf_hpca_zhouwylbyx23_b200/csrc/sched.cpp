@@ -558,14 +558,16 @@ extern "C" int mpress_autotune(mpress_ctx_t* c, uint64_t probe_bytes, int trials
     for (int i = 0; i < 3 && e == cudaSuccess; ++i) e = cudaEventCreate(&ev[i]);
     if (e != cudaSuccess) rc = cuda_fail(e, "mpress_autotune: probe buffers");
   }
-  // Two probes per path.  Class 1 ("large"): the whole probe, one launch
-  // each way.  Class 0 ("small"): launches of kSmallProbe (split over the
-  // peers), kSmallReps back to back each way, each on the next window of the
-  // probe buffers, so the working set (the whole probe) exceeds L2 as a
-  // pipeline's stream of fresh tensors does -- repeating one 16 MiB window
-  // would time L2, not HBM / NVLink.
+  // Two probes per path, each a run of back-to-back launches over successive
+  // windows of the probe buffers, as a pipeline streams fresh tensors: the
+  // working set is the whole probe (beyond L2 for >= 256 MiB, so HBM / NVLink
+  // is timed, not L2) and launch ramps overlap their predecessors (PDL) as in
+  // steady state -- one isolated launch per trial overstated the bulk
+  // kernel's ramp and flipped a 1% decision against it.
+  // Class 1 ("large"): kLargeReps launches of probe/kLargeReps.  Class 0
+  // ("small"): kSmallReps launches of kSmallProbe (both split over the peers).
   constexpr uint64_t kSmallProbe = 16ull << 20;
-  constexpr int kSmallReps = 16;
+  constexpr int kSmallReps = 16, kLargeReps = 4;
   std::vector<CopyDesc> dout[2][kSmallReps], din[2][kSmallReps];
   std::vector<int> grp;
   uint64_t at = 0;
@@ -574,14 +576,17 @@ extern "C" int mpress_autotune(mpress_ctx_t* c, uint64_t probe_bytes, int trials
   for (int p : peers) {
     if (!len[p]) continue;
     grp.push_back(p);
-    dout[1][0].push_back({src + at, c->parts[p].base + off[p], len[p]});
-    din[1][0].push_back({c->parts[p].base + off[p], dst + at, len[p]});
-    const uint64_t n = std::min(len[p], small_share);
-    const uint64_t windows = std::max<uint64_t>(1, len[p] / n);
-    for (int w = 0; w < kSmallReps; ++w) {
-      const uint64_t o = (w % windows) * n;
-      dout[0][w].push_back({src + at + o, c->parts[p].base + off[p] + o, n});
-      din[0][w].push_back({c->parts[p].base + off[p] + o, dst + at + o, n});
+    for (int cls = 0; cls < 2; ++cls) {
+      const int reps = cls ? kLargeReps : kSmallReps;
+      const uint64_t n = cls ? std::max<uint64_t>(MPRESS_ALIGN, len[p] / kLargeReps / MPRESS_ALIGN * MPRESS_ALIGN)
+                             : std::min(len[p], small_share);
+      const uint64_t windows = std::max<uint64_t>(1, len[p] / n);
+      for (int w = 0; w < reps; ++w) {
+        const uint64_t o = (w % windows) * n;
+        const uint64_t m = std::min(n, len[p] - o);
+        dout[cls][w].push_back({src + at + o, c->parts[p].base + off[p] + o, m});
+        din[cls][w].push_back({c->parts[p].base + off[p] + o, dst + at + o, m});
+      }
     }
     at += len[p];
   }
@@ -590,7 +595,7 @@ extern "C" int mpress_autotune(mpress_ctx_t* c, uint64_t probe_bytes, int trials
   std::vector<float> t[2][2][2];  // [class][path][dir], ms per launch
   for (int r = -1; r < trials; ++r) {
     for (int cls = 0; cls < 2; ++cls) {
-      const int reps = cls ? 1 : kSmallReps;
+      const int reps = cls ? kLargeReps : kSmallReps;
       for (int k = 0; k < 2; ++k) {
         const int pi = (r & 1) ? 1 - k : k;
         rc = autotune_barrier(c, rc);
@@ -629,11 +634,11 @@ extern "C" int mpress_autotune(mpress_ctx_t* c, uint64_t probe_bytes, int trials
     for (int pi = 0; pi < 2; ++pi)
       for (int d = 0; d < 2; ++d) m[pi][d] = median(t[cls][pi][d]);
     if (!grp.empty())
-      for (int d = 0; d < 2; ++d) {  // the class default stays unless the other kernel is >= 1% faster
+      for (int d = 0; d < 2; ++d) {  // the class's choice stays unless the other kernel is >= 2% faster
         const int def = c->auto_path[d][cls];
         const int other = def == MPRESS_PATH_DIRECT ? MPRESS_PATH_BULK : MPRESS_PATH_DIRECT;
         const float t_def = m[def == MPRESS_PATH_BULK][d], t_other = m[other == MPRESS_PATH_BULK][d];
-        c->auto_path[d][cls] = t_other < 0.99f * t_def ? other : def;
+        c->auto_path[d][cls] = t_other < 0.98f * t_def ? other : def;
       }
     if (ms_out)
       for (int pi = 0; pi < 2; ++pi)
