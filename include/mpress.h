@@ -26,6 +26,11 @@
  *   mpress_wait / mpress_query -- completion is signalled with CUDA events,
  *                       so the compute stream overlaps the swap and the host
  *                       never blocks.
+ *   mpress_autotune  -- times the two SM kernels on the context's own links
+ *                       and sets the default path per direction and size.
+ *   Beyond the hot path: the multi-source and
+ *   global planners, the device-stage mapping search, the 1F1B schedule and
+ *   executor, the compaction decision rule, and a pinned host pool as a peer.
  *
  * Conventions
  *   - Every entry point returns int: MPRESS_OK (0) or a negative MPRESS_ERR_*;
