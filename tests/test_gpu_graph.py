@@ -121,6 +121,7 @@ def test_graph_cross_stream_join():
         ctx.finalize()
 
 
+@pytest.mark.filterwarnings("ignore:The CUDA Graph is empty")  # refused calls leave the capture empty
 def test_graph_misuse():
     sizes, o, pl, ctx = _setup(mp.PATH_DIRECT, copies=3)
     try:
