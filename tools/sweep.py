@@ -23,7 +23,7 @@ import paper_conf_hpca_zhouwylbyx23_b200 as mp  # noqa: E402
 from synth import device as synth_dev  # noqa: E402
 from synth import workloads  # noqa: E402
 
-PATHS = {"direct": mp.PATH_DIRECT, "bulk": mp.PATH_BULK, "ce": mp.PATH_CE}
+PATHS = {"direct": mp.PATH_DIRECT, "bulk": mp.PATH_BULK, "ce": mp.PATH_CE, "auto": mp.PATH_AUTO}
 
 
 def setup(sizes, peers_n, copies=1):
