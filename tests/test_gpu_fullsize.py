@@ -180,3 +180,12 @@ def test_sanitizer_multi_piece_ctas(tool):
     out = r.stdout + r.stderr
     assert r.returncode == 0 and "multi-piece ok" in out, (out[-3000:])
     assert ("ERROR SUMMARY: 0 errors" in out) or ("0 hazards displayed (0 errors" in out)
+
+
+@pytest.mark.parametrize("path", [None, mp.PATH_DIRECT], ids=["auto", "direct"])
+def test_stripe_longer_than_4gib(path):
+    """One 6 GiB + 17 B tensor to one peer: a single stripe longer than 2^32
+    bytes (64-bit lengths and offsets through the tables and the kernels'
+    chunk arithmetic), with a ragged tail."""
+    spare = [0, 8 << 30]
+    _sampled_roundtrip(2, 0, spare, [0, 1], [(6 << 30) + 17], seed=4100, path=path)
