@@ -1,0 +1,61 @@
+"""Performance floors on one B200 (loopback peers): generous lower bounds that
+only a gross regression would break -- the measured values are ~1.25x above
+them (profiles/r01/bench.json).  The bench, not these tests, is the
+measurement."""
+import statistics
+
+import pytest
+import torch
+
+import paper_conf_hpca_zhouwylbyx23_b200 as mp
+from synth import device as synth_dev
+from synth import workloads
+
+pytestmark = pytest.mark.gpu
+
+
+def _rate(ctx, pl, src, dst, s, nbytes, reps=10):
+    ts = []
+    for _ in range(reps + 2):
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(s)
+        h = ctx.swap_out(pl, src, stream=s)
+        ctx.swap_in(h, dst, stream=s)
+        e1.record(s)
+        h.free()
+        ts.append((e0, e1))
+    torch.cuda.synchronize()
+    ms = statistics.median(a.elapsed_time(b) for a, b in ts[2:])
+    return 2 * nbytes / ms / 1e6
+
+
+def test_cfg2_micro_batch_round_trip_floor():
+    """One Bert stage-0 micro-batch (47 tensors, 900 MiB) over 3 loopback
+    peers, default path and grid: >= 2500 GB/s of swapped bytes (measured
+    ~3150-3200; roofline 3276 = half the measured HBM copy bandwidth)."""
+    sizes = workloads.cfg2_sizes(1)
+    peers = [1, 2, 3]
+    spare = workloads.spare_vector(4, 0, peers, spare=24 << 30)
+    bw = workloads.bw_vector(4, 0, peers)
+    pl = mp.plan(4, 0, spare, bw, sizes)
+    part = [[0] * 4 for _ in range(4)]
+    part[0] = [u * mp.DEFAULT_GRANULE for u in pl.units]
+    ctx = mp.Context.local(4, 0, [0] * 4, part)
+    try:
+        src = [torch.empty(n, dtype=torch.uint8, device="cuda") for n in sizes]
+        for i, t in enumerate(src):
+            synth_dev.fill(t, 90, i)
+        dst = [torch.empty(n, dtype=torch.uint8, device="cuda") for n in sizes]
+        torch.cuda.synchronize()
+        s = torch.cuda.Stream()
+        ps, pd = mp.pointers(src), mp.pointers(dst)
+        gbs = _rate(ctx, pl, ps, pd, s, sum(sizes))
+        assert all(synth_dev.check(d, 90, i) == 0 for i, d in enumerate(dst))
+        assert gbs >= 2500, "cfg2 round trip %.0f GB/s (floor 2500)" % gbs
+        # the GEMM-concurrent shape (capped, direct 128x4x32 B at 64 CTAs) alone
+        ctx.set_option(mp.OPT_MAX_CTAS, 64)
+        capped = _rate(ctx, pl, ps, pd, s, sum(sizes))
+        assert capped >= 800, "capped round trip %.0f GB/s (floor 800)" % capped
+    finally:
+        ctx.finalize()
