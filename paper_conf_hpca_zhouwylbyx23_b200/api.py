@@ -518,11 +518,13 @@ class Context:
         _check(lib.mpress_get_option(self._h, key, byref(v)))
         return v.value
 
-    def autotune(self, probe_bytes=256 << 20, trials=5, stream=None):
+    def autotune(self, probe_bytes=1 << 30, trials=5, stream=None):
         """mpress_autotune: time the direct and bulk kernels on this
-        context's links and let MPRESS_PATH_AUTO keep the faster per
-        direction (collective for a distributed context).  Returns the
-        chosen paths and the median probe times in ms."""
+        context's links (back-to-back launches over a `probe_bytes` working
+        set) and let MPRESS_PATH_AUTO keep the faster per direction and size
+        class (collective for a distributed context).  Returns the chosen
+        paths (out / in for launches >= AUTO_SMALL_BYTES, out_small /
+        in_small below) and the median ms per launch of every probe."""
         ms = (ctypes.c_float * 8)()
         _check(lib.mpress_autotune(self._h, probe_bytes, trials, _stream(stream, self.device), ms))
         names = [c + "_" + k + "_" + d for c in ("small", "large") for k in ("direct", "bulk") for d in ("out", "in")]
