@@ -63,10 +63,12 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
     ap.add_argument("--gemm-cap", type=int, default=0,
-                    help="swap grid cap (CTAs = SMs touched) while the concurrent GEMM runs; 0 = calibrate: "
-                         "the smallest of --gemm-cap-candidates whose swap rate on this run's links reaches "
-                         "--gemm-target-gbs / 0.85")
-    ap.add_argument("--gemm-cap-candidates", default="64,96,128,148")
+                    help="swap grid cap (CTAs = SMs touched) while the concurrent GEMM runs (AUTO path -> "
+                         "direct shape 7); 0 = calibrate: the first of --gemm-swap-candidates whose swap rate "
+                         "on this run's links reaches --gemm-target-gbs / 0.85")
+    ap.add_argument("--gemm-swap-candidates", default="auto:-1:64,bulk:5:148,auto:-1:96,auto:-1:128,auto:-1:148",
+                    help="path:variant:max_ctas settings for the GEMM-concurrent swap, cheapest for the GEMM "
+                         "first (profiles/r01/sweep_gemm_*)")
     ap.add_argument("--gemm-target-gbs", type=float, default=720.0,
                     help="per-source swap rate the GEMM-concurrent swap should sustain (BJ:5: 80%% of 900)")
     ap.add_argument("--no-gemm", action="store_true")
@@ -513,10 +515,11 @@ def main():
 
     e2e = leg(run_e2e, args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap_stream, n, dist)
     cap_cal = None
+    args.gemm_swap = "auto:-1:%d" % (args.gemm_cap if args.gemm_cap > 0 else 64)
     if not args.no_gemm and args.gemm_cap <= 0:
         cap_cal = calibrate_gemm_cap(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap_stream, n,
                                      dist)
-        args.gemm_cap = cap_cal["chosen"]
+        args.gemm_swap = cap_cal["chosen"]
     gemm = None if args.no_gemm else leg(gemm_interference, args, ctx, mp, world, source, per_copy, bw,
                                          sizes, src, dst, swap_stream, n, dist)
     gemm_ce = None if (args.no_gemm or args.no_gemm_ce) else leg(
@@ -716,29 +719,51 @@ class _Local:
             return None
 
 
+def set_gemm_swap(ctx, mp, spec):
+    """Apply a GEMM-concurrent swap setting "path:variant:max_ctas" (path
+    auto/direct/bulk; auto with a cap <= the SM count runs direct shape 7);
+    returns the previous (path, variant, max_ctas) for restore_swap."""
+    prev = (ctx.get_option(mp.OPT_PATH), ctx.get_option(mp.OPT_VARIANT), ctx.get_option(mp.OPT_MAX_CTAS))
+    name, var, cap = spec.split(":")
+    paths = {"auto": mp.PATH_AUTO, "direct": mp.PATH_DIRECT, "bulk": mp.PATH_BULK, "ce": mp.PATH_CE}
+    ctx.set_option(mp.OPT_PATH, paths[name])
+    if name != "auto":
+        ctx.set_option(mp.OPT_VARIANT, int(var))
+    ctx.set_option(mp.OPT_MAX_CTAS, int(cap))
+    return prev
+
+
+def restore_swap(ctx, mp, prev):
+    ctx.set_option(mp.OPT_PATH, prev[0])
+    if prev[0] != mp.PATH_AUTO:
+        ctx.set_option(mp.OPT_VARIANT, prev[1])
+    ctx.set_option(mp.OPT_MAX_CTAS, prev[2])
+
+
 def calibrate_gemm_cap(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap, n, dist):
-    """Grid cap of the GEMM-concurrent swap, measured on this run's links
-    (HBM loopback at N = 1, NVLink at N > 1, where every remote access pays
-    ~2x the latency, so the same cap keeps fewer bytes in flight per µs):
-    for each candidate cap the capped swap (AUTO -> direct shape 7) runs
-    alone, out + in, on every rank at once; the smallest cap whose slowest
-    rank reaches --gemm-target-gbs / 0.85 (headroom for the GEMM's
-    contention) is chosen, else the largest candidate.  Collective: every rank
+    """The GEMM-concurrent swap setting, measured on this run's links (HBM
+    loopback at N = 1, NVLink at N > 1, where every remote access pays ~2x
+    the latency, so a setting keeps fewer bytes in flight per µs): every
+    candidate of --gemm-swap-candidates (ordered cheapest for the GEMM first:
+    128-thread direct CTAs at 64, small-smem bulk CTAs on every SM, then
+    more direct CTAs) runs alone, out + in, on every rank at once; the first
+    whose slowest rank reaches --gemm-target-gbs / 0.85 (headroom for the
+    GEMM's contention) is chosen, else the fastest.  Collective: every rank
     reaches every barrier and reduction even if its own work fails."""
     import torch
-    caps = [int(c) for c in args.gemm_cap_candidates.split(",") if c.strip()]
-    old = ctx.get_option(mp.OPT_MAX_CTAS)
+    specs = [c.strip() for c in args.gemm_swap_candidates.split(",") if c.strip()]
     pl = mp.plan(world, source, per_copy, bw, sizes)
     nbytes = sum(sizes)
     reps = 3
     table, err = {}, None
-    for cap in caps:
+    for spec in specs:
         rate = 0.0
         if n > 1:
             dist.barrier()
         if err is None:
+            prev = None
             try:
-                ctx.set_option(mp.OPT_MAX_CTAS, cap)
+                prev = set_gemm_swap(ctx, mp, spec)
                 h = ctx.swap_out(pl, src[0], stream=swap)     # warm-up
                 ctx.swap_in(h, dst[0], stream=swap)
                 h.free()
@@ -755,19 +780,24 @@ def calibrate_gemm_cap(args, ctx, mp, world, source, per_copy, bw, sizes, src, d
                 rate = 2 * reps * nbytes / e0.elapsed_time(e1) / 1e6
             except Exception as exc:  # pragma: no cover - reported in the line
                 err = "%s: %s" % (type(exc).__name__, exc)
+            finally:
+                if prev is not None:
+                    try:
+                        restore_swap(ctx, mp, prev)
+                    except Exception:  # pragma: no cover
+                        pass
         t = torch.tensor([rate if err is None else 0.0], dtype=torch.float64)
         if n > 1:
             dist.all_reduce(t, op=dist.ReduceOp.MIN)
-        table[cap] = float(t.item())
-    try:
-        ctx.set_option(mp.OPT_MAX_CTAS, old)
-    except Exception:  # pragma: no cover
-        pass
+        table[spec] = float(t.item())
     need = args.gemm_target_gbs / 0.85
-    ok = [c for c in caps if table[c] >= need]
-    chosen = (min(ok) if ok else max(caps)) if err is None else 64
+    ok = [c for c in specs if table[c] >= need]
+    if err is not None:
+        chosen = "auto:-1:64"
+    else:
+        chosen = ok[0] if ok else max(specs, key=lambda c: table[c])
     return {"chosen": chosen, "target_gbs": args.gemm_target_gbs, "needed_alone_gbs": need,
-            "alone_gbs_by_cap_min_over_ranks": {str(c): table[c] for c in caps}, "error": err}
+            "alone_gbs_min_over_ranks": table, "error": err}
 
 
 def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap, n, dist, ce=False):
@@ -801,11 +831,7 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
         st["b"] = torch.randn(K, N, dtype=torch.bfloat16, device="cuda")
         st["c"] = torch.empty(M, N, dtype=torch.bfloat16, device="cuda")
         st["pl"] = mp.plan(world, source, per_copy, bw, sizes)
-        st["old_cap"] = ctx.get_option(mp.OPT_MAX_CTAS)
-        ctx.set_option(mp.OPT_MAX_CTAS, args.gemm_cap)
-        if ce:
-            st["old_path"] = ctx.get_option(mp.OPT_PATH)
-            ctx.set_option(mp.OPT_PATH, mp.PATH_CE)
+        st["prev"] = set_gemm_swap(ctx, mp, "ce:0:0" if ce else args.gemm_swap)
         # swap time at this cap, to size the loop that must cover the GEMM window
         e0 = torch.cuda.Event(enable_timing=True)
         e1 = torch.cuda.Event(enable_timing=True)
@@ -864,10 +890,8 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
     for _ in range(8):
         L(round_)
     st["ran"] = ctx.get_option(mp.OPT_LAST_PATH)
-    if "old_cap" in st:
-        L(ctx.set_option, mp.OPT_MAX_CTAS, st["old_cap"])
-    if "old_path" in st:
-        L(ctx.set_option, mp.OPT_PATH, st["old_path"])
+    if "prev" in st:
+        L(restore_swap, ctx, mp, st["prev"])
     t = torch.tensor([statistics.median(alone) if alone else float("nan"),
                       statistics.median(during) if during else float("nan"),
                       1.0 if L.err is not None else 0.0,
@@ -888,7 +912,9 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
             "rounds": len(ratios),
             "slowdown_per_round": [r - 1 for r in ratios],
             "swap_path": {mp.PATH_DIRECT: "direct", mp.PATH_BULK: "bulk", mp.PATH_CE: "ce"}.get(
-                st.get("ran"), args.path), "swap_max_ctas": None if ce else args.gemm_cap,
+                st.get("ran"), args.path),
+            "swap_setting": "ce:0:0" if ce else args.gemm_swap,
+            "swap_max_ctas": None if ce else int(args.gemm_swap.split(":")[2]),
             # MPRESS_OPT_PDL 1 (default) launches a capped grid without PDL
             "swap_pdl_mode": ctx.get_option(mp.OPT_PDL),
             "swap_gbs_during": statistics.median(swap_gbs),
@@ -947,9 +973,7 @@ def cfg5_leg(args, mp, rank, n, device, dist, ce=False):
                 st["pl"] = mp.plan(n, rank, rem, bwm[rank], sizes)
             for p in range(n):
                 rem[p] -= part[s][p]
-        ctx.set_option(mp.OPT_MAX_CTAS, args.gemm_cap)
-        if ce:
-            ctx.set_option(mp.OPT_PATH, mp.PATH_CE)
+        set_gemm_swap(ctx, mp, "ce:0:0" if ce else args.gemm_swap)
         st["a"] = torch.randn(M, M, dtype=torch.bfloat16, device="cuda")
         st["b"] = torch.randn(M, M, dtype=torch.bfloat16, device="cuda")
         st["c"] = torch.empty(M, M, dtype=torch.bfloat16, device="cuda")
@@ -1039,8 +1063,7 @@ def cfg5_leg(args, mp, rank, n, device, dist, ce=False):
     return {"config": "cfg5 imbalanced all-stage swap: sources %s -> importers %s, source s swaps %s micro-batch "
                       "sets (900 MiB each, one plan), bf16 %dx%dx%d GEMMs on every rank" %
                       (sources, peers, [H - s for s in sources], M, M, M),
-            "swap_path": "ce" if ce else "auto (capped -> direct)",
-            "swap_max_ctas": None if ce else args.gemm_cap,
+            "swap_setting": "ce:0:0" if ce else args.gemm_swap,
             "per_source_gbs": [float(row[s, 2]) for s in sources],
             "per_source_bytes": [sum(workloads.cfg2_sizes(H - s)) for s in sources],
             "gemm_alone_ms": [float(row[r, 0]) for r in range(n)],
