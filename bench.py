@@ -393,38 +393,37 @@ def main():
     timing = {"out": [], "in": []}
     launches = [0]
 
-    # Per-kernel timing events are recorded around ONE swap-out and ONE
-    # swap-in per step (micro-batch k % mb in step k): a timing event between
-    # two kernels serialises them, which would switch off the programmatic
-    # dependent launch (PDL) overlap of every other launch boundary.
+    # Per-kernel timing: timing events bracket the RUN of mb swap-out
+    # launches and the run of mb swap-in launches of every timed step, and the
+    # average launch duration is the run's time / mb.  A timing event between
+    # two kernels serialises them and switches off their programmatic
+    # dependent launch (PDL) overlap, so none is recorded inside a run: the
+    # runs are timed as the step runs them (an earlier version bracketed one
+    # launch per direction, which cost that launch its PDL overlap and
+    # understated the kernel's in-step speed by ~1%).
     ran_dir = {}   # path each direction ran (MPRESS_OPT_LAST_PATH), from the first warm-up step
 
     def step(record=False, k=0, probe_path=False):
         pl = mp.plan(world, source, per_copy, bw, sizes)              # a1
         hs = []
-        tm = k % mb
+        if record:
+            e0 = torch.cuda.Event(enable_timing=True); e0.record(swap_stream)
         for m in range(mb):                                            # a3 + a4
-            rec = record and m == tm
-            if rec:
-                e0 = torch.cuda.Event(enable_timing=True); e0.record(swap_stream)
             hs.append(ctx.swap_out(pl, src[m], stream=swap_stream))
             launches[0] += ctx.last_launches
             if probe_path and m == 0:
                 ran_dir["out"] = ctx.get_option(mp.OPT_LAST_PATH)
-            if rec:
-                e1 = torch.cuda.Event(enable_timing=True); e1.record(swap_stream)
-                timing["out"].append((e0, e1))
+        if record:
+            e1 = torch.cuda.Event(enable_timing=True); e1.record(swap_stream)
         for m in range(mb):                                            # a5
-            rec = record and m == tm
-            if rec:
-                e0 = torch.cuda.Event(enable_timing=True); e0.record(swap_stream)
             ctx.swap_in(hs[m], dst[m], stream=swap_stream)
             launches[0] += ctx.last_launches
             if probe_path and m == 0:
                 ran_dir["in"] = ctx.get_option(mp.OPT_LAST_PATH)
-            if rec:
-                e1 = torch.cuda.Event(enable_timing=True); e1.record(swap_stream)
-                timing["in"].append((e0, e1))
+        if record:
+            e2 = torch.cuda.Event(enable_timing=True); e2.record(swap_stream)
+            timing["out"].append((e0, e1))
+            timing["in"].append((e1, e2))
         ctx.wait(hs[-1], compute)                                      # a6
         for h in hs:
             h.free()
@@ -472,8 +471,8 @@ def main():
 
     names = {mp.PATH_DIRECT: "direct", mp.PATH_BULK: "bulk", mp.PATH_CE: "ce"}
     ran_by_dir = {k: names.get(v, "?") for k, v in ran_dir.items()}
-    # per-kernel durations (each swap call here is exactly one kernel launch)
-    dur = {k: [a.elapsed_time(b) for a, b in v] for k, v in timing.items()}
+    # per-launch durations: each timed run is mb launches (one per swap call)
+    dur = {k: [a.elapsed_time(b) / mb for a, b in v] for k, v in timing.items()}
     tot = {k: sum(v) for k, v in dur.items()}
     dom = max(tot, key=tot.get)
     ran = ran_by_dir.get(dom, "?")   # the dominant kernel's path
@@ -491,9 +490,9 @@ def main():
                 # sampled launches: average kernel time x launches per step / step time
                 "share_of_step": (statistics.mean(dur["out"]) + statistics.mean(dur["in"])) * mb / ms_step
                 if ms_step > 0 else None,
-                "timed_launches": "1 swap-out + 1 swap-in per step (micro-batch k mod %d in step k); a "
-                                  "bracketed launch loses its PDL overlap, so its mean can exceed an "
-                                  "unbracketed launch's and share_of_step can exceed 1" % mb}
+                "timed_launches": "every timed step: the run of %d swap-out launches and the run of %d "
+                                  "swap-in launches, each bracketed by CUDA events on the swap stream; "
+                                  "avg_launch_ms = run time / %d" % (mb, mb, mb)}
     else:
         algo_bytes = bytes_per_mb           # bytes over NVLink per launch (one direction)
         achieved = algo_bytes / (avg_ms / 1e3) / 1e9
