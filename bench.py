@@ -831,7 +831,14 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
         st["c"] = torch.empty(M, N, dtype=torch.bfloat16, device="cuda")
         st["pl"] = mp.plan(world, source, per_copy, bw, sizes)
         st["prev"] = set_gemm_swap(ctx, mp, "ce:0:0" if ce else args.gemm_swap)
-        # swap time at this cap, to size the loop that must cover the GEMM window
+        # swap time at this setting, to size the loop that must cover the GEMM
+        # window; one untimed pair first (the copy-engine path creates its
+        # side streams on first use, which once inflated the estimate so much
+        # that the loop ended before the counted GEMMs did)
+        h = ctx.swap_out(st["pl"], src[0], stream=swap)
+        ctx.swap_in(h, dst[0], stream=swap)
+        h.free()
+        torch.cuda.synchronize()
         e0 = torch.cuda.Event(enable_timing=True)
         e1 = torch.cuda.Event(enable_timing=True)
         e0.record(swap)
@@ -858,7 +865,9 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
         a_r = [x.elapsed_time(y) for x, y in evs[4:]]
         alone.extend(a_r)
         gemm_ms = statistics.median(alone)
-        n_swap = int(2.0 * G * gemm_ms / st["per_swap_ms"]) + 2
+        # cover the GEMM run twice over (3x for the copy engines, whose
+        # host-side issue rate is the slower one)
+        n_swap = int((3.0 if ce else 2.0) * G * gemm_ms / st["per_swap_ms"]) + 2
         s0 = torch.cuda.Event(enable_timing=True)
         s1 = torch.cuda.Event(enable_timing=True)
         # The SM paths enqueue in ~10 us per call, far ahead of the GPU, so
@@ -880,13 +889,17 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
         win = s0.elapsed_time(s1)
         d_r = [x.elapsed_time(y) for x, y in evs[4:]
                if s0.elapsed_time(x) >= 0 and s0.elapsed_time(y) <= win]
+        if os.environ.get("BENCH_DEBUG"):
+            print("gemm round ce=%s n_swap=%d win=%.2f ms gemm starts %s ends %s" % (
+                ce, n_swap, win, [round(s0.elapsed_time(x), 2) for x, _ in evs[::6]],
+                [round(s0.elapsed_time(y), 2) for _, y in evs[::6]]), file=sys.stderr)
         during.extend(d_r)
         if d_r:
             ratios.append(statistics.median(d_r) / statistics.median(a_r))
         swap_gbs.append(2 * n_swap * sum(sizes) / win / 1e6)
 
     L(setup)
-    for _ in range(8):
+    for _ in range(12):
         L(round_)
     st["ran"] = ctx.get_option(mp.OPT_LAST_PATH)
     if "prev" in st:
@@ -981,6 +994,10 @@ def cfg5_leg(args, mp, rank, n, device, dist, ce=False):
             st["dst"] = [torch.empty(x, dtype=torch.uint8, device="cuda") for x in sizes]
             for i, t in enumerate(st["src"]):
                 synth_dev.fill(t, 5000 + rank, i)
+            h = ctx.swap_out(st["pl"], st["src"], stream=swap)   # untimed first pair (see gemm_interference)
+            ctx.swap_in(h, st["dst"], stream=swap)
+            h.free()
+            torch.cuda.synchronize()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(swap)
             h = ctx.swap_out(st["pl"], st["src"], stream=swap)
@@ -1017,7 +1034,7 @@ def cfg5_leg(args, mp, rank, n, device, dist, ce=False):
         s0 = s1 = None
         evs = gemms() if ce else None   # copy engines: GEMMs first (see gemm_interference)
         if is_src:
-            n_swap = int(2.0 * G * statistics.median(alone) / st["per_swap_ms"]) + 2
+            n_swap = int((3.0 if ce else 2.0) * G * statistics.median(alone) / st["per_swap_ms"]) + 2
             s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             s0.record(swap)
             for _ in range(n_swap):
