@@ -1,0 +1,50 @@
+"""The committed bench line (profiles/r01/bench.json, written by bench.py on
+a B200) satisfies the driver's contract: strict JSON, the required keys and
+types, the roofline / cpu_baseline / e2e / clocks objects, and internal
+consistency (value from ms_per_step, roofline frac = achieved / peak)."""
+import json
+import math
+import os
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _line():
+    with open(os.path.join(ROOT, "profiles", "r01", "bench.json")) as f:
+        text = f.read().strip().splitlines()[-1]
+
+    def bad(c):
+        raise ValueError("non-finite constant %s in the bench line" % c)
+    return json.loads(text, parse_constant=bad)
+
+
+def test_required_keys_and_types():
+    d = _line()
+    for k, t in (("metric", str), ("value", float), ("unit", str), ("n_gpus", int), ("steps", int),
+                 ("warmup", int), ("ms_per_step", float), ("higher_is_better", bool), ("scaling", str),
+                 ("dtype", str), ("data", str), ("config", dict), ("roofline", dict),
+                 ("cpu_baseline", dict), ("e2e", dict), ("gpu_launches", int), ("clocks", dict)):
+        assert isinstance(d[k], t), k
+    assert d["warmup"] >= 3 and d["steps"] >= 1
+    assert "workload" in d["config"] and "l2" in d["config"]
+    assert d["vs_baseline"] is None          # no published number for this metric
+    assert d["gpu_launches"] > 0
+
+
+def test_internal_consistency():
+    d = _line()
+    r = d["roofline"]
+    assert r["bound"] in ("hbm", "nvlink", "tensor", "alu")
+    assert math.isclose(r["frac"], r["achieved"] / r["peak"], rel_tol=1e-9)
+    assert 0 < r["frac"] <= 1.05
+    assert r["traffic"] is None or r["traffic"] > 0
+    # value = swapped bytes (out + in) of all micro-batches per step / step time
+    per_step = 2 * d["config"]["micro_batch_bytes"] * d["config"]["micro_batches"] * d["n_gpus"]
+    assert math.isclose(d["value"], per_step / (d["ms_per_step"] / 1e3) / 1e9, rel_tol=1e-6)
+    c = d["cpu_baseline"]
+    assert c["kind"] == "oracle" and c["cores"] >= 1 and c["value"] > 0
+    e = d["e2e"]
+    assert e["h2d_bytes_per_step"] > 0 and e["d2h_bytes_per_step"] > 0 and e["value"] > 0
+    assert d["clocks"]["sm_mhz"] > 0
+    bad = {"hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown"}
+    assert not bad & set(d["clocks"]["reasons"])
