@@ -2,6 +2,7 @@
 waits, queries and frees across two streams, with a partition that only
 holds a few handles at once (slices are reused under fences, R21/R22) and a
 mix of kernel paths.  Every restored tensor must equal the generator."""
+import os
 import random
 
 import pytest
@@ -13,11 +14,20 @@ from synth import device as synth_dev
 pytestmark = pytest.mark.gpu
 
 
-@pytest.mark.parametrize("seed", [1, 2, 3])
+# MPRESS_FUZZ_EXTRA=N adds N more seeds (a soak run; the default suite runs 3)
+SEEDS = [1, 2, 3] + list(range(1000, 1000 + int(os.environ.get("MPRESS_FUZZ_EXTRA", "0"))))
+
+
+@pytest.mark.parametrize("seed", SEEDS)
 def test_random_interleavings(seed):
     rng = random.Random(seed)
     world = 4
-    sizes = [rng.randint(1, 3 << 20) for _ in range(5)]
+    # every third seed: 140 small tensors, so launches exceed 128 descriptors
+    # and read device-resident tables (the staging/device ring) mid-interleaving
+    if seed % 3 == 0:
+        sizes = [rng.randint(1, 64 << 10) for _ in range(140)]
+    else:
+        sizes = [rng.randint(1, 3 << 20) for _ in range(5)]
     spare = [0, 1 << 30, 1 << 30, 1 << 30]
     bw = [0, 1, 2, 1]
     pl = mp.plan(world, 0, spare, bw, sizes, 4096)
@@ -33,8 +43,10 @@ def test_random_interleavings(seed):
             op = rng.random()
             if op < 0.45:
                 if step % 17 == 0:
-                    ctx.set_option(mp.OPT_PATH, rng.choice([mp.PATH_DIRECT, mp.PATH_BULK, mp.PATH_CE]))
+                    ctx.set_option(mp.OPT_PATH, rng.choice([mp.PATH_DIRECT, mp.PATH_BULK, mp.PATH_CE,
+                                                            mp.PATH_AUTO]))
                     ctx.set_option(mp.OPT_MAX_CTAS, rng.choice([0, 1, 7, 64]))
+                    ctx.set_option(mp.OPT_PDL, rng.choice([0, 1, 2]))
                 src = [torch.empty(n, dtype=torch.uint8, device="cuda") for n in sizes]
                 for i, t in enumerate(src):
                     synth_dev.fill(t, next_seed, i)
