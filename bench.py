@@ -373,11 +373,14 @@ def main():
     if path == mp.PATH_AUTO and not args.no_autotune:
         # which SM kernel an uncapped AUTO swap runs on THIS run's links
         # (loopback HBM at N=1, NVLink at N>1), measured before the timed steps
+        t_at = time.perf_counter()
         res = ctx.autotune(probe_bytes=AUTOTUNE_PROBE, trials=5)
+        t_at = (time.perf_counter() - t_at) * 1e3
         nm = {mp.PATH_DIRECT: "direct", mp.PATH_BULK: "bulk"}
         autotune = {"out": nm[res["out"]], "in": nm[res["in"]], "out_small": nm[res["out_small"]],
                     "in_small": nm[res["in_small"]], "small_below_bytes": mp.AUTO_SMALL_BYTES,
-                    "probe_bytes": AUTOTUNE_PROBE, "trials": 5, "median_ms_per_launch": res["ms"]}
+                    "probe_bytes": AUTOTUNE_PROBE, "trials": 5, "median_ms_per_launch": res["ms"],
+                    "wall_ms": t_at}
 
     seed0 = 2000 + 100 * rank
     src = [[torch.empty(s, dtype=torch.uint8, device="cuda") for s in sizes] for _ in range(mb)]
