@@ -424,9 +424,8 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
  * per SM),
  * 5 = 2 x 8 KiB, 6 = 3 x 4 KiB (one per SM; small enough to share an SM
  * with a GEMM CTA);
- * copy engines: 0 = cudaMemcpyAsync per stripe on one side stream per peer,
- * 1 = the whole swap as one cudaMemcpyBatchAsync on the swap stream (not on
- * the legacy NULL stream);
+ * copy engines: 0 = cudaMemcpyAsync per stripe on one side stream per peer
+ * (the only copy-engine variant);
  * MPRESS_VARIANT_AUTO (-1, default) = direct 7 when the grid is capped at
  * <= one CTA per SM (small CTAs co-reside with a GEMM), else 5; bulk 3; copy
  * engines 0.

@@ -17,7 +17,6 @@
 // the fences of its slices, fences are reaped oldest-first, and descriptor
 // buffers are reused.
 #include <algorithm>
-#include <cstring>
 
 #include "ctx.h"
 #include "hostprof.h"
@@ -168,9 +167,9 @@ int run_copy(mpress_ctx_s* c, int dir, const std::vector<CopyDesc>& d,
                        c->pdl, stream, &c->last_launches, graph ? nullptr : c->ring);
   }
 
-  // Copy-engine comparator, variant 1: the whole swap as one
-  // cudaMemcpyBatchAsync on `stream` (CUDA 12.8+); the driver spreads the
-  // copies over the copy engines.  Stream-ordered source access.
+  // Copy-engine comparator (the prior-art mechanism):
+  // one cudaMemcpyAsync per stripe, one side stream per peer so the engines of
+  // different peers overlap; fork/join by events.
   if (c->ce_streams.empty()) {
     c->ce_streams.assign(c->world, nullptr);
     for (int p = 0; p < c->world; ++p) {
@@ -178,46 +177,6 @@ int run_copy(mpress_ctx_s* c, int dir, const std::vector<CopyDesc>& d,
       if (e != cudaSuccess) return cuda_fail(e, "cudaStreamCreate (copy-engine path)");
     }
   }
-  if (c->variant == 1) {
-    const size_t n = d.size();
-    if (n == 0) return MPRESS_OK;
-    // The batch call rejects the legacy NULL stream: there, run it on a side
-    // stream (the source's slot, which no stripe uses) forked and joined by
-    // events.
-    const bool legacy = stream == nullptr || stream == cudaStreamLegacy;
-    cudaStream_t bs = legacy ? c->ce_streams[c->source] : stream;
-    EvRef fork, join;
-    if (legacy) {
-      fork = take_event(c);
-      join = take_event(c);
-      if (!fork || !join) return fail(MPRESS_ERR_CUDA, "cudaEventCreate failed");
-      cudaEventRecord(fork.get(), stream);
-      cudaStreamWaitEvent(bs, fork.get(), 0);
-    }
-    std::vector<void*> dsts(n), srcs(n);
-    std::vector<size_t> lens(n);
-    for (size_t i = 0; i < n; ++i) {
-      dsts[i] = d[i].dst;
-      srcs[i] = const_cast<void*>(d[i].src);
-      lens[i] = d[i].len;
-    }
-    cudaMemcpyAttributes attr;
-    std::memset(&attr, 0, sizeof(attr));
-    attr.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
-    size_t attr_idx = 0, fail_idx = SIZE_MAX;
-    const cudaError_t e = cudaMemcpyBatchAsync(dsts.data(), srcs.data(), lens.data(), n, &attr, &attr_idx, 1,
-                                               &fail_idx, bs);
-    if (legacy) {
-      cudaEventRecord(join.get(), bs);
-      cudaStreamWaitEvent(stream, join.get(), 0);
-    }
-    if (e != cudaSuccess) return cuda_fail(e, "cudaMemcpyBatchAsync (copy-engine path)");
-    return MPRESS_OK;
-  }
-
-  // Copy-engine comparator, variant 0 (default): cudaMemcpyAsync per stripe,
-  // one side stream per peer so the engines of different peers overlap;
-  // fork/join by events.
   EvRef fork = take_event(c);
   if (!fork) return fail(MPRESS_ERR_CUDA, "cudaEventCreate failed");
   cudaEventRecord(fork.get(), stream);

@@ -66,7 +66,7 @@ def paths():
     nbytes = sum(sizes)
     ctx, pl, src, dst = setup(sizes, 3)
     s = torch.cuda.Stream()
-    nvar = {"direct": 10, "bulk": 7, "ce": 2, "auto": 0}  # plus -1 = auto
+    nvar = {"direct": 10, "bulk": 7, "ce": 1, "auto": 0}  # plus -1 = auto
     only = os.environ.get("SWEEP_PATHS")        # e.g. "direct"
     var_sel = os.environ.get("SWEEP_VARIANTS")  # e.g. "0,5,6,8"
     cap_sel = os.environ.get("SWEEP_CAPS")      # e.g. "0,148,296"
@@ -100,10 +100,8 @@ def sizes_sweep():
     for peers_n in (1, 3, 7):
         for size in workloads.cfg4_sizes():
             ctx, pl, src, dst = setup([size], peers_n, copies=2)
-            for name in os.environ.get("SWEEP_SIZE_PATHS", "direct,bulk,ce,ce_batch").split(","):
-                ctx.set_option(mp.OPT_PATH, PATHS[name.split("_")[0]])
-                if name == "ce_batch":
-                    ctx.set_option(mp.OPT_VARIANT, 1)   # one cudaMemcpyBatchAsync
+            for name in os.environ.get("SWEEP_SIZE_PATHS", "direct,bulk,ce").split(","):
+                ctx.set_option(mp.OPT_PATH, PATHS[name])
                 reps = 20 if size < (256 << 20) else 5
                 to, ti = time_swaps(ctx, pl, src, dst, reps, s)
                 # back to back: R swap pairs enqueued while the GPU is busy, so
@@ -123,25 +121,23 @@ def sizes_sweep():
                 torch.cuda.synchronize()
                 warm.free()
                 pair_us = e0.elapsed_time(e1) * 1e3 / R
-                graph_us = None
-                if name != "ce_batch":
-                    # the pair captured once into a CUDA graph, one replay timed
-                    g = torch.cuda.CUDAGraph()
-                    with torch.cuda.graph(g, stream=s):
-                        gh = ctx.swap_out(pl, src)
-                        ctx.swap_in(gh, dst)
-                    ts = []
-                    with torch.cuda.stream(s):
-                        for r in range(12):
-                            e0.record()
-                            g.replay()
-                            e1.record()
-                            torch.cuda.synchronize()
-                            if r >= 2:
-                                ts.append(e0.elapsed_time(e1) * 1e3)
-                    del g
-                    gh.free()
-                    graph_us = statistics.median(ts)
+                # the pair captured once into a CUDA graph, one replay timed
+                g = torch.cuda.CUDAGraph()
+                with torch.cuda.graph(g, stream=s):
+                    gh = ctx.swap_out(pl, src)
+                    ctx.swap_in(gh, dst)
+                ts = []
+                with torch.cuda.stream(s):
+                    for r in range(12):
+                        e0.record()
+                        g.replay()
+                        e1.record()
+                        torch.cuda.synchronize()
+                        if r >= 2:
+                            ts.append(e0.elapsed_time(e1) * 1e3)
+                del g
+                gh.free()
+                graph_us = statistics.median(ts)
                 print(json.dumps({"sweep": "sizes", "peers": peers_n, "bytes": size, "path": name,
                                   "out_gbs": size / to / 1e6, "in_gbs": size / ti / 1e6,
                                   "out_us": to * 1e3, "in_us": ti * 1e3,
