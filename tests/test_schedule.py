@@ -27,6 +27,20 @@ def test_golden_two_stage_timeline():
     assert mp.schedule_1f1b(*args, duplex=bool(q["duplex"])) == (g["slots"], g["summary"])
 
 
+@pytest.mark.parametrize("case", range(4))
+def test_golden_slack(case):
+    """The swap-in slack rule (fn.1 P:226, reading R24): hand-derived
+    triggers for slack > 0, the fall-back to F(m) itself when no op qualifies,
+    and the <= boundary; by the oracle and by the library."""
+    g = json.load(open(os.path.join(GOLDEN, "p1_1f1b_slack.json")))["cases"][case]
+    q = g["params"]
+    args = (q["stages"], q["stage"], q["micro_batches"], q["t_fwd_ns"], q["t_bwd_ns"],
+            q["t_out_ns"], q["t_in_ns"])
+    assert P.schedule(*args, duplex=bool(q["duplex"]), slack=q["slack_ns"]) == (g["slots"], g["summary"])
+    assert mp.schedule_1f1b(*args, duplex=bool(q["duplex"]), slack_ns=q["slack_ns"]) == \
+        (g["slots"], g["summary"])
+
+
 @pytest.mark.parametrize("S,M", [(1, 1), (1, 5), (2, 3), (4, 8), (8, 8), (8, 16), (5, 2)])
 def test_1f1b_closed_form_makespan(S, M):
     s, e = P.timeline_noswap(S, M, 7, 13)
