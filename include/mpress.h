@@ -324,6 +324,11 @@ MPRESS_API int mpress_schedule_1f1b(const mpress_1f1b_params* params, mpress_1f1
  *       swap-out stream after the op; then enqueues every swap-in this op
  *       triggers on the swap-in stream, into the buffers given by
  *       mpress_executor_restore_to(x, m, dst) beforehand.
+ * mpress_executor_release(x, m, stream) -- makes `stream` wait until m's
+ *       swap-out has read its activations (between after(F(m)) and
+ *       before(B(m))).  Freeing the activations is the point of the swap
+ *       (memory saving operators); a caching allocator on `stream`
+ *       may hand their memory to the next op only after this call.
  * Enqueue-only.  One executor serves any number of steps.
  * An executor step cannot be captured into a CUDA graph (MPRESS_ERR_STATE
  * while any of its streams is capturing): it recycles stash slices between
@@ -345,6 +350,7 @@ MPRESS_API int mpress_executor_before(mpress_executor_t* x, uint32_t op, void* c
                                       uint32_t* kind, uint32_t* micro_batch);
 MPRESS_API int mpress_executor_after(mpress_executor_t* x, uint32_t op, void* compute_stream,
                                      void* const* activations);
+MPRESS_API int mpress_executor_release(mpress_executor_t* x, uint32_t micro_batch, void* stream);
 MPRESS_API int mpress_executor_free(mpress_executor_t* x);
 
 /* ---- peer-memory layer ----------------------------------------------------- */

@@ -43,7 +43,7 @@ EXPORTED = [
     "mpress_plan_from_units", "mpress_schedule_1f1b", "mpress_map_search",
     "mpress_compaction_plan", "mpress_executor_create", "mpress_executor_ops",
     "mpress_executor_slot", "mpress_executor_restore_to", "mpress_executor_before",
-    "mpress_executor_after", "mpress_executor_free", "mpress_init",
+    "mpress_executor_after", "mpress_executor_release", "mpress_executor_free", "mpress_init",
     "mpress_init_local",
     "mpress_finalize", "mpress_stash_free", "mpress_set_option", "mpress_get_option", "mpress_autotune",
     "mpress_swap_out", "mpress_swap_in", "mpress_wait", "mpress_query", "mpress_handle_state",
@@ -114,6 +114,7 @@ def _load():
         "mpress_executor_restore_to": (c_int, [P, c_uint32, P]),
         "mpress_executor_before": (c_int, [P, c_uint32, P, POINTER(c_uint32), POINTER(c_uint32)]),
         "mpress_executor_after": (c_int, [P, c_uint32, P, P]),
+        "mpress_executor_release": (c_int, [P, c_uint32, P]),
         "mpress_executor_free": (c_int, [P]),
         "mpress_compaction_plan": (c_int, [c_uint32, P, c_uint64, P, P, POINTER(c_uint64),
                                            POINTER(c_uint64)]),
@@ -449,6 +450,11 @@ class Executor:
     def after(self, op, compute=None, activations=None):
         _check(lib.mpress_executor_after(self._h, op, _stream(compute),
                                          None if activations is None else _ptr_array(activations)))
+
+    def release(self, m, stream=None):
+        """mpress_executor_release: `stream` waits until micro-batch m's
+        swap-out has read its activations, so they may be freed on it."""
+        _check(lib.mpress_executor_release(self._h, m, _stream(stream)))
 
     def free(self):
         if self._h is not None:

@@ -150,6 +150,17 @@ extern "C" int mpress_executor_after(mpress_executor_t* x, uint32_t op, void* co
   return MPRESS_OK;
 }
 
+extern "C" int mpress_executor_release(mpress_executor_t* x, uint32_t micro_batch, void* stream) {
+  if (!x || micro_batch >= x->handle.size()) return fail(MPRESS_ERR_ARG, "mpress_executor_release: bad argument");
+  mpress_handle_t* h = x->handle[micro_batch];
+  if (!h || !h->out_done)
+    return fail(MPRESS_ERR_STATE, "mpress_executor_release: micro-batch %u is not swapped out", micro_batch);
+  DeviceGuard g(x->ctx->device);
+  const cudaError_t e = cudaStreamWaitEvent(static_cast<cudaStream_t>(stream), h->out_done.get(), 0);
+  if (e != cudaSuccess) return fail(MPRESS_ERR_CUDA, "mpress_executor_release: %s", cudaGetErrorString(e));
+  return MPRESS_OK;
+}
+
 extern "C" int mpress_executor_slot(const mpress_executor_t* x, uint32_t micro_batch, mpress_1f1b_slot* slot) {
   if (!x || !slot || micro_batch >= x->slots.size())
     return fail(MPRESS_ERR_ARG, "mpress_executor_slot: bad argument");

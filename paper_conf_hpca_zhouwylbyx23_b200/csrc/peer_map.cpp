@@ -494,6 +494,7 @@ extern "C" int mpress_set_option(mpress_ctx_t* c, int key, int64_t value) {
 
 extern "C" int mpress_get_option(const mpress_ctx_t* c, int key, int64_t* value) {
   if (!c || !value) return fail(MPRESS_ERR_ARG, "mpress_get_option: null argument");
+  std::lock_guard<std::mutex> lk(const_cast<mpress_ctx_t*>(c)->mu);  // set_option/autotune/run_copy write these
   switch (key) {
     case MPRESS_OPT_PATH: *value = c->path; return MPRESS_OK;
     case MPRESS_OPT_MAX_CTAS: *value = c->max_ctas; return MPRESS_OK;

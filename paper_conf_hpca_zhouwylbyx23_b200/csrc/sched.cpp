@@ -505,6 +505,10 @@ extern "C" int mpress_autotune(mpress_ctx_t* c, uint64_t probe_bytes, int trials
       for (auto& kv : c->parts[p].free) best = std::max(best, kv.second);
       len[p] = std::min(share, best / MPRESS_ALIGN * MPRESS_ALIGN);
       if (len[p] == 0 || !alloc_slice(&c->parts[p], len[p], &off[p])) { len[p] = 0; continue; }
+      // A freed IN_PENDING handle leaves fences whose swap-in may still read
+      // these bytes: the probe writes them only after those swap-ins.
+      for (const Fence& f : c->parts[p].fences)
+        if (f.off < off[p] + len[p] && off[p] < f.off + f.len) cudaStreamWaitEvent(stream, f.ev.get(), 0);
       total += len[p];
     }
   }

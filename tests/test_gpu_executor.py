@@ -92,3 +92,49 @@ def test_executor_refuses_graph_capture():
         ex.free()
     finally:
         ctx.finalize()
+
+
+def test_executor_release_then_reuse():
+    """freeing the activations right after F(m) is the point of the
+    swap.  After mpress_executor_release(m, compute) the caching
+    allocator may hand their memory to the next op on the compute stream; the
+    swap-out stream is held back by a sleep so that, without the release, the
+    overwrite would land before the swap-out read the bytes."""
+    M = 3
+    ctx, pl, sizes = _setup(M)
+    s_out, s_in = torch.cuda.Stream(), torch.cuda.Stream()
+    comp = torch.cuda.current_stream()
+    try:
+        ex = mp.Executor(ctx, pl, 2, 0, M, 10_000, 20_000, 5_000, 5_000, s_out, s_in)
+        dst = [[torch.zeros(n, dtype=torch.uint8, device="cuda") for n in sizes] for _ in range(M)]
+        for m in range(M):
+            ex.restore_to(m, dst[m])
+        for j in range(ex.ops):
+            kind, m = ex.before(j, comp)
+            if kind == "F":
+                act = [torch.empty(n, dtype=torch.uint8, device="cuda") for n in sizes]
+                for i, t in enumerate(act):
+                    synth_dev.fill(t, 900 + m, i)
+                with torch.cuda.stream(s_out):
+                    torch.cuda._sleep(20_000_000)      # ~10 ms: the swap-out starts late
+                ex.after(j, comp, act)
+                ex.release(m, comp)
+                ptrs = {t.data_ptr() for t in act}
+                del act                                  # freed on the compute stream
+                reuse = [torch.empty(n, dtype=torch.uint8, device="cuda") for n in sizes]
+                for t in reuse:
+                    t.fill_(0xA5)                        # the next op overwrites the memory
+                assert ptrs & {t.data_ptr() for t in reuse}, "allocator did not reuse the block"
+                del reuse
+            else:
+                ex.after(j, comp, None)
+        with pytest.raises(mp.MPressError) as ei:        # every handle is gone after B(m)
+            ex.release(0, comp)
+        assert ei.value.code == mp.ERR_STATE
+        torch.cuda.synchronize()
+        for m in range(M):
+            for i, t in enumerate(dst[m]):
+                assert synth_dev.check(t, 900 + m, i) == 0, (m, i)
+        ex.free()
+    finally:
+        ctx.finalize()
