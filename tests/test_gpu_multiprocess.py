@@ -187,12 +187,23 @@ def test_bench_torchrun_two_ranks_one_gpu():
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
            "--master-addr=127.0.0.1", "--master-port=%d" % _free_port(), "bench.py", "--gpus", "2",
-           "--steps", "3", "--warmup", "1", "--micro-batches", "2", "--e2e-steps", "1", "--no-gemm"]
+           "--steps", "3", "--warmup", "1", "--micro-batches", "2", "--e2e-steps", "1", "--no-gemm",
+           "--ss-sizes", "4096,1048576,67108864"]
     r = subprocess.run(cmd, cwd=root, capture_output=True, text=True, timeout=600)
     assert r.returncode == 0, r.stderr[-3000:]
     line = json.loads([l for l in r.stdout.splitlines() if l.startswith("{")][-1])
     assert line["n_gpus"] == 2 and line["value"] > 0 and line["roofline"]["bound"] == "nvlink"
     assert "bit-exact" in line["parity"]
+    # value is per source GPU; the whole-job sum is its own key
+    assert line["value"] == line["per_rank_gbs"] and abs(line["all_ranks_gbs"] - 2 * line["value"]) < 1e-6
+    # config 4 single source: P = 1 peer at N = 2, three sizes x three paths, out and in
+    ss = line["single_source"]
+    assert ss["error"] is None and ss["all_bit_exact"], ss
+    assert {(r["peers"], r["bytes"], r["path"]) for r in ss["rows"]} == \
+        {(1, b, p) for b in (4096, 1048576, 67108864) for p in ("direct", "bulk", "ce")}
+    assert all(r["out_gbs"] > 0 and r["in_gbs"] > 0 for r in ss["rows"])
+    d = line["duplex"]
+    assert d["bit_exact"] and line["duplex_gbs"] == d["duplex_gbs"] > 0
 
 
 def test_bench_cfg5_leg_two_ranks_one_gpu():
