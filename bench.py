@@ -59,6 +59,8 @@ def parse():
     ap.add_argument("--pdl", type=int, default=1, choices=[0, 1, 2],
                     help="MPRESS_OPT_PDL: 0 never, 1 uncapped grids only (default), 2 always")
     ap.add_argument("--micro-batches", type=int, default=MICRO_BATCHES)
+    ap.add_argument("--split", type=int, default=0, choices=[0, 1],
+                    help="MPRESS_OPT_SPLIT: 0 = contiguous block per CTA (default), 1 = grid stride (round 1)")
     ap.add_argument("--e2e-steps", type=int, default=16)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
@@ -318,6 +320,7 @@ def workload_config(args, n):
     return {"workload": wl, "tensors_per_micro_batch": 47, "micro_batch_bytes": 900 << 20,
             "micro_batches": args.micro_batches, "peers": 3 if n == 1 else n - 1,
             "path": args.path, "variant": args.variant, "max_ctas": args.max_ctas, "pdl": 0 if args.no_pdl else args.pdl,
+            "split": ["blocked", "strided"][args.split],
             "l2": "inputs %.2f GiB per rank > 126 MB L2: no flush needed" %
                   (args.micro_batches * 900 / 1024)}
 
@@ -387,6 +390,7 @@ def main():
     ctx.set_option(mp.OPT_VARIANT, args.variant)
     ctx.set_option(mp.OPT_MAX_CTAS, args.max_ctas)
     ctx.set_option(mp.OPT_PDL, 0 if args.no_pdl else args.pdl)
+    ctx.set_option(mp.OPT_SPLIT, args.split)
     autotune = None
     if path == mp.PATH_AUTO and not args.no_autotune:
         # which SM kernel an uncapped AUTO swap runs on THIS run's links

@@ -361,7 +361,12 @@ MPRESS_API int mpress_executor_free(mpress_executor_t* x);
 typedef int (*mpress_exchange_fn)(void* user, const void* mine, size_t len, void* all);
 
 /*
- * mpress_init -- collective over `world` processes, one per GPU (torchrun).
+ * mpress_init -- the memory manager's allocation side for the D2D tier
+ * ("the memory manager takes over the memory allocation/deallocation";
+ * it "is responsible for allocating and releasing the GPU/CPU memory
+ * space"): each light-load GPU reserves the spare HBM the plan stripes into
+ * and every source maps its partitions on those peers.
+ * Collective over `world` processes, one per GPU (torchrun).
  *   device     CUDA ordinal this rank runs on
  *   partition  [world*world], identical on all ranks (see
  *              mpress_partition_sequential).  Rank p creates a stash pool of
@@ -380,7 +385,8 @@ MPRESS_API int mpress_init(int device, int world, int rank, const uint64_t* part
                 mpress_ctx_t** out);
 
 /*
- * mpress_init_local -- single-process variant: peer p's pool lives on
+ * mpress_init_local -- single-process variant of mpress_init (same passages,
+ * P:145 / P:236 / P:151): peer p's pool lives on
  * devices[p] and holds only this source's partition (partition[source*world+p]
  * bytes).  With every devices[p] equal it is the 1-GPU "loopback" mode: the
  * peers are disjoint VMM pools of the same GPU, so the whole data path
@@ -395,12 +401,20 @@ MPRESS_API int mpress_init(int device, int world, int rank, const uint64_t* part
 MPRESS_API int mpress_init_local(int world, int source, const int* devices,
                       const uint64_t* partition, mpress_ctx_t** out);
 
-/* Collective for contexts made by mpress_init (barrier, unmap, release).
- * Outstanding handles are freed.  NULL is a no-op. */
+/* mpress_finalize -- the memory manager's release side ("the memory
+ * manager takes over the memory allocation/deallocation"; it is
+ * "responsible for allocating and releasing the GPU/CPU memory space"):
+ * collective for contexts made by mpress_init (barrier, unmap, release of
+ * the pools); a local context releases at once.  Outstanding handles are
+ * freed (their stashed data is dropped).  NULL is a no-op.
+ * Errors: MPRESS_ERR_SYS (the closing barrier failed), MPRESS_ERR_CUDA. */
 MPRESS_API int mpress_finalize(mpress_ctx_t* ctx);
 
-/* Largest contiguous free extent of this source's partition on each peer
- * [world] -> the spare_bytes argument of mpress_plan for the next batch. */
+/* mpress_stash_free -- the memory manager "monitoring the per-device memory
+ * usage" for the D2D tier: largest contiguous free extent of this
+ * source's partition on each peer, written to free_bytes [world, caller
+ * owned] -> the spare_bytes argument of mpress_plan for the next batch
+ * (reading R21).  Errors: MPRESS_ERR_ARG (NULL argument). */
 MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
 
 /* Tunables.  MPRESS_OPT_PATH: 0 = SM kernel, direct 16/32-B loads/stores;
@@ -423,8 +437,9 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
  * MPRESS_OPT_VARIANT: kernel shape within the path -- direct: 0 = 256
  * threads x 8 vectors (2 CTAs/SM by default), 1 = 512x8, 2 = 256x16,
  * 3 = 1024x4, 4 = 128x8 (16-byte vectors), 5 = 256x4, 6 = 256x8, 7 = 128x4,
- * 8 = 256x4 with L2 evict-first loads, 9 = 128x8 (32-byte vectors, used
- * only when every address is 32-byte aligned, else the 16-byte shape);
+ * 8 = 256x4 with L2 evict-first loads, 9 = 128x8, 10 = 128x16, 11 = 64x16
+ * (32-byte vectors, used only when every address is 32-byte aligned, else
+ * the 16-byte shape);
  * bulk: 0 = 6 slots x 32 KiB, 1 = 12 x 16 KiB, 2 = 3 x 64 KiB (one CTA per
  * SM), 3 = 3 x 32 KiB (one per SM; twice as many fit), 4 = 4 x 16 KiB (three
  * per SM),
@@ -452,6 +467,23 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
 #define MPRESS_OPT_VARIANT   3
 #define MPRESS_OPT_ORDER     4
 #define MPRESS_OPT_PDL       7
+/* MPRESS_OPT_PACE_MBPS: 0 (default) = the SM kernels move bytes as fast as
+ * the links allow; R > 0 = each swap launch moves at most R MB/s: its CTAs
+ * space their chunks on the GPU's global timer.  A swap is free when it
+ * finishes within its tensor's live interval (fn.1 P:226), so a swap
+ * beside compute needs only bytes / live-interval; pacing it there leaves
+ * the rest of HBM, L2 and the issue slots to the compute.  Not applied to
+ * the copy-engine path. */
+#define MPRESS_OPT_PACE_MBPS 12
+/* MPRESS_OPT_SPLIT: how one launch's chunks (interleaved over the peers, see
+ * MPRESS_OPT_ORDER) are shared by its CTAs -- MPRESS_SPLIT_BLOCKED (0,
+ * default): each CTA takes a contiguous block of the sequence, so every CTA
+ * moves the same number of chunks +- one per peer; MPRESS_SPLIT_STRIDED (1,
+ * round 1): a grid stride over the sequence, whose skipped positions alias
+ * with the stride (up to 1.7x the mean chunk count on one CTA). */
+#define MPRESS_OPT_SPLIT     13
+#define MPRESS_SPLIT_BLOCKED 0
+#define MPRESS_SPLIT_STRIDED 1
 /* Read-only (mpress_get_option): how the peer pools were mapped --
  * MPRESS_TRANSPORT_LOCAL (mpress_init_local), _VMM_FD (cuMem pools exported
  * as POSIX fds, passed over Unix sockets), or _LEGACY_IPC (cudaMalloc pools
@@ -483,7 +515,11 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
 #define MPRESS_PATH_AUTO     3
 MPRESS_API int mpress_set_option(mpress_ctx_t* ctx, int key, int64_t value);
 
-/* Measure, don't guess: which SM kernel MPRESS_PATH_AUTO should run for an
+/* mpress_autotune -- not a paper operation: a B200 addition.
+ * The paper's transfer mechanism is fixed (cudaMemcpyPeer over NVLink,
+ * P:121); here two SM kernels and the copy engines can move a stripe, so
+ * the library measures which is faster on the context's own links.
+ * Measure, don't guess: which SM kernel MPRESS_PATH_AUTO should run for an
  * uncapped grid on THIS context's links (HBM loopback on one GPU, NVLink /
  * NVSwitch on several -- the kernels were only ever compared on loopback,
  * DESIGN.md §7), per direction and size class.  The probe is `probe_bytes`
@@ -599,15 +635,29 @@ MPRESS_API int mpress_handle_is_graph(const mpress_handle_t* handle);
  * pool [world]; UINT64_MAX for peers the plan does not use (tests). */
 MPRESS_API int mpress_handle_slices(const mpress_handle_t* handle, uint64_t* slice_off);
 
-/* Release a handle.  A handle still OUT_PENDING or OUT (data only in the
- * stash) is an error (MPRESS_ERR_STATE) unless `force` is nonzero.  An
- * IN_PENDING handle may be freed: its slices stay fenced by the swap-in event. */
+/* mpress_handle_free -- retire the tensor batch's metadata-table entry
+ * (recorded before the swap-out, "used to guide the execution of the
+ * latter swap-in operator and updated when it completes").  A handle still
+ * OUT_PENDING or OUT (data only in the stash) is an error (MPRESS_ERR_STATE)
+ * unless `force` is nonzero.  `force` is not in the paper (a deviation, see
+ * DESIGN.md §9): it drops stashed data the caller no longer needs, e.g. when
+ * a pipeline aborts a step.  An IN_PENDING handle may be freed: its slices
+ * stay fenced by the swap-in event.  Errors: MPRESS_ERR_ARG (NULL, or a
+ * handle of another context), MPRESS_ERR_STATE. */
 MPRESS_API int mpress_handle_free(mpress_ctx_t* ctx, mpress_handle_t* handle, int force);
 
 /* Debug / test: synchronous copy of `len` bytes at byte `offset` of this
  * source's partition on `peer` into host memory `host_dst`. */
 MPRESS_API int mpress_peer_read(mpress_ctx_t* ctx, int peer, uint64_t offset, uint64_t len,
                      void* host_dst);
+
+/* Debug / test: *out = this process's device address of byte `offset` of
+ * this source's partition on `peer` (its peer mapping, P:211's "indices of
+ * target GPU devices" resolved to memory), so a device-side checker can read
+ * a whole stash slice in place without a host copy.  The address stays valid
+ * until mpress_finalize; the bytes are defined only inside stripes of a
+ * swapped-out handle.  Errors: MPRESS_ERR_ARG, MPRESS_ERR_PEER (not mapped). */
+MPRESS_API int mpress_peer_ptr(const mpress_ctx_t* ctx, int peer, uint64_t offset, void** out);
 
 /* Kernel launches the last swap_out / swap_in call enqueued (for accounting). */
 MPRESS_API int mpress_last_launches(const mpress_ctx_t* ctx);

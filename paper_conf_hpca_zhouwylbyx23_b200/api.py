@@ -25,6 +25,9 @@ DEVICE_HOST = -1   # mpress_init_local: a pinned host pool as a peer (NEXT-4)
 OPT_TRANSPORT = 5  # read-only
 OPT_LAST_PATH = 6  # read-only: path of the last swap call
 OPT_PDL = 7
+OPT_PACE_MBPS = 12
+OPT_SPLIT = 13
+SPLIT_BLOCKED, SPLIT_STRIDED = 0, 1
 OPT_AUTO_OUT, OPT_AUTO_IN = 8, 9   # read-only: AUTO's uncapped-grid path per direction (large launches)
 OPT_AUTO_OUT_SMALL, OPT_AUTO_IN_SMALL = 10, 11   # ... for launches < AUTO_SMALL_BYTES
 AUTO_SMALL_BYTES = 32 << 20
@@ -48,7 +51,7 @@ EXPORTED = [
     "mpress_finalize", "mpress_stash_free", "mpress_set_option", "mpress_get_option", "mpress_autotune",
     "mpress_swap_out", "mpress_swap_in", "mpress_wait", "mpress_query", "mpress_handle_state",
     "mpress_handle_is_graph",
-    "mpress_handle_slices", "mpress_handle_free", "mpress_peer_read", "mpress_last_launches",
+    "mpress_handle_slices", "mpress_handle_free", "mpress_peer_read", "mpress_peer_ptr", "mpress_last_launches",
     "mpress_share_fds", "mpress_last_error", "mpress_version",
 ]
 
@@ -136,6 +139,7 @@ def _load():
         "mpress_handle_slices": (c_int, [P, P]),
         "mpress_handle_free": (c_int, [P, P, c_int]),
         "mpress_peer_read": (c_int, [P, c_int, c_uint64, c_uint64, P]),
+        "mpress_peer_ptr": (c_int, [P, c_int, c_uint64, POINTER(P)]),
         "mpress_last_launches": (c_int, [P]),
         "mpress_share_fds": (c_int, [c_int, c_int, c_int, P, EXCHANGE_FN, P, P]),
         "mpress_last_error": (c_char_p, []),
@@ -559,6 +563,13 @@ class Context:
 
     def query(self, handle):
         return _check(lib.mpress_query(self._h, handle._h)) == 1
+
+    def peer_ptr(self, peer, offset=0):
+        """mpress_peer_ptr: device address (int) of byte `offset` of this
+        source's partition on `peer` (debug / test)."""
+        out = c_void_p()
+        _check(lib.mpress_peer_ptr(self._h, peer, offset, byref(out)))
+        return out.value or 0
 
     def peer_read(self, peer, offset, length):
         buf = ctypes.create_string_buffer(max(1, length))

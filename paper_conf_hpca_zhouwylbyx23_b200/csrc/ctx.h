@@ -104,6 +104,8 @@ struct mpress_ctx_s {
   int variant = MPRESS_VARIANT_AUTO;
   int order = MPRESS_ORDER_INTERLEAVE;
   int pdl = 1;                        // MPRESS_OPT_PDL
+  uint64_t pace_mbps = 0;             // MPRESS_OPT_PACE_MBPS (0 = unpaced)
+  int split = 0;                      // MPRESS_OPT_SPLIT
   // SM path MPRESS_PATH_AUTO takes for an uncapped grid, per direction
   // (kDirOut, kDirIn) and size class (a launch moving < MPRESS_AUTO_SMALL_BYTES,
   // or more); until mpress_autotune measures otherwise: direct for small

@@ -479,6 +479,17 @@ extern "C" int mpress_set_option(mpress_ctx_t* c, int key, int64_t value) {
         return fail(MPRESS_ERR_ARG, "unknown chunk order %lld", (long long)value);
       c->order = (int)value;
       return MPRESS_OK;
+    case MPRESS_OPT_PACE_MBPS:
+      if (value < 0 || value > (int64_t)100000000)
+        return fail(MPRESS_ERR_ARG, "MPRESS_OPT_PACE_MBPS is 0 (off) or a rate in MB/s up to 1e8, not %lld",
+                    (long long)value);
+      c->pace_mbps = (uint64_t)value;
+      return MPRESS_OK;
+    case MPRESS_OPT_SPLIT:
+      if (value != MPRESS_SPLIT_BLOCKED && value != MPRESS_SPLIT_STRIDED)
+        return fail(MPRESS_ERR_ARG, "MPRESS_OPT_SPLIT is 0 (blocked) or 1 (strided), not %lld", (long long)value);
+      c->split = (int)value;
+      return MPRESS_OK;
     case MPRESS_OPT_VARIANT: {
       const int nvar = c->path == MPRESS_PATH_BULK ? kBulkVariants
                        : c->path == MPRESS_PATH_CE ? kCeVariants
@@ -501,6 +512,8 @@ extern "C" int mpress_get_option(const mpress_ctx_t* c, int key, int64_t* value)
     case MPRESS_OPT_VARIANT: *value = c->variant; return MPRESS_OK;
     case MPRESS_OPT_ORDER: *value = c->order; return MPRESS_OK;
     case MPRESS_OPT_PDL: *value = c->pdl; return MPRESS_OK;
+    case MPRESS_OPT_PACE_MBPS: *value = (int64_t)c->pace_mbps; return MPRESS_OK;
+    case MPRESS_OPT_SPLIT: *value = c->split; return MPRESS_OK;
     case MPRESS_OPT_TRANSPORT: *value = c->transport; return MPRESS_OK;
     case MPRESS_OPT_LAST_PATH: *value = c->last_path; return MPRESS_OK;
     case MPRESS_OPT_AUTO_OUT: *value = c->auto_path[mpress::kDirOut][1]; return MPRESS_OK;
@@ -522,6 +535,18 @@ extern "C" int mpress_peer_read(mpress_ctx_t* c, int peer, uint64_t offset, uint
   DeviceGuard g(c->device);
   cudaError_t e = cudaMemcpy(host_dst, part.base + offset, len, cudaMemcpyDeviceToHost);
   if (e != cudaSuccess) return fail(MPRESS_ERR_CUDA, "mpress_peer_read: %s", cudaGetErrorString(e));
+  return MPRESS_OK;
+}
+
+extern "C" int mpress_peer_ptr(const mpress_ctx_t* c, int peer, uint64_t offset, void** out) {
+  if (!c || !out || peer < 0 || peer >= c->world) return fail(MPRESS_ERR_ARG, "mpress_peer_ptr: bad argument");
+  *out = nullptr;
+  const Partition& part = c->parts[peer];
+  if (!part.base) return fail(MPRESS_ERR_PEER, "mpress_peer_ptr: peer %d not mapped", peer);
+  if (offset > part.size)
+    return fail(MPRESS_ERR_ARG, "mpress_peer_ptr: offset %llu outside the partition (%llu B)",
+                (unsigned long long)offset, (unsigned long long)part.size);
+  *out = part.base + offset;
   return MPRESS_OK;
 }
 

@@ -164,7 +164,7 @@ int run_copy(mpress_ctx_s* c, int dir, const std::vector<CopyDesc>& d,
     if (!graph && d.size() > (size_t)kParamDescMax && !c->ring) MP_TRY(table_ring_create(c->device, &c->ring));
     return launch_copy(path, c->variant, dir, d.data(),
                        c->order == MPRESS_ORDER_INTERLEAVE ? desc_peer.data() : nullptr, d.size(), c->max_ctas,
-                       c->pdl, stream, &c->last_launches, graph ? nullptr : c->ring);
+                       c->pdl, stream, &c->last_launches, graph ? nullptr : c->ring, c->pace_mbps, c->split);
   }
 
   // Copy-engine comparator (the prior-art mechanism):

@@ -64,7 +64,9 @@ struct CopyTable {
   uint32_t n;                        // descriptors
   uint32_t n_groups;                 // runs of descriptors with the same peer
   uint32_t rounds_log2;              // R = 2^rounds_log2 >= chunks of the largest group
-  uint32_t pad;
+  uint32_t pace_ns;                  // 0, or ns between the starts of one CTA's chunks (rate pacing)
+  uint32_t split;                    // kSplitBlocked / kSplitStrided: positions -> CTAs (Cursor)
+  uint32_t pad[3];
   uint32_t g_chunk[kGroups + 1];     // first chunk of each group (prefix)
   uint32_t g_desc[kGroups + 1];      // first descriptor of each group (prefix)
   uint32_t first_chunk[CAP + 1];     // first chunk of each descriptor (prefix)
@@ -86,25 +88,67 @@ __device__ __forceinline__ uint32_t upper_idx(const uint32_t* a, uint32_t n, uin
 // (r, g) holds chunk k = floor(r * n_g / R) of group g.  k is non-decreasing
 // in r with steps of 0 or 1 and reaches n_g - 1 by r = R - 1, so taking only
 // the first round that reaches each k visits every chunk exactly once; the
-// other positions are skipped.  A CTA walks positions blockIdx.x,
-// + gridDim.x, ... with (r, g) advanced incrementally (no division per step).
+// other positions are skipped.
+//
+// Which CTA takes which positions (CopyTable::split):
+//   kSplitBlocked (default): CTA b walks the contiguous block of positions
+//     [b*P/grid, (b+1)*P/grid), P = R * n_groups.  Every group's valid
+//     positions are spread evenly over the sequence, so every block holds
+//     total/grid +- n_groups chunks, and inside a block the CTA still visits
+//     the peers in proportion.
+//   kSplitStrided (round 1): CTA b walks positions b, b + grid, ...  The
+//     skip pattern aliases with the stride, so CTAs got up to 1.7x the mean
+//     chunk count (cfg2 micro-batch, 128 CTAs of 32 KiB chunks: 0 .. 384
+//     chunks, mean 225) -- a tail, and a rate-paced launch ran at mean/max of
+//     its rate.
+// (r, g) is advanced incrementally (no division per step).
+enum : uint32_t { kSplitBlocked = 0, kSplitStrided = 1 };
+
 template <int CAP>
 struct Cursor {
   const CopyTable<CAP>& t;
   uint32_t g, gm, gd;
   uint64_t r;
-  __device__ explicit Cursor(const CopyTable<CAP>& tt) : Cursor(tt, blockIdx.x, gridDim.x) {}
-  // positions start, start + stride, ...
-  __device__ Cursor(const CopyTable<CAP>& tt, uint32_t start, uint32_t stride) : t(tt) {
-    g = start % t.n_groups;
-    r = start / t.n_groups;
-    gm = stride % t.n_groups;
-    gd = stride / t.n_groups;
+  uint64_t left;  // positions this cursor still visits
+  // This CTA's positions under the table's split (one cursor per CTA).
+  __device__ explicit Cursor(const CopyTable<CAP>& tt) : t(tt) {
+    uint64_t start, stride, end;
+    span(tt, 0, 1, &start, &stride, &end);
+    init(start, stride, end);
   }
-  // Next chunk of this CTA: its index *c and its descriptor *s.
+  // Lane `lane` of `lanes` cursors sharing this CTA's positions (the bulk
+  // kernel's 32 resolver lanes): every lanes-th position of the CTA's share.
+  __device__ Cursor(const CopyTable<CAP>& tt, uint32_t lane, uint32_t lanes) : t(tt) {
+    uint64_t start, stride, end;
+    span(tt, lane, lanes, &start, &stride, &end);
+    init(start, stride, end);
+  }
+  __device__ static void span(const CopyTable<CAP>& tt, uint32_t lane, uint32_t lanes, uint64_t* start,
+                              uint64_t* stride, uint64_t* end) {
+    const uint64_t P = (uint64_t)tt.n_groups << tt.rounds_log2;
+    if (tt.split == kSplitStrided) {
+      *start = blockIdx.x + (uint64_t)lane * gridDim.x;
+      *stride = (uint64_t)lanes * gridDim.x;
+      *end = P;
+    } else {
+      const uint64_t b0 = (uint64_t)(((unsigned __int128)P * blockIdx.x) / gridDim.x);
+      const uint64_t b1 = (uint64_t)(((unsigned __int128)P * (blockIdx.x + 1)) / gridDim.x);
+      *start = b0 + lane;
+      *stride = lanes;
+      *end = b1;
+    }
+  }
+  __device__ void init(uint64_t start, uint64_t stride, uint64_t end) {
+    g = (uint32_t)(start % t.n_groups);
+    r = start / t.n_groups;
+    gm = (uint32_t)(stride % t.n_groups);
+    gd = (uint32_t)(stride / t.n_groups);
+    left = start < end ? (end - start + stride - 1) / stride : 0;
+  }
+  // Next chunk of this cursor: its index *c and its descriptor *s.
   __device__ bool next(uint32_t* c, uint32_t* s) {
-    const uint64_t R = 1ull << t.rounds_log2;
-    while (r < R) {
+    while (left) {
+      --left;
       const uint32_t gg = g;
       const uint64_t rr = r;
       g += gm;
@@ -188,6 +232,35 @@ __device__ __forceinline__ void pdl_enter() {
   asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
 }
 
+// Rate pacing (MPRESS_OPT_PACE_MBPS): chunk i of a CTA may start no earlier
+// than t0 + i * pace_ns (%globaltimer, ns), so the launch moves at most the
+// requested rate however fast the links are.  A swap only has to finish
+// within its tensor's live interval; moving it faster than that only
+// takes HBM, L2 and issue slots from the compute it runs beside.  The
+// schedule is absolute, so timer granularity and sleep overshoot do not
+// accumulate.
+struct Pacer {
+  uint64_t t0 = 0, next = 0;
+  uint32_t step;
+  __device__ explicit Pacer(uint32_t pace_ns) : step(pace_ns) {
+    if (step) {
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+      next = t0;
+    }
+  }
+  __device__ __forceinline__ void wait() {
+    if (!step) return;
+    for (;;) {
+      uint64_t now;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(now));
+      if (now >= next) break;
+      const uint64_t d = next - now;
+      __nanosleep(d > 100000 ? 100000u : (unsigned)d);
+    }
+    next += step;
+  }
+};
+
 // ---------------------------------------------------------------- direct path
 
 struct Span {
@@ -223,9 +296,11 @@ __device__ __forceinline__ void direct_body(const CopyTable<CAP>& t) {
   uint32_t c, s;
   if (!cur.next(&c, &s)) return;
   Span sp = span_of<kShift>(t, c, s);
+  Pacer pace(t.pace_ns);
   for (;;) {
     Span nx{nullptr, nullptr, 0};
     bool more = false;
+    pace.wait();
     if (sp.rem >= kChunk) {
       const VT* sv = reinterpret_cast<const VT*>(sp.src) + threadIdx.x;
       VT* dv = reinterpret_cast<VT*>(sp.dst) + threadIdx.x;
@@ -350,8 +425,8 @@ __device__ __forceinline__ uint64_t shfl64(uint64_t v, int lane) {
 // One warp per CTA: lane 0 streams pieces of 2^SHIFT bytes through STAGES
 // shared-memory slots with the SM's bulk-copy engine (cp.async.bulk G->S with
 // mbarrier completion, then S->G bulk stores).  The 32 lanes resolve the
-// chunk sequence in parallel -- lane j walks positions blockIdx.x +
-// (j + 32i) * gridDim.x with its own cursor -- and hand the pieces to lane 0
+// chunk sequence in parallel -- lane j walks every 32nd position of the
+// CTA's share from the j-th on, with its own cursor -- and hand the pieces to lane 0
 // by shuffles, so the descriptor lookups (dependent constant-bank loads) are
 // off the issuing thread's critical path (profiles/r01: with one cursor on
 // lane 0 they took ~75% of its issue samples).  Each lane also copies the
@@ -377,6 +452,7 @@ __device__ __forceinline__ void bulk_body(const CopyTable<CAP>& t) {
   __syncwarp();
 
   uint32_t loaded = 0, stored = 0;  // pieces whose load / store was issued (lane 0)
+  Pacer pace(lane == 0 ? t.pace_ns : 0u);
   // lane 0: issue the stores of pieces [stored, upto) in order
   auto store_until = [&](uint32_t upto) {
     for (; stored < upto; ++stored) {
@@ -387,7 +463,7 @@ __device__ __forceinline__ void bulk_body(const CopyTable<CAP>& t) {
     }
   };
 
-  Cursor<CAP> cur(t, blockIdx.x + lane * gridDim.x, 32u * gridDim.x);
+  Cursor<CAP> cur(t, lane, 32u);
   for (;;) {
     uint32_t c, sd;
     const bool v = cur.next(&c, &sd);
@@ -418,6 +494,7 @@ __device__ __forceinline__ void bulk_body(const CopyTable<CAP>& t) {
           store_until(k - STAGES + 2 <= k ? k - STAGES + 2 : k);  // stores through piece k-STAGES+1
           bulk_wait_read1();  // all but the newest store have left smem: slot of k-STAGES is free
         }
+        pace.wait();
         const uint32_t q = k % STAGES;
         ring_dst[q] = dst;
         ring_bytes[q] = bytes;
@@ -460,13 +537,15 @@ struct Shape {
 // direct (threads, unroll, vector bytes): 0 (256,8,16) 1 (512,8,16)
 // 2 (256,16,16) 3 (1024,4,16) 4 (128,8,16) 5 (256,4,32) 6 (256,8,32)
 // 7 (128,4,32) 8 (256,4,32 + L2 evict-first loads) 9 (128,8,32)
+// 10 (128,16,32) 11 (64,16,32) -- 32 / 64 KiB in flight per CTA with few
+// warps, for a capped grid beside a GEMM (its CTA leaves ~22.5K registers)
 // bulk (piece, stages, CTAs/SM): 0 (32K,6,1) 1 (16K,12,1) 2 (64K,3,1) 3 (32K,3,1)
 // 4 (16K,4,3) 5 (8K,2,1) 6 (4K,3,1) -- 5 and 6 use 16 / 12 KB of shared
 // memory, small enough to sit beside a cuBLAS GEMM CTA (214 KB)
 constexpr Shape kDirect[kDirectVariants] = {
     {256, 15, 0, 2, 16, 0}, {512, 16, 0, 1, 16, 1}, {256, 16, 0, 2, 16, 2}, {1024, 16, 0, 1, 16, 3},
     {128, 14, 0, 4, 16, 4}, {256, 15, 0, 2, 32, 0}, {256, 16, 0, 2, 32, 2}, {128, 14, 0, 4, 32, 4},
-    {256, 15, 0, 2, 32, 0}, {128, 15, 0, 4, 32, 4}};
+    {256, 15, 0, 2, 32, 0}, {128, 15, 0, 4, 32, 4}, {128, 16, 0, 4, 32, 4}, {64, 15, 0, 8, 32, 4}};
 constexpr Shape kBulk[kBulkVariants] = {
     {32, 15, 6u << 15, 1, 16, 0}, {32, 14, 12u << 14, 1, 16, 1}, {32, 16, 3u << 16, 1, 16, 2},
     {32, 15, 3u << 15, 1, 16, 3}, {32, 14, 4u << 14, 3, 16, 4}, {32, 13, 2u << 13, 1, 16, 5},
@@ -521,6 +600,8 @@ std::conditional_t<G, KernelFnG<CAP>, KernelFn<CAP>> kernel_for(int path, int va
       case 7: k = MP_DIRECT(128, 4, 32, false); break;
       case 8: k = MP_DIRECT(256, 4, 32, true); break;
       case 9: k = MP_DIRECT(128, 8, 32, false); break;
+      case 10: k = MP_DIRECT(128, 16, 32, false); break;
+      case 11: k = MP_DIRECT(64, 16, 32, false); break;
       default: k = MP_DIRECT(256, 8, 16, false); break;
     }
   }
@@ -563,7 +644,8 @@ template <int CAP>
 int build_table(CopyTable<CAP>& t, const CopyDesc* d, const int* gid, uint32_t n, uint32_t shift,
                 uint64_t* chunks_out) {
   t.n = n;
-  t.pad = 0;
+  t.pace_ns = 0;
+  t.split = 0;
   uint64_t chunks = 0;
   uint32_t ng = 0;
   for (uint32_t i = 0; i < n; ++i) {
@@ -587,6 +669,14 @@ int build_table(CopyTable<CAP>& t, const CopyDesc* d, const int* gid, uint32_t n
   while ((1ull << t.rounds_log2) < largest) ++t.rounds_log2;
   *chunks_out = chunks;
   return MPRESS_OK;
+}
+
+// ns between one CTA's chunks so that `grid` CTAs move 2^shift-byte chunks
+// at pace_mbps MB/s in total (0 = unpaced).
+uint32_t pace_ns_of(uint64_t pace_mbps, uint32_t shift, unsigned grid) {
+  if (!pace_mbps) return 0;
+  const uint64_t ns = ((uint64_t)grid << shift) * 1000ull / pace_mbps;
+  return (uint32_t)std::min<uint64_t>(std::max<uint64_t>(ns, 1), 0xFFFFFFFFull);
 }
 
 template <typename K, typename Arg>
@@ -613,13 +703,16 @@ int launch_kernel(K k, const Shape& sh, unsigned grid, bool pdl, cudaStream_t st
 // One launch with the table as a kernel parameter.
 template <int CAP>
 int launch_batch(int path, int variant, int dir, const CopyDesc* d, const int* gid, uint32_t n,
-                 uint32_t shift, int cap, int sms, bool pdl, cudaStream_t stream, bool* launched) {
+                 uint32_t shift, int cap, int sms, bool pdl, uint64_t pace_mbps, int split, cudaStream_t stream,
+                 bool* launched) {
   CopyTable<CAP> t;
   uint64_t chunks = 0;
   *launched = false;
   MP_TRY(build_table(t, d, gid, n, shift, &chunks));
   if (chunks == 0) return MPRESS_OK;
   const unsigned grid = (unsigned)std::min<uint64_t>(chunks, (uint64_t)cap);
+  t.pace_ns = pace_ns_of(pace_mbps, shift, grid);
+  t.split = (uint32_t)split;
   const Shape& sh = shape_of(path, variant);
   MP_TRY(launch_kernel(kernel_for<CAP, false>(path, variant, dir, (int)grid <= sms), sh, grid, pdl, stream, t));
   *launched = true;
@@ -631,7 +724,8 @@ int launch_batch(int path, int variant, int dir, const CopyDesc* d, const int* g
 // read by the kernel through a pointer; the slot's event, recorded after the
 // kernel, guards both slots' reuse.
 int launch_batch_ring(TableRing* r, int path, int variant, int dir, const CopyDesc* d, const int* gid, uint32_t n,
-                      uint32_t shift, int cap, int sms, bool pdl, cudaStream_t stream, bool* launched) {
+                      uint32_t shift, int cap, int sms, bool pdl, uint64_t pace_mbps, int split,
+                      cudaStream_t stream, bool* launched) {
   using T = CopyTable<kMaxDescPerLaunch>;
   *launched = false;
   const int slot = r->next;
@@ -646,10 +740,12 @@ int launch_batch_ring(TableRing* r, int path, int variant, int dir, const CopyDe
   MP_TRY(build_table(*ht, d, gid, n, shift, &chunks));
   if (chunks == 0) return MPRESS_OK;
   r->next = (slot + 1) % r->nslots;
+  const unsigned grid = (unsigned)std::min<uint64_t>(chunks, (uint64_t)cap);
+  ht->pace_ns = pace_ns_of(pace_mbps, shift, grid);
+  ht->split = (uint32_t)split;
   const size_t bytes = offsetof(T, d) + (size_t)n * sizeof(CopyDesc);
   cudaError_t e = cudaMemcpyAsync(dt, ht, bytes, cudaMemcpyHostToDevice, stream);
   if (e != cudaSuccess) return fail(MPRESS_ERR_CUDA, "descriptor upload: %s", cudaGetErrorString(e));
-  const unsigned grid = (unsigned)std::min<uint64_t>(chunks, (uint64_t)cap);
   const Shape& sh = shape_of(path, variant);
   MP_TRY(launch_kernel(kernel_for<kMaxDescPerLaunch, true>(path, variant, dir, (int)grid <= sms), sh, grid, pdl,
                        stream, static_cast<const T*>(dt)));
@@ -746,7 +842,8 @@ void table_ring_destroy(TableRing* r) {
 }
 
 int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* group, size_t n,
-                int max_ctas, int pdl_mode, cudaStream_t stream, int* launches, TableRing* ring) {
+                int max_ctas, int pdl_mode, cudaStream_t stream, int* launches, TableRing* ring,
+                uint64_t pace_mbps, int split) {
   int dev = 0, sms = 0;
   if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess)
     return fail(MPRESS_ERR_CUDA, "cannot query the SM count");
@@ -788,17 +885,17 @@ int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* gr
     const int* g = group ? group + base : nullptr;
     bool launched = false;
     if (ring && m > (uint32_t)kParamDescMax)
-      MP_TRY(launch_batch_ring(ring, path, variant, dir, d + base, g, m, shift, cap, sms, pdl, stream, &launched));
+      MP_TRY(launch_batch_ring(ring, path, variant, dir, d + base, g, m, shift, cap, sms, pdl, pace_mbps, split, stream, &launched));
     else if (m <= 16)
-      MP_TRY(launch_batch<16>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, stream, &launched));
+      MP_TRY(launch_batch<16>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, pace_mbps, split, stream, &launched));
     else if (m <= 32)
-      MP_TRY(launch_batch<32>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, stream, &launched));
+      MP_TRY(launch_batch<32>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, pace_mbps, split, stream, &launched));
     else if (m <= 64)
-      MP_TRY(launch_batch<64>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, stream, &launched));
+      MP_TRY(launch_batch<64>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, pace_mbps, split, stream, &launched));
     else if (m <= 128)
-      MP_TRY(launch_batch<128>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, stream, &launched));
+      MP_TRY(launch_batch<128>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, pace_mbps, split, stream, &launched));
     else
-      MP_TRY(launch_batch<kMaxDescPerLaunch>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, stream, &launched));
+      MP_TRY(launch_batch<kMaxDescPerLaunch>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, pace_mbps, split, stream, &launched));
     if (launched && launches) ++*launches;
   }
   return MPRESS_OK;

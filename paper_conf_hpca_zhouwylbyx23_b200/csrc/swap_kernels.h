@@ -18,7 +18,7 @@ struct CopyDesc {
 };
 
 constexpr int kMaxDescPerLaunch = 1024;  // fits the 32 KB kernel-parameter space
-constexpr int kDirectVariants = 10;      // MPRESS_OPT_VARIANT range, direct path
+constexpr int kDirectVariants = 12;      // MPRESS_OPT_VARIANT range, direct path
 constexpr int kBulkVariants = 7;         // MPRESS_OPT_VARIANT range, bulk path
 constexpr int kCeVariants = 1;           // copy engines: 0 = cudaMemcpyAsync per stripe, per-peer streams
 
@@ -54,9 +54,14 @@ void table_ring_destroy(TableRing* r);
 // of kernel launches to *launches.  Returns MPRESS_OK or MPRESS_ERR_*.
 // `ring` (may be null): device-resident tables for launches of more than
 // kParamDescMax descriptors.
+// `pace_mbps` (MPRESS_OPT_PACE_MBPS, 0 = off): the launch's CTAs space their
+// chunks so the whole launch moves at most pace_mbps MB/s.  `split`
+// (MPRESS_OPT_SPLIT): 0 = each CTA takes a contiguous block of the
+// interleaved chunk sequence, 1 = a grid stride over it (round 1).
 int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* group, size_t n,
                 int max_ctas, int pdl_mode,
-                cudaStream_t stream, int* launches, TableRing* ring = nullptr);
+                cudaStream_t stream, int* launches, TableRing* ring = nullptr, uint64_t pace_mbps = 0,
+                int split = 0);
 
 // Default grid of a path/variant on the current device (SMs x CTAs per SM).
 int copy_wave_ctas(int path, int variant);

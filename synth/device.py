@@ -45,6 +45,15 @@ def check(t, seed, tensor_id, start=0, nbytes=None, stream=None):
     return r
 
 
+def check_ptr(ptr, nbytes, seed, tensor_id, start=0, stream=None):
+    """Number of bytes at device address `ptr` (nbytes of them) that differ
+    from generator bytes [start, start+nbytes) of tensor `tensor_id`."""
+    r = _get().synth_check(ptr, nbytes, seed, tensor_id, start, _stream(stream))
+    if r < 0:
+        raise RuntimeError("synth_check failed")
+    return r
+
+
 def stamp(base_u64, stream=None):
     """Write %globaltimer into base_u64 (a 1-element int64 CUDA tensor)."""
     lib = _get()

@@ -1,9 +1,10 @@
 """Full-size parity at BASELINE.json's sizes, in the launch configurations
 bench.py times (default grid; AUTO's default kernel and the direct kernel,
-the two mpress_autotune chooses between): sampled stash windows against the
-oracle's plan + the generator (the oracle computes each window one by one),
-and the round trip checked on the device against the generator for every
-byte.  Plus compute-sanitizer memcheck of the smoke path."""
+the two mpress_autotune chooses between): EVERY stash byte of every stripe
+of the oracle's plan checked in place on the device (mpress_peer_ptr + the
+generator's check kernel) against the oracle's byte model, sampled windows
+also copied to the host and compared with the generator there, and the
+round trip checked on the device against the generator for every byte.  Plus compute-sanitizer memcheck of the smoke path."""
 import os
 import random
 import shutil
@@ -46,6 +47,16 @@ def _sampled_roundtrip(world, source, spare, bw, sizes, seed, samples=64, path=N
         h = ctx.swap_out(pl, src, stream=s)
         s.synchronize()
         sl = h.slices()
+        # every stash byte of every stripe, on the device: the oracle's byte
+        # model (stash[p][dst_off:+len] =
+        # tensor[i][src_off:+len]) over the oracle's own stripes, with the
+        # tensor bytes regenerated from (seed, i, src_off)
+        bad, checked = 0, 0
+        for (i, p, so, do, ln) in o["stripes"]:
+            bad += synth_dev.check_ptr(ctx.peer_ptr(p, sl[p] + do), ln, seed, i, start=so)
+            checked += ln
+        assert bad == 0, "%d of %d stash bytes differ from the oracle's byte model" % (bad, checked)
+        assert checked == sum(sizes)
         rng = random.Random(seed)
         picks = list(o["stripes"])
         rng.shuffle(picks)

@@ -178,3 +178,93 @@ def test_autotune_local():
                 h.free()
     finally:
         ctx.finalize()
+
+
+@pytest.mark.parametrize("path,cap", [(mp.PATH_DIRECT, 32), (mp.PATH_DIRECT, 0), (mp.PATH_BULK, 0)])
+def test_pace_limits_rate_and_keeps_bytes(path, cap):
+    """MPRESS_OPT_PACE_MBPS: a paced swap moves at most the requested rate
+    (it only has to fit the live interval), and its stash and restored
+    bytes still equal the oracle's byte model."""
+    import oracle
+    from _swaputil import check_stash, host_inputs, make_inputs
+    from synth import device as synth_dev
+    world, G = 4, 65536
+    sizes = [(64 << 20) + 48, 3 << 20, 1000]
+    spare, bw = [0, 1 << 30, 1 << 30, 1 << 30], [0, 1, 2, 1]
+    pl = mp.plan(world, 0, spare, bw, sizes, G)
+    o = oracle.plan(world, 0, spare, bw, sizes, G)
+    part = [[0] * world for _ in range(world)]
+    part[0] = [u * G for u in pl.units]
+    ctx = mp.Context.local(world, 0, [0] * world, part)
+    try:
+        ctx.set_option(mp.OPT_PATH, path)
+        ctx.set_option(mp.OPT_MAX_CTAS, cap)
+        src = make_inputs(sizes, 31)
+        dst = [torch.zeros_like(t) for t in src]
+        nbytes = sum(sizes)
+        s = torch.cuda.Stream()
+        for pace in (0, 100_000):          # off, then 100 GB/s
+            ctx.set_option(mp.OPT_PACE_MBPS, pace)
+            assert ctx.get_option(mp.OPT_PACE_MBPS) == pace
+            e = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
+            e[0].record(s)
+            h = ctx.swap_out(pl, src, stream=s)
+            e[1].record(s)
+            torch.cuda.synchronize()
+            check_stash(ctx, h, o, host_inputs(sizes, 31))
+            e[2].record(s)
+            ctx.swap_in(h, dst, stream=s)
+            e[3].record(s)
+            torch.cuda.synchronize()
+            h.free()
+            for i, t in enumerate(dst):
+                assert synth_dev.check(t, 31, i) == 0
+                t.zero_()
+            if pace:
+                for a, b in ((e[0], e[1]), (e[2], e[3])):
+                    gbs = nbytes / a.elapsed_time(b) / 1e6
+                    assert 60 < gbs <= 100 * 1.03, gbs
+        with pytest.raises(mp.MPressError):
+            ctx.set_option(mp.OPT_PACE_MBPS, -1)
+    finally:
+        ctx.finalize()
+
+
+@pytest.mark.parametrize("split", [0, 1], ids=["blocked", "strided"])
+@pytest.mark.parametrize("path,variant,cap", [(mp.PATH_DIRECT, 7, 5), (mp.PATH_DIRECT, 11, 128),
+                                              (mp.PATH_DIRECT, 5, 0), (mp.PATH_BULK, 3, 0),
+                                              (mp.PATH_BULK, 6, 7)])
+def test_split_modes_are_oracle_exact(split, path, variant, cap):
+    """MPRESS_OPT_SPLIT: both ways of sharing a launch's interleaved chunks
+    among CTAs write exactly the oracle's stash bytes and restore every
+    tensor, with ragged stripes over three peers of unequal weight."""
+    import oracle
+    from _swaputil import check_stash, host_inputs, make_inputs
+    from synth import device as synth_dev
+    world, G = 4, 65536
+    sizes = [(5 << 20) + 48, 777, 3 << 20, 70001]
+    spare, bw = [0, 1 << 30, 1 << 30, 1 << 30], [0, 1, 3, 2]
+    pl = mp.plan(world, 0, spare, bw, sizes, G)
+    o = oracle.plan(world, 0, spare, bw, sizes, G)
+    part = [[0] * world for _ in range(world)]
+    part[0] = [u * G for u in pl.units]
+    ctx = mp.Context.local(world, 0, [0] * world, part)
+    try:
+        ctx.set_option(mp.OPT_PATH, path)
+        ctx.set_option(mp.OPT_VARIANT, variant)
+        ctx.set_option(mp.OPT_MAX_CTAS, cap)
+        ctx.set_option(mp.OPT_SPLIT, split)
+        assert ctx.get_option(mp.OPT_SPLIT) == split
+        src = make_inputs(sizes, 41)
+        h = ctx.swap_out(pl, src)
+        torch.cuda.synchronize()
+        check_stash(ctx, h, o, host_inputs(sizes, 41))
+        dst = [torch.zeros_like(t) for t in src]
+        ctx.swap_in(h, dst)
+        torch.cuda.synchronize()
+        h.free()
+        assert all(synth_dev.check(t, 41, i) == 0 for i, t in enumerate(dst))
+        with pytest.raises(mp.MPressError):
+            ctx.set_option(mp.OPT_SPLIT, 2)
+    finally:
+        ctx.finalize()

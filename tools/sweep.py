@@ -36,6 +36,7 @@ def setup(sizes, peers_n, copies=1):
     part[0] = [copies * u * mp.DEFAULT_GRANULE for u in pl.units]
     ctx = mp.Context.local(world, 0, [0] * world, part)
     ctx.set_option(mp.OPT_PDL, int(os.environ.get("SWEEP_PDL", "1")))
+    ctx.set_option(mp.OPT_SPLIT, int(os.environ.get("SWEEP_SPLIT", "0")))
     src = [torch.empty(s, dtype=torch.uint8, device="cuda") for s in sizes]
     for i, t in enumerate(src):
         synth_dev.fill(t, 77, i)
@@ -66,7 +67,7 @@ def paths():
     nbytes = sum(sizes)
     ctx, pl, src, dst = setup(sizes, 3)
     s = torch.cuda.Stream()
-    nvar = {"direct": 10, "bulk": 7, "ce": 1, "auto": 0}  # plus -1 = auto
+    nvar = {"direct": 12, "bulk": 7, "ce": 1, "auto": 0}  # plus -1 = auto
     only = os.environ.get("SWEEP_PATHS")        # e.g. "direct"
     var_sel = os.environ.get("SWEEP_VARIANTS")  # e.g. "0,5,6,8"
     cap_sel = os.environ.get("SWEEP_CAPS")      # e.g. "0,148,296"
@@ -202,19 +203,22 @@ def gemm():
         if os.environ.get("GEMM_COMBOS"):  # e.g. "direct:4:64,96,128;ce:0:0"
             combos = []
             for part in os.environ["GEMM_COMBOS"].split(";"):
-                nm, v, caps = part.split(":")
-                combos += [(nm, int(v), int(cap)) for cap in caps.split(",")]
+                f = part.split(":")     # path:variant:caps[:pace MB/s]
+                pace = int(f[3]) if len(f) > 3 else 0
+                combos += [(f[0], int(f[1]), int(cap), pace) for cap in f[2].split(",")]
         else:
-            combos = [("direct", v, cap) for v in (0, 1, 4) for cap in (16, 32, 64, 96, 148)]
-            combos += [("bulk", 0, cap) for cap in (8, 16, 32)] + [("ce", 0, 0)]
-        for name, var, cap in combos:
+            combos = [("direct", v, cap, 0) for v in (0, 1, 4) for cap in (16, 32, 64, 96, 148)]
+            combos += [("bulk", 0, cap, 0) for cap in (8, 16, 32)] + [("ce", 0, 0, 0)]
+        rounds = int(os.environ.get("GEMM_ROUNDS", "2"))
+        for name, var, cap, pace in combos:
             ctx.set_option(mp.OPT_PATH, PATHS[name])
             if name != "ce":
                 ctx.set_option(mp.OPT_VARIANT, var)
             ctx.set_option(mp.OPT_MAX_CTAS, cap)
+            ctx.set_option(mp.OPT_PACE_MBPS, pace)
             to, ti = time_swaps(ctx, pl, src, dst, 3, swap)
-            alone, during, gbs = [], [], []
-            for _ in range(2):
+            alone, during, gbs, ratios = [], [], [], []
+            for _ in range(rounds):
                 evs = gemms()
                 torch.cuda.synchronize()
                 alone += [x.elapsed_time(y) for x, y in evs[4:]]
@@ -230,13 +234,19 @@ def gemm():
                 evs = gemms()
                 torch.cuda.synchronize()
                 win = s0.elapsed_time(s1)
-                during += [x.elapsed_time(y) for x, y in evs[4:]
-                           if s0.elapsed_time(x) >= 0 and s0.elapsed_time(y) <= win]
+                d_r = [x.elapsed_time(y) for x, y in evs[4:]
+                       if s0.elapsed_time(x) >= 0 and s0.elapsed_time(y) <= win]
+                during += d_r
+                if d_r:
+                    ratios.append(statistics.median(d_r) / statistics.median(alone[-(G - 4):]) - 1)
                 gbs.append(2 * n_swap * nbytes / win / 1e6)
             am = statistics.median(alone)
             dm = statistics.median(during) if during else float("nan")
             print(json.dumps({"sweep": "gemm", "shape": sname, "path": name, "variant": var,
-                              "max_ctas": cap, "alone_ms": am, "gemm_ms": dm, "slowdown": dm / am - 1,
+                              "max_ctas": cap, "pace_mbps": pace, "alone_ms": am, "gemm_ms": dm,
+                              "slowdown": dm / am - 1,
+                              "slowdown_paired_median": statistics.median(ratios) if ratios else None,
+                              "rounds": len(ratios),
                               "counted": len(during), "swap_alone_gbs": 2 * nbytes / (to + ti) / 1e6,
                               "swap_gbs_under_gemm": statistics.median(gbs)}), flush=True)
     ctx.finalize()
