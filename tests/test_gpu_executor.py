@@ -4,6 +4,7 @@ import pytest
 import torch
 
 import paper_conf_hpca_zhouwylbyx23_b200 as mp
+from oracle import pipeline as P
 from synth import device as synth_dev
 
 pytestmark = pytest.mark.gpu
@@ -43,13 +44,21 @@ def test_executor_steps_and_errors():
                 for i, t in enumerate(src[m]):
                     synth_dev.fill(t, 50 * step + m, i)
                 ex.restore_to(m, dst[m])
+            ops = []
             for j in range(ex.ops):
                 kind, m = ex.before(j, comp)
+                ops.append((kind, m))
                 ex.after(j, comp, src[m] if kind == "F" else None)
+            # the executor runs the oracle's 1F1B op order (reading R24) ...
+            assert ops == P.stage_ops(2, 0, M)
             torch.cuda.synchronize()
             for m in range(M):
                 for i, t in enumerate(dst[m]):
                     assert synth_dev.check(t, 50 * step + m, i) == 0, (step, m, i)
+        # ... and swaps at the oracle's points: every slot equals
+        # oracle.pipeline.schedule for the same parameters
+        slots, _ = P.schedule(2, 0, M, 10_000, 20_000, 5_000, 5_000)
+        assert [ex.slot(m) for m in range(M)] == slots
         ex.free()
     finally:
         ctx.finalize()
