@@ -66,13 +66,16 @@ def parse():
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
     ap.add_argument("--gemm-cap", type=int, default=0,
                     help="swap grid cap (CTAs = SMs touched) while the concurrent GEMM runs (AUTO path -> "
-                         "direct shape 7); 0 = calibrate: the first of --gemm-swap-candidates whose swap rate "
+                         "direct shape 9); 0 = calibrate: the first of --gemm-swap-candidates whose swap rate "
                          "on this run's links reaches --gemm-target-gbs / 0.85")
     ap.add_argument("--gemm-swap-candidates", default="auto:-1:64,bulk:5:148,auto:-1:96,auto:-1:128,auto:-1:148",
                     help="path:variant:max_ctas settings for the GEMM-concurrent swap, cheapest for the GEMM "
                          "first (profiles/r01/sweep_gemm_*)")
     ap.add_argument("--gemm-target-gbs", type=float, default=720.0,
                     help="per-source swap rate the GEMM-concurrent swap should sustain (BJ:5: 80%% of 900)")
+    ap.add_argument("--gemm-no-pace", action="store_true",
+                    help="run the GEMM-concurrent SM swap unpaced (default: paced to --gemm-target-gbs / 0.85 "
+                         "with MPRESS_OPT_PACE_MBPS)")
     ap.add_argument("--no-gemm", action="store_true")
     ap.add_argument("--no-gemm-ce", action="store_true", help="skip the copy-engine pass of the GEMM leg")
     ap.add_argument("--gemm-settle-s", type=float, default=2.0,
@@ -765,17 +768,20 @@ def bootstrap_ci95(xs, resamples=4000, seed=219):
     return meds[int(0.025 * (resamples - 1))], meds[int(0.975 * (resamples - 1))]
 
 
-def set_gemm_swap(ctx, mp, spec):
+def set_gemm_swap(ctx, mp, spec, pace_mbps=0):
     """Apply a GEMM-concurrent swap setting "path:variant:max_ctas" (path
-    auto/direct/bulk; auto with a cap <= the SM count runs direct shape 7);
-    returns the previous (path, variant, max_ctas) for restore_swap."""
-    prev = (ctx.get_option(mp.OPT_PATH), ctx.get_option(mp.OPT_VARIANT), ctx.get_option(mp.OPT_MAX_CTAS))
+    auto/direct/bulk; auto with a cap <= the SM count runs the capped direct
+    shape) and the rate pace (MPRESS_OPT_PACE_MBPS, 0 = unpaced; not applied
+    to the copy engines); returns the previous options for restore_swap."""
+    prev = (ctx.get_option(mp.OPT_PATH), ctx.get_option(mp.OPT_VARIANT), ctx.get_option(mp.OPT_MAX_CTAS),
+            ctx.get_option(mp.OPT_PACE_MBPS))
     name, var, cap = spec.split(":")
     paths = {"auto": mp.PATH_AUTO, "direct": mp.PATH_DIRECT, "bulk": mp.PATH_BULK, "ce": mp.PATH_CE}
     ctx.set_option(mp.OPT_PATH, paths[name])
     if name != "auto":
         ctx.set_option(mp.OPT_VARIANT, int(var))
     ctx.set_option(mp.OPT_MAX_CTAS, int(cap))
+    ctx.set_option(mp.OPT_PACE_MBPS, int(pace_mbps))
     return prev
 
 
@@ -784,6 +790,14 @@ def restore_swap(ctx, mp, prev):
     if prev[0] != mp.PATH_AUTO:
         ctx.set_option(mp.OPT_VARIANT, prev[1])
     ctx.set_option(mp.OPT_MAX_CTAS, prev[2])
+    ctx.set_option(mp.OPT_PACE_MBPS, prev[3])
+
+
+def gemm_pace_mbps(args):
+    """MB/s the GEMM-concurrent SM swap is paced to: the rate the calibration
+    asks of it (--gemm-target-gbs / 0.85), so the swap takes only the
+    bandwidth its target needs; 0 with --gemm-no-pace."""
+    return 0 if args.gemm_no_pace else int(round(args.gemm_target_gbs / 0.85 * 1000))
 
 
 def calibrate_gemm_cap(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap, n, dist):
@@ -877,7 +891,7 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
         st["b"] = torch.randn(K, N, dtype=torch.bfloat16, device="cuda")
         st["c"] = torch.empty(M, N, dtype=torch.bfloat16, device="cuda")
         st["pl"] = mp.plan(world, source, per_copy, bw, sizes)
-        st["prev"] = set_gemm_swap(ctx, mp, "ce:0:0" if ce else args.gemm_swap)
+        st["prev"] = set_gemm_swap(ctx, mp, "ce:0:0" if ce else args.gemm_swap, 0 if ce else gemm_pace_mbps(args))
         # swap time at this setting, to size the loop that must cover the GEMM
         # window; one untimed pair first (the copy-engine path creates its
         # side streams on first use, which once inflated the estimate so much
@@ -988,6 +1002,7 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
                 st.get("ran"), args.path),
             "swap_setting": "ce:0:0" if ce else args.gemm_swap,
             "swap_max_ctas": None if ce else int(args.gemm_swap.split(":")[2]),
+            "swap_pace_mbps": None if ce else gemm_pace_mbps(args),
             # MPRESS_OPT_PDL 1 (default) launches a capped grid without PDL
             "swap_pdl_mode": ctx.get_option(mp.OPT_PDL),
             "swap_gbs_during": statistics.median(swap_gbs),
@@ -1046,7 +1061,7 @@ def cfg5_leg(args, mp, rank, n, device, dist, ce=False):
                 st["pl"] = mp.plan(n, rank, rem, bwm[rank], sizes)
             for p in range(n):
                 rem[p] -= part[s][p]
-        set_gemm_swap(ctx, mp, "ce:0:0" if ce else args.gemm_swap)
+        set_gemm_swap(ctx, mp, "ce:0:0" if ce else args.gemm_swap, 0 if ce else gemm_pace_mbps(args))
         st["a"] = torch.randn(M, M, dtype=torch.bfloat16, device="cuda")
         st["b"] = torch.randn(M, M, dtype=torch.bfloat16, device="cuda")
         st["c"] = torch.empty(M, M, dtype=torch.bfloat16, device="cuda")
@@ -1142,6 +1157,7 @@ def cfg5_leg(args, mp, rank, n, device, dist, ce=False):
                       "sets (900 MiB each, one plan), bf16 %dx%dx%d GEMMs on every rank" %
                       (sources, peers, [H - s for s in sources], M, M, M),
             "swap_setting": "ce:0:0" if ce else args.gemm_swap,
+            "swap_pace_mbps": None if ce else gemm_pace_mbps(args),
             "per_source_gbs": [float(row[s, 2]) for s in sources],
             "per_source_bytes": [sum(workloads.cfg2_sizes(H - s)) for s in sources],
             "gemm_alone_ms": [float(row[r, 0]) for r in range(n)],

@@ -447,9 +447,9 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
  * with a GEMM CTA);
  * copy engines: 0 = cudaMemcpyAsync per stripe on one side stream per peer
  * (the only copy-engine variant);
- * MPRESS_VARIANT_AUTO (-1, default) = direct 7 when the grid is capped at
- * <= one CTA per SM (small CTAs co-reside with a GEMM), else 5; bulk 3; copy
- * engines 0.
+ * MPRESS_VARIANT_AUTO (-1, default) = direct 9 when the grid is capped at
+ * <= one CTA per SM (128-thread CTAs co-reside with a GEMM), else 5; bulk 3;
+ * copy engines 0.
  * MPRESS_OPT_ORDER: chunk order inside one launch -- 0 = interleave the
  * peers by a weighted round robin, so every peer link carries its share of
  * the swap at every moment (default; needed when several sources share

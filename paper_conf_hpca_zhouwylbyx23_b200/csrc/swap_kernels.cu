@@ -862,8 +862,12 @@ int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* gr
     // vectors (LDG/STG .256, +1% over 16-byte ones; 16-byte fallback when the
     // data is only 16-byte aligned).  bulk: 3 x 32 KiB, one CTA per SM
     // (profiles/r01/sweep_bulk_variants.jsonl).
+    // Capped: 128 x 8 x 32 B (shape 9), 32 KiB of loads in flight per CTA --
+    // twice shape 7's, which left a 64-CTA swap latency-bound at 1.2 TB/s on
+    // loopback (2x that latency over NVLink); 1.8 TB/s now, ~96 registers x
+    // 128 threads, still beside a GEMM CTA (profiles/r02/capped_*).
     if (path == MPRESS_PATH_DIRECT)
-      variant = (max_ctas > 0 && max_ctas <= sms) ? 7 : 5;
+      variant = (max_ctas > 0 && max_ctas <= sms) ? 9 : 5;
     else
       variant = 3;
   }

@@ -27,6 +27,12 @@ KEYS = [
     "lts__t_bytes.sum", "l1tex__t_bytes.sum",
     "smsp__average_warps_issue_stalled_long_scoreboard_per_issue_active.ratio",
     "smsp__pcsamp_warps_issue_stalled_long_scoreboard",
+    "smsp__average_warps_issue_stalled_lg_throttle_per_issue_active.ratio",
+    "smsp__average_warps_issue_stalled_drain_per_issue_active.ratio",
+    "smsp__average_warps_issue_stalled_sleeping_per_issue_active.ratio",
+    "smsp__average_warps_issue_stalled_mio_throttle_per_issue_active.ratio",
+    "smsp__average_warp_latency_per_inst_issued.ratio",
+    "smsp__issue_active.avg.pct_of_peak_sustained_active",
     "nvltx__bytes.sum", "nvlrx__bytes.sum",
 ]
 
