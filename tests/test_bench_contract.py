@@ -1,4 +1,4 @@
-"""The committed bench line (profiles/r01/bench.json, written by bench.py on
+"""The committed bench line (profiles/r02/bench.json, written by bench.py on
 a B200) satisfies the driver's contract: strict JSON, the required keys and
 types, the roofline / cpu_baseline / e2e / clocks objects, and internal
 consistency (value from ms_per_step, roofline frac = achieved / peak)."""
@@ -10,7 +10,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
 def _line():
-    with open(os.path.join(ROOT, "profiles", "r01", "bench.json")) as f:
+    with open(os.path.join(ROOT, "profiles", "r02", "bench.json")) as f:
         text = f.read().strip().splitlines()[-1]
 
     def bad(c):
@@ -39,7 +39,7 @@ def test_internal_consistency():
     assert 0 < r["frac"] <= 1.05
     assert r["traffic"] is None or r["traffic"] > 0
     # value = swapped bytes (out + in) of all micro-batches per step / step time
-    per_step = 2 * d["config"]["micro_batch_bytes"] * d["config"]["micro_batches"] * d["n_gpus"]
+    per_step = 2 * d["config"]["micro_batch_bytes"] * d["config"]["micro_batches"]   # per source GPU
     assert math.isclose(d["value"], per_step / (d["ms_per_step"] / 1e3) / 1e9, rel_tol=1e-6)
     c = d["cpu_baseline"]
     assert c["kind"] == "oracle" and c["cores"] >= 1 and c["value"] > 0
@@ -48,3 +48,19 @@ def test_internal_consistency():
     assert d["clocks"]["sm_mhz"] > 0
     bad = {"hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown"}
     assert not bad & set(d["clocks"]["reasons"])
+
+
+def test_round2_keys():
+    """Round-2 additions: the per-source value with the whole-job sum beside
+    it, the duplex leg, and the GEMM slowdown as a bootstrap interval over
+    >= 30 paired rounds with its regime and the pace of the swap."""
+    d = _line()
+    assert d["per_rank_gbs"] == d["value"] and math.isclose(d["all_ranks_gbs"], d["n_gpus"] * d["value"])
+    assert d["duplex_gbs"] > 0 and d["duplex"]["bit_exact"]
+    for key in ("gemm_slowdown", "gemm_slowdown_ce"):
+        g = d[key]
+        lo, hi = g["slowdown_ci95"]
+        assert lo <= g["slowdown"] <= hi and g["rounds"] >= 30
+        assert g["regime"] in ("burst", "sustained")
+        assert g["meets_10pct"] == (hi < 0.10)
+    assert d["gemm_slowdown"]["swap_pace_mbps"] > 0
