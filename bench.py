@@ -68,9 +68,10 @@ def parse():
                     help="swap grid cap (CTAs = SMs touched) while the concurrent GEMM runs (AUTO path -> "
                          "direct shape 9); 0 = calibrate: the first of --gemm-swap-candidates whose swap rate "
                          "on this run's links reaches --gemm-target-gbs / 0.85")
-    ap.add_argument("--gemm-swap-candidates", default="auto:-1:64,bulk:5:148,auto:-1:96,auto:-1:128,auto:-1:148",
+    ap.add_argument("--gemm-swap-candidates", default="auto:-1:148,auto:-1:96,auto:-1:64,bulk:5:148",
                     help="path:variant:max_ctas settings for the GEMM-concurrent swap, cheapest for the GEMM "
-                         "first (profiles/r01/sweep_gemm_*)")
+                         "first: paced to the same rate, one light CTA on every SM cost the GEMM no more than "
+                         "64 or 96 heavier-loaded SMs (profiles/r02/gemm_leg_settings.jsonl)")
     ap.add_argument("--gemm-target-gbs", type=float, default=720.0,
                     help="per-source swap rate the GEMM-concurrent swap should sustain (BJ:5: 80%% of 900)")
     ap.add_argument("--gemm-no-pace", action="store_true",
@@ -546,7 +547,7 @@ def main():
     duplex = None if args.no_duplex else leg(duplex_leg, ctx, mp, world, source, per_copy, bw, sizes, src, dst,
                                              n, dist)
     cap_cal = None
-    args.gemm_swap = "auto:-1:%d" % (args.gemm_cap if args.gemm_cap > 0 else 64)
+    args.gemm_swap = "auto:-1:%d" % (args.gemm_cap if args.gemm_cap > 0 else 148)
     if not args.no_gemm and args.gemm_cap <= 0:
         cap_cal = calibrate_gemm_cap(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap_stream, n,
                                      dist)
@@ -664,9 +665,29 @@ def other_configs(args, mp, device):
                 if r >= 2:
                     ts.append(e0.elapsed_time(e1))
             ms = statistics.median(ts)
+            # back to back: R round trips enqueued at once, as a pipeline
+            # issues them (the host runs ahead of the GPU, so per-call host
+            # latency hides behind the previous pair's kernels)
+            R = 32 if sum(sizes) <= (64 << 20) else 4
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            h = ctx.swap_out(pl, src, stream=s)     # keeps the GPU busy while the rest is enqueued
+            ctx.swap_in(h, dst, stream=s)
+            hs = [h]
+            e0.record(s)
+            for _ in range(R):
+                h = ctx.swap_out(pl, src, stream=s)
+                ctx.swap_in(h, dst, stream=s)
+                hs.append(h)
+            e1.record(s)
+            torch.cuda.synchronize()
+            for h in hs:
+                h.free()
+            b2b_ms = e0.elapsed_time(e1) / R
             bad = sum(synth_dev.check(t, 1000 * (len(out) + 1), i) for i, t in enumerate(dst))
             row = {"config": name, "bytes": sum(sizes), "stripes": len(pl.stripes),
                    "round_trip_ms": ms, "gbs": 2 * sum(sizes) / (ms / 1e3) / 1e9,
+                   "b2b_round_trip_ms": b2b_ms, "b2b_gbs": 2 * sum(sizes) / (b2b_ms / 1e3) / 1e9,
                    "bit_exact": bad == 0}
             if sum(sizes) <= 256 << 20:
                 row.update(graph_round_trip(ctx, mp, pl, src, dst, s, synth_dev, 1000 * (len(out) + 1)))
@@ -805,10 +826,11 @@ def calibrate_gemm_cap(args, ctx, mp, world, source, per_copy, bw, sizes, src, d
     loopback at N = 1, NVLink at N > 1, where every remote access pays ~2x
     the latency, so a setting keeps fewer bytes in flight per µs): every
     candidate of --gemm-swap-candidates (ordered cheapest for the GEMM first:
-    128-thread direct CTAs at 64, small-smem bulk CTAs on every SM, then
-    more direct CTAs) runs alone, out + in, on every rank at once; the first
-    whose slowest rank reaches --gemm-target-gbs / 0.85 (headroom for the
-    GEMM's contention) is chosen, else the fastest.  Collective: every rank
+    one 128-thread direct CTA on every SM, then 96 and 64 of them, then
+    small-smem bulk CTAs) runs alone and unpaced, out + in, on every rank at
+    once; the first whose slowest rank reaches --gemm-target-gbs / 0.85
+    (headroom for the GEMM's contention) is chosen, else the fastest.  The
+    GEMM leg then paces the chosen setting to that rate (gemm_pace_mbps).  Collective: every rank
     reaches every barrier and reduction even if its own work fails."""
     import torch
     specs = [c.strip() for c in args.gemm_swap_candidates.split(",") if c.strip()]
@@ -853,7 +875,7 @@ def calibrate_gemm_cap(args, ctx, mp, world, source, per_copy, bw, sizes, src, d
     need = args.gemm_target_gbs / 0.85
     ok = [c for c in specs if table[c] >= need]
     if err is not None:
-        chosen = "auto:-1:64"
+        chosen = "auto:-1:148"
     else:
         chosen = ok[0] if ok else max(specs, key=lambda c: table[c])
     return {"chosen": chosen, "target_gbs": args.gemm_target_gbs, "needed_alone_gbs": need,
