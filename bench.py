@@ -878,8 +878,20 @@ def calibrate_gemm_cap(args, ctx, mp, world, source, per_copy, bw, sizes, src, d
         chosen = "auto:-1:148"
     else:
         chosen = ok[0] if ok else max(specs, key=lambda c: table[c])
+    # the chosen setting's capability against its link roofline: loopback
+    # moves 2 B of HBM per swapped byte (measured copy peak), NVLink 1 B per
+    # direction (the guide's 770 GB/s)
+    peaks, _ = measured_peaks()
+    cap_gbs = table.get(chosen, 0.0)
+    if n == 1:
+        roof = {"bound": "hbm", "achieved": 2 * cap_gbs, "peak": float(peaks.get("hbm_gbs", FALLBACK_HBM)),
+                "unit": "GB/s", "what": "HBM traffic of the chosen capped swap running alone (out + in)"}
+    else:
+        roof = {"bound": "nvlink", "achieved": cap_gbs, "peak": NVLINK_GUIDE, "unit": "GB/s",
+                "what": "swapped bytes per second of the chosen capped swap alone, per source"}
+    roof["frac"] = roof["achieved"] / roof["peak"] if roof["peak"] else None
     return {"chosen": chosen, "target_gbs": args.gemm_target_gbs, "needed_alone_gbs": need,
-            "alone_gbs_min_over_ranks": table, "error": err}
+            "alone_gbs_min_over_ranks": table, "chosen_roofline": roof, "error": err}
 
 
 def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap, n, dist, ce=False):
@@ -1266,21 +1278,31 @@ def single_source_leg(args, mp, rank, n, device, dist):
                      "swap-out and swap-in timed separately" % sorted({r["peers"] for r in rows}),
            "unit": "GB/s (tensor bytes / time, one NVLink direction)", "rows": rows, "error": err,
            "all_bit_exact": all(r["bit_exact"] for r in rows) if rows else None}
-    # the north-star point: N-1 peers, >= 256 MiB, best SM path, min of out / in
-    head = [r for r in rows if r["peers"] == n - 1 and r["bytes"] >= (256 << 20) and r["path"] != "ce"]
-    if head:
-        best = {}
-        for r in head:
-            v = min(r["out_gbs"], r["in_gbs"])
-            if v > best.get(r["bytes"], (0, None))[0]:
-                best[r["bytes"]] = (v, r["path"])
-        worst = min(v for v, _ in best.values())
-        out["north_star"] = {"peers": n - 1, "sizes": sorted(best), "best_sm_path_per_size":
-                             {str(k): v[1] for k, v in sorted(best.items())},
-                             "min_gbs_over_sizes_and_directions": worst,
-                             "frac_of_900": worst / NVLINK_NOMINAL, "target_frac": 0.8,
-                             "meets_target": worst >= 0.8 * NVLINK_NOMINAL}
+    ns = north_star_summary(rows, n)
+    if ns is not None:
+        out["north_star"] = ns
     return out
+
+
+def north_star_summary(rows, n):
+    """BASELINE.json's target on config 4's rows: at N GPUs, one source
+    striping to its N-1 peers, tensors >= 256 MiB, the better SM kernel per
+    size, the slower of swap-out and swap-in -- the minimum of that over the
+    sizes against 80% of 900 GB/s.  None when no such row was measured."""
+    head = [r for r in rows if r["peers"] == n - 1 and r["bytes"] >= (256 << 20) and r["path"] != "ce"]
+    if not head:
+        return None
+    best = {}
+    for r in head:
+        v = min(r["out_gbs"], r["in_gbs"])
+        if v > best.get(r["bytes"], (0, None))[0]:
+            best[r["bytes"]] = (v, r["path"])
+    worst = min(v for v, _ in best.values())
+    return {"peers": n - 1, "sizes": sorted(best), "best_sm_path_per_size":
+            {str(k): v[1] for k, v in sorted(best.items())},
+            "min_gbs_over_sizes_and_directions": worst,
+            "frac_of_900": worst / NVLINK_NOMINAL, "target_frac": 0.8,
+            "meets_target": worst >= 0.8 * NVLINK_NOMINAL}
 
 
 def duplex_leg(ctx, mp, world, source, per_copy, bw, sizes, src, dst, n, dist):

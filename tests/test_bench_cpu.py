@@ -68,3 +68,29 @@ def test_bootstrap_ci95():
     assert b.bootstrap_ci95([0.05] * 30) == (0.05, 0.05)
     lo, hi = b.bootstrap_ci95([])
     assert lo != lo and hi != hi                     # NaN when there is nothing to resample
+
+
+def test_north_star_summary():
+    """Config 4's target row (BJ:5, BJ:10): N-1 peers, sizes >= 256 MiB, the
+    better SM kernel per size, the slower direction, min over sizes, against
+    0.8 x 900 GB/s; copy-engine rows and smaller sizes / fewer peers ignored."""
+    b = _bench()
+    M = 1 << 20
+
+    def row(P, size, path, o, i):
+        return {"peers": P, "bytes": size, "path": path, "out_gbs": o, "in_gbs": i}
+    rows = [row(7, 256 * M, "direct", 700, 760), row(7, 256 * M, "bulk", 745, 750),
+            row(7, 1024 * M, "direct", 790, 780), row(7, 1024 * M, "bulk", 770, 800),
+            row(7, 1024 * M, "ce", 890, 890), row(3, 1024 * M, "bulk", 100, 100),
+            row(7, 64 * M, "bulk", 10, 10)]
+    ns = b.north_star_summary(rows, 8)
+    assert ns["sizes"] == [256 * M, 1024 * M]
+    assert ns["best_sm_path_per_size"] == {str(256 * M): "bulk", str(1024 * M): "direct"}
+    assert ns["min_gbs_over_sizes_and_directions"] == 745
+    assert ns["meets_target"] and abs(ns["frac_of_900"] - 745 / 900) < 1e-12
+    rows[1] = row(7, 256 * M, "bulk", 719, 750)
+    ns = b.north_star_summary(rows, 8)
+    assert ns["min_gbs_over_sizes_and_directions"] == 719 and not ns["meets_target"]
+    ns4 = b.north_star_summary(rows, 4)                # N = 4: the 3-peer rows only
+    assert ns4["sizes"] == [1024 * M] and ns4["min_gbs_over_sizes_and_directions"] == 100
+    assert b.north_star_summary(rows, 2) is None       # no 1-peer row >= 256 MiB
