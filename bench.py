@@ -79,6 +79,8 @@ def parse():
                          "with MPRESS_OPT_PACE_MBPS)")
     ap.add_argument("--no-gemm", action="store_true")
     ap.add_argument("--no-gemm-ce", action="store_true", help="skip the copy-engine pass of the GEMM leg")
+    ap.add_argument("--no-gemm-fc1", action="store_true",
+                    help="skip the GEMM leg on config 5's second shape (GPT-10.3B FC1, 4096x5120x20480)")
     ap.add_argument("--gemm-settle-s", type=float, default=2.0,
                     help="back-to-back GEMMs before the GEMM-slowdown rounds (power state)")
     ap.add_argument("--gemm-rounds", type=int, default=40,
@@ -554,6 +556,9 @@ def main():
         args.gemm_swap = cap_cal["chosen"]
     gemm = None if args.no_gemm else leg(gemm_interference, args, ctx, mp, world, source, per_copy, bw,
                                          sizes, src, dst, swap_stream, n, dist)
+    gemm_fc1 = None if (args.no_gemm or args.no_gemm_fc1) else leg(
+        gemm_interference, args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap_stream, n, dist, False,
+        "gpt_fc1")
     gemm_ce = None if (args.no_gemm or args.no_gemm_ce) else leg(
         gemm_interference, args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap_stream, n, dist, True)
     cfg5 = None
@@ -588,6 +593,7 @@ def main():
             "per_direction_gbs": per_dir,
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": launches[0], "clocks": clk, "gemm_slowdown": gemm, "gemm_slowdown_ce": gemm_ce,
+            "gemm_slowdown_gpt_fc1": gemm_fc1,
             "gemm_cap_calibration": cap_cal,
             "planner": planner, "other_configs": others, "cfg5": cfg5, "cfg5_ce": cfg5_ce,
             "single_source": single, "duplex": duplex,
@@ -894,16 +900,24 @@ def calibrate_gemm_cap(args, ctx, mp, world, source, per_copy, bw, sizes, src, d
             "alone_gbs_min_over_ranks": table, "chosen_roofline": roof, "error": err}
 
 
-def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap, n, dist, ce=False):
+GEMM_SHAPES = {"8192^3": (8192, 8192, 8192),
+               # config 5 (ii): the FC1 of config 3's GPT-10.3B at
+               # micro-batch 2 x seq 2048: [4096 x 5120] . [5120 x 20480]
+               "gpt_fc1": (4096, 5120, 20480)}
+
+
+def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap, n, dist, ce=False,
+                      shape="8192^3"):
     """Second half of the metric: slowdown of a bf16 GEMM (8192^3, the shape
-    MEASURED_PEAKS.json is quoted on) on the compute stream while swaps loop on
-    the side stream with the grid capped at --gemm-cap CTAs.  Alone and
-    with-swap rounds alternate (so power-cap drift hits both), and only GEMMs
-    that ran entirely inside the swap window count.  ce=True: the same with
-    the copy-engine comparator (a7, no SMs) moving the swap."""
+    MEASURED_PEAKS.json is quoted on, or config 5's GPT FC1 stage GEMM) on the
+    compute stream while swaps loop on the side stream with the grid capped
+    at --gemm-cap CTAs.  Alone and with-swap rounds alternate (so power-cap
+    drift hits both), and only GEMMs that ran entirely inside the swap window
+    count.  ce=True: the same with the copy-engine comparator (a7, no SMs)
+    moving the swap."""
     import torch
     comp = torch.cuda.current_stream()
-    M = K = N = 8192
+    M, K, N = GEMM_SHAPES[shape]
     G = 24
     L = _Local()
     st = {}
@@ -1015,7 +1029,7 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
     regime = None
     if burst and sus:
         regime = "sustained" if a_tflops < (burst + sus) / 2 else "burst"
-    return {"gemm": "bf16 8192x8192x8192 torch.matmul (cuBLAS) on the compute stream",
+    return {"gemm": "bf16 %dx%dx%d torch.matmul (cuBLAS) on the compute stream" % (M, K, N), "shape": shape,
             "alone_ms": a_ms, "with_swap_ms": d_ms,
             "alone_tflops": a_tflops,
             "regime": regime,
@@ -1209,7 +1223,7 @@ def single_source_leg(args, mp, rank, n, device, dist):
     first P peers, P in {1, 3, N-1}, over NVLink, for every size of
     --ss-sizes and every transfer path (direct kernel, bulk/TMA kernel, copy
     engines), swap-out and swap-in timed separately (CUDA events on the swap
-    stream, median of `reps` after one warm-up pair).  GB/s = tensor bytes /
+    stream, median of 20 reps -- 5 from 256 MiB -- after 3 warm-up pairs).  GB/s = tensor bytes /
     time, i.e. one direction of NVLink per byte, reported as a fraction of the
     900 GB/s nominal and of the guide's 770 GB/s.  The other ranks are passive
     importers (their pools are mapped by rank 0).  The restored tensor is
@@ -1246,7 +1260,7 @@ def single_source_leg(args, mp, rank, n, device, dist):
                         b.zero_()
                         reps = 20 if size < (256 << 20) else 5
                         to, ti = [], []
-                        for r in range(reps + 1):
+                        for r in range(reps + 3):                      # 3 warm-ups
                             e = [torch.cuda.Event(enable_timing=True) for _ in range(3)]
                             e[0].record(swap)
                             h = ctx.swap_out(pl, [a], stream=swap)
@@ -1255,7 +1269,7 @@ def single_source_leg(args, mp, rank, n, device, dist):
                             e[2].record(swap)
                             torch.cuda.synchronize()
                             h.free()
-                            if r:
+                            if r >= 3:
                                 to.append(e[0].elapsed_time(e[1]))
                                 ti.append(e[1].elapsed_time(e[2]))
                         mo, mi = statistics.median(to), statistics.median(ti)
