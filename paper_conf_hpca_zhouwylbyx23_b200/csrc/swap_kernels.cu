@@ -206,18 +206,33 @@ __device__ __forceinline__ void st_stream(V8* p, const V8& r) {
                   "r"(r.v[6]), "r"(r.v[7]) : "memory");
 }
 
-// One vector load of width VB (16 or 32 bytes); HINT = L2 evict-first (32 only).
+// 32-byte store whose L2 lines are marked evict-first (a createpolicy cache
+// hint: st has no L2 eviction-priority qualifier), so a swap streaming
+// through L2 beside a GEMM does not push the GEMM's tiles out.
+__device__ __forceinline__ void st_stream_ef(V8* p, const V8& r, uint64_t pol) {
+  asm volatile("st.global.L1::no_allocate.L2::cache_hint.v8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8}, %9;"
+               :: "l"(p), "r"(r.v[0]), "r"(r.v[1]), "r"(r.v[2]), "r"(r.v[3]), "r"(r.v[4]), "r"(r.v[5]),
+                  "r"(r.v[6]), "r"(r.v[7]), "l"(pol) : "memory");
+}
+
+// One vector load / store of width VB (16 or 32 bytes); HINT (32 only) = L2
+// evict-first on the loads and on the stores.
 template <int VB, bool HINT>
 struct Vec;
 template <bool HINT>
 struct Vec<16, HINT> {
   using T = int4;
   static __device__ __forceinline__ T ld(const T* p) { return ld_stream(p); }
+  static __device__ __forceinline__ void st(T* p, const T& v, uint64_t) { st_stream(p, v); }
 };
 template <bool HINT>
 struct Vec<32, HINT> {
   using T = V8;
   static __device__ __forceinline__ T ld(const T* p) { return ld_stream<HINT>(p); }
+  static __device__ __forceinline__ void st(T* p, const T& v, uint64_t pol) {
+    if (HINT) st_stream_ef(p, v, pol);
+    else st_stream(p, v);
+  }
 };
 
 // Programmatic dependent launch (PDL): a swap kernel is launched with
@@ -297,6 +312,8 @@ __device__ __forceinline__ void direct_body(const CopyTable<CAP>& t) {
   if (!cur.next(&c, &s)) return;
   Span sp = span_of<kShift>(t, c, s);
   Pacer pace(t.pace_ns);
+  uint64_t pol = 0;
+  if (HINT && VB == 32) asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
   for (;;) {
     Span nx{nullptr, nullptr, 0};
     bool more = false;
@@ -312,7 +329,7 @@ __device__ __forceinline__ void direct_body(const CopyTable<CAP>& t) {
         if (more) nx = span_of<kShift>(t, c, s);
       }
 #pragma unroll
-      for (int j = 0; j < UNROLL; ++j) st_stream(dv + j * THREADS, r[j]);
+      for (int j = 0; j < UNROLL; ++j) Vec<VB, HINT>::st(dv + j * THREADS, r[j], pol);
       if (!PF) {
         more = cur.next(&c, &s);
         if (more) nx = span_of<kShift>(t, c, s);
@@ -539,13 +556,15 @@ struct Shape {
 // 7 (128,4,32) 8 (256,4,32 + L2 evict-first loads) 9 (128,8,32)
 // 10 (128,16,32) 11 (64,16,32) -- 32 / 64 KiB in flight per CTA with few
 // warps, for a capped grid beside a GEMM (its CTA leaves ~22.5K registers)
+// 12 (128,8,32 + L2 evict-first loads and stores)
 // bulk (piece, stages, CTAs/SM): 0 (32K,6,1) 1 (16K,12,1) 2 (64K,3,1) 3 (32K,3,1)
 // 4 (16K,4,3) 5 (8K,2,1) 6 (4K,3,1) -- 5 and 6 use 16 / 12 KB of shared
 // memory, small enough to sit beside a cuBLAS GEMM CTA (214 KB)
 constexpr Shape kDirect[kDirectVariants] = {
     {256, 15, 0, 2, 16, 0}, {512, 16, 0, 1, 16, 1}, {256, 16, 0, 2, 16, 2}, {1024, 16, 0, 1, 16, 3},
     {128, 14, 0, 4, 16, 4}, {256, 15, 0, 2, 32, 0}, {256, 16, 0, 2, 32, 2}, {128, 14, 0, 4, 32, 4},
-    {256, 15, 0, 2, 32, 0}, {128, 15, 0, 4, 32, 4}, {128, 16, 0, 4, 32, 4}, {64, 15, 0, 8, 32, 4}};
+    {256, 15, 0, 2, 32, 0}, {128, 15, 0, 4, 32, 4}, {128, 16, 0, 4, 32, 4}, {64, 15, 0, 8, 32, 4},
+    {128, 15, 0, 4, 32, 4}};
 constexpr Shape kBulk[kBulkVariants] = {
     {32, 15, 6u << 15, 1, 16, 0}, {32, 14, 12u << 14, 1, 16, 1}, {32, 16, 3u << 16, 1, 16, 2},
     {32, 15, 3u << 15, 1, 16, 3}, {32, 14, 4u << 14, 3, 16, 4}, {32, 13, 2u << 13, 1, 16, 5},
@@ -602,6 +621,7 @@ std::conditional_t<G, KernelFnG<CAP>, KernelFn<CAP>> kernel_for(int path, int va
       case 9: k = MP_DIRECT(128, 8, 32, false); break;
       case 10: k = MP_DIRECT(128, 16, 32, false); break;
       case 11: k = MP_DIRECT(64, 16, 32, false); break;
+      case 12: k = MP_DIRECT(128, 8, 32, true); break;
       default: k = MP_DIRECT(256, 8, 16, false); break;
     }
   }

@@ -268,3 +268,35 @@ def test_split_modes_are_oracle_exact(split, path, variant, cap):
             ctx.set_option(mp.OPT_SPLIT, 2)
     finally:
         ctx.finalize()
+
+
+def test_autotune_waits_for_inflight_swap_in():
+    """a freed IN_PENDING handle leaves its slices fenced by the
+    swap-in's event; mpress_autotune uses the stash as probe scratch and must
+    not write those bytes before that swap-in has read them.  The swap-in's
+    stream is held back by a sleep, the handle freed, autotune run on
+    another stream: the restored tensors must still be the original bytes."""
+    from synth import device as synth_dev
+    world, G = 3, 65536
+    sizes = [8 << 20, 3 << 20]
+    spare, bw = [0, 1 << 30, 1 << 30], [0, 1, 1]
+    pl = mp.plan(world, 0, spare, bw, sizes, G)
+    part = [[0] + [u * G for u in pl.units[1:]], [0] * 3, [0] * 3]   # room for exactly one handle
+    ctx = mp.Context.local(world, 0, [0] * world, part)
+    try:
+        src = [torch.empty(n, dtype=torch.uint8, device="cuda") for n in sizes]
+        for i, t in enumerate(src):
+            synth_dev.fill(t, 61, i)
+        dst = [torch.zeros(n, dtype=torch.uint8, device="cuda") for n in sizes]
+        s_in, s_probe = torch.cuda.Stream(), torch.cuda.Stream()
+        torch.cuda.synchronize()
+        h = ctx.swap_out(pl, src, stream=s_in)
+        with torch.cuda.stream(s_in):
+            torch.cuda._sleep(50_000_000)             # ~25 ms: the swap-in starts late
+        ctx.swap_in(h, dst, stream=s_in)
+        h.free()                                      # IN_PENDING: slices released, fenced
+        ctx.autotune(probe_bytes=sum(sizes), trials=1, stream=s_probe)
+        torch.cuda.synchronize()
+        assert all(synth_dev.check(t, 61, i) == 0 for i, t in enumerate(dst))
+    finally:
+        ctx.finalize()
