@@ -18,3 +18,12 @@ def test_replay_restores_every_byte(S):
     assert r["restored_bytes_wrong"] == 0
     assert r["peak_resident_sets_noswap"] == min(S, 4)
     assert r["measured_stage_ms_swap"] > 0
+
+
+def test_replay_paced_to_live_interval():
+    """The executor's swaps paced to the live interval: every byte
+    still restored, and the scheduler is fed the paced swap times."""
+    import replay_1f1b
+    r = replay_1f1b.replay(4, 0, 4, scale=64, n_fwd_gemms=2, max_ctas=32, pace_frac=0.7)
+    assert r["restored_bytes_wrong"] == 0 and r["pace_mbps"] > 0
+    assert r["t_out_ms"] >= r["micro_batch_bytes"] / (r["pace_mbps"] * 1e3) * 0.99

@@ -55,7 +55,12 @@ def timed(fn, stream, reps=5):
     return statistics.median(ts[1:]) * 1e6  # ns
 
 
-def replay(S, e, M, scale, n_fwd_gemms, max_ctas, seed=7000, slack=0.5):
+def replay(S, e, M, scale, n_fwd_gemms, max_ctas, seed=7000, slack=0.5, pace_frac=0.0):
+    """pace_frac > 0: pace every swap (MPRESS_OPT_PACE_MBPS) so that one
+    micro-batch's swap-out + swap-in takes pace_frac of the shortest live
+    interval of the no-swap timeline (hidden if the live interval
+    exceeds the swap time -- so move no faster than that needs), and give the
+    scheduler those paced swap times."""
     sizes = [max(16, b // scale) for b in workloads.cfg2_sizes(1)]
     world, peers = 4, [1, 2, 3]
     spare = workloads.spare_vector(world, 0, peers, spare=64 << 30)
@@ -97,6 +102,15 @@ def replay(S, e, M, scale, n_fwd_gemms, max_ctas, seed=7000, slack=0.5):
             ins.append(e1.elapsed_time(e2))
         t_out = int(statistics.median(outs[1:]) * 1e6)
         t_in = int(statistics.median(ins[1:]) * 1e6)
+        pace_mbps = 0
+        if pace_frac > 0:
+            live0, _ = mp.schedule_1f1b(S, e, M, t_f, t_b, 0, 0)
+            min_live = min(x["live_ns"] for x in live0)
+            # bytes per ns = GB/s; x1000 = MB/s; never slower than 1 GB/s
+            pace_mbps = max(1000, int(2 * sum(sizes) / (pace_frac * min_live) * 1000))
+            ctx.set_option(mp.OPT_PACE_MBPS, pace_mbps)
+            t_paced = int(sum(sizes) / (pace_mbps / 1000))          # ns per paced launch
+            t_out, t_in = max(t_out, t_paced), max(t_in, t_paced)
 
         # swap-ins keep `slack` x t_in of lead: the swap slows down beside the
         # GEMMs (shared HBM in loopback), so the alone-measured t_in is optimistic
@@ -161,7 +175,7 @@ def replay(S, e, M, scale, n_fwd_gemms, max_ctas, seed=7000, slack=0.5):
         mb = sum(sizes)
         return {
             "stages": S, "stage": e, "micro_batches": M, "micro_batch_bytes": mb,
-            "swap_max_ctas": max_ctas, "swap_in_slack": slack,
+            "swap_max_ctas": max_ctas, "swap_in_slack": slack, "pace_frac": pace_frac, "pace_mbps": pace_mbps,
             "t_fwd_ms": t_f / 1e6, "t_bwd_ms": t_b / 1e6, "t_out_ms": t_out / 1e6, "t_in_ms": t_in / 1e6,
             "swap_gbs_alone": 2 * mb / ((t_out + t_in) / 1e9) / 1e9,
             "live_interval_ms": [s["live_ns"] / 1e6 for s in sched],
@@ -188,11 +202,14 @@ def main():
     ap.add_argument("--fwd-gemms", type=int, default=10)
     ap.add_argument("--max-ctas", type=int, default=64)
     ap.add_argument("--slack", type=float, default=0.5, help="swap-in lead, in units of t_in")
+    ap.add_argument("--pace-frac", type=float, nargs="+", default=[0.0],
+                    help="0 = unpaced; f > 0 = pace each swap so out + in takes f x the shortest live interval")
     args = ap.parse_args()
     for S in args.stages:
-        r = replay(S, 0, args.micro_batches, args.scale, args.fwd_gemms, args.max_ctas,
-                   slack=args.slack)
-        print(json.dumps(r), flush=True)
+        for f in args.pace_frac:
+            r = replay(S, 0, args.micro_batches, args.scale, args.fwd_gemms, args.max_ctas,
+                       slack=args.slack, pace_frac=f)
+            print(json.dumps(r), flush=True)
 
 
 if __name__ == "__main__":
