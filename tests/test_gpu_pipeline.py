@@ -21,7 +21,7 @@ def test_replay_restores_every_byte(S):
 
 
 def test_replay_paced_to_live_interval():
-    """The executor's swaps paced to the live interval: every byte
+    """The executor's swaps paced to the 1F1B period: every byte
     still restored, and the scheduler is fed the paced swap times."""
     import replay_1f1b
     r = replay_1f1b.replay(4, 0, 4, scale=64, n_fwd_gemms=2, max_ctas=32, pace_frac=0.7)

@@ -56,11 +56,13 @@ def timed(fn, stream, reps=5):
 
 
 def replay(S, e, M, scale, n_fwd_gemms, max_ctas, seed=7000, slack=0.5, pace_frac=0.0):
-    """pace_frac > 0: pace every swap (MPRESS_OPT_PACE_MBPS) so that one
-    micro-batch's swap-out + swap-in takes pace_frac of the shortest live
-    interval of the no-swap timeline (hidden if the live interval
-    exceeds the swap time -- so move no faster than that needs), and give the
-    scheduler those paced swap times."""
+    """pace_frac > 0: pace every swap launch (MPRESS_OPT_PACE_MBPS) to take
+    pace_frac of the 1F1B period t_f + t_b, and give the scheduler those
+    paced swap times.  In the steady state the swap-out stream and the
+    swap-in stream each move one micro-batch per period, so the period -- not
+    one micro-batch's live interval -- bounds how slow a swap may be
+    (round-2 finding: pacing to 0.7 of the shortest live interval made the
+    serialised swap-ins miss their backwards)."""
     sizes = [max(16, b // scale) for b in workloads.cfg2_sizes(1)]
     world, peers = 4, [1, 2, 3]
     spare = workloads.spare_vector(world, 0, peers, spare=64 << 30)
@@ -104,10 +106,8 @@ def replay(S, e, M, scale, n_fwd_gemms, max_ctas, seed=7000, slack=0.5, pace_fra
         t_in = int(statistics.median(ins[1:]) * 1e6)
         pace_mbps = 0
         if pace_frac > 0:
-            live0, _ = mp.schedule_1f1b(S, e, M, t_f, t_b, 0, 0)
-            min_live = min(x["live_ns"] for x in live0)
             # bytes per ns = GB/s; x1000 = MB/s; never slower than 1 GB/s
-            pace_mbps = max(1000, int(2 * sum(sizes) / (pace_frac * min_live) * 1000))
+            pace_mbps = max(1000, int(sum(sizes) / (pace_frac * (t_f + t_b)) * 1000))
             ctx.set_option(mp.OPT_PACE_MBPS, pace_mbps)
             t_paced = int(sum(sizes) / (pace_mbps / 1000))          # ns per paced launch
             t_out, t_in = max(t_out, t_paced), max(t_in, t_paced)
@@ -203,7 +203,7 @@ def main():
     ap.add_argument("--max-ctas", type=int, default=64)
     ap.add_argument("--slack", type=float, default=0.5, help="swap-in lead, in units of t_in")
     ap.add_argument("--pace-frac", type=float, nargs="+", default=[0.0],
-                    help="0 = unpaced; f > 0 = pace each swap so out + in takes f x the shortest live interval")
+                    help="0 = unpaced; f > 0 = pace each swap launch to take f x the 1F1B period t_f + t_b")
     args = ap.parse_args()
     for S in args.stages:
         for f in args.pace_frac:
