@@ -473,7 +473,11 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
  * finishes within its tensor's live interval (fn.1 P:226), so a swap
  * beside compute needs only bytes / live-interval; pacing it there leaves
  * the rest of HBM, L2 and the issue slots to the compute.  Not applied to
- * the copy-engine path. */
+ * the copy-engine path.  A paced launch keeps its CTAs resident (sleeping)
+ * for longer, and a paced swap-out keeps its source tensors in use for
+ * longer: pace a swap beside a long kernel whose CTAs co-reside with the
+ * swap's, not a swap-out that should free memory at once (DESIGN.md §7c,
+ * NEXT-2 replay). */
 #define MPRESS_OPT_PACE_MBPS 12
 /* MPRESS_OPT_SPLIT: how one launch's chunks (interleaved over the peers, see
  * MPRESS_OPT_ORDER) are shared by its CTAs -- MPRESS_SPLIT_BLOCKED (0,
