@@ -16,6 +16,11 @@ def test_replay_restores_every_byte(S):
     import replay_1f1b
     r = replay_1f1b.replay(S, 0, 4, scale=64, n_fwd_gemms=2, max_ctas=32)
     assert r["restored_bytes_wrong"] == 0
+    # the schedule the native executor ran is the oracle's for the measured times
+    from oracle import pipeline as P
+    q = r["schedule_params_ns"]
+    assert P.schedule(S, 0, 4, q["t_fwd"], q["t_bwd"], q["t_out"], q["t_in"], slack=q["slack"]) == \
+        (r["schedule_slots"], r["schedule_summary"])
     assert r["peak_resident_sets_noswap"] == min(S, 4)
     assert r["measured_stage_ms_swap"] > 0
 

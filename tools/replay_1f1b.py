@@ -177,6 +177,9 @@ def replay(S, e, M, scale, n_fwd_gemms, max_ctas, seed=7000, slack=0.5, pace_fra
             "stages": S, "stage": e, "micro_batches": M, "micro_batch_bytes": mb,
             "swap_max_ctas": max_ctas, "swap_in_slack": slack, "pace_frac": pace_frac, "pace_mbps": pace_mbps,
             "t_fwd_ms": t_f / 1e6, "t_bwd_ms": t_b / 1e6, "t_out_ms": t_out / 1e6, "t_in_ms": t_in / 1e6,
+            "schedule_params_ns": {"t_fwd": t_f, "t_bwd": t_b, "t_out": t_out, "t_in": t_in,
+                                   "slack": int(slack * t_in)},
+            "schedule_slots": sched, "schedule_summary": summ,
             "swap_gbs_alone": 2 * mb / ((t_out + t_in) / 1e9) / 1e9,
             "live_interval_ms": [s["live_ns"] / 1e6 for s in sched],
             "predicted_hidden": sum(s["hidden"] for s in sched),
