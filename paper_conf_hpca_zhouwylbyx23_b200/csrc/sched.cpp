@@ -149,9 +149,7 @@ int run_copy(mpress_ctx_s* c, int dir, const std::vector<CopyDesc>& d,
     // MPRESS_AUTO_SMALL_BYTES, bulk above -- TMA, +0.8% on B200 loopback);
     // direct when the grid is capped to <= one CTA per SM (small CTAs that
     // co-reside with a GEMM) or a peer is pinned host memory
-    int dev = 0, sms = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const int sms = sm_count(nullptr);
     const bool capped = c->max_ctas > 0 && c->max_ctas <= sms;
     uint64_t total = 0;
     for (const CopyDesc& x : d) total += x.len;

@@ -36,6 +36,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <atomic>
 #include <cstddef>
 #include <type_traits>
 #include <mutex>
@@ -778,6 +779,25 @@ int launch_batch_ring(TableRing* r, int path, int variant, int dir, const CopyDe
 
 }  // namespace
 
+int sm_count(int* dev_out) {
+  // per device, queried once (every swap call needs it: grid caps, PDL and
+  // the AUTO path depend on "capped to <= one CTA per SM")
+  static std::atomic<int> cache[64];
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) return 0;
+  if (dev_out) *dev_out = dev;
+  if (dev < 0 || dev >= 64) {
+    int sms = 0;
+    return cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) == cudaSuccess ? sms : 0;
+  }
+  int sms = cache[dev].load(std::memory_order_relaxed);
+  if (sms == 0) {
+    if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) return 0;
+    cache[dev].store(sms, std::memory_order_relaxed);
+  }
+  return sms;
+}
+
 int copy_wave_ctas(int path, int variant) {
   int dev = 0;
   if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return 0;
@@ -864,9 +884,8 @@ void table_ring_destroy(TableRing* r) {
 int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* group, size_t n,
                 int max_ctas, int pdl_mode, cudaStream_t stream, int* launches, TableRing* ring,
                 uint64_t pace_mbps, int split) {
-  int dev = 0, sms = 0;
-  if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess)
-    return fail(MPRESS_ERR_CUDA, "cannot query the SM count");
+  const int sms = sm_count(nullptr);
+  if (sms <= 0) return fail(MPRESS_ERR_CUDA, "cannot query the SM count");
   // PDL (MPRESS_OPT_PDL): mode 1 only for an uncapped grid.  A capped swap
   // runs beside a GEMM, and there a PDL chain of swap kernels (the next one
   // launched early, parked in griddepcontrol.wait) cost the concurrent cuBLAS

@@ -63,6 +63,10 @@ int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* gr
                 cudaStream_t stream, int* launches, TableRing* ring = nullptr, uint64_t pace_mbps = 0,
                 int split = 0);
 
+// SM count of the current device (cached per device; 0 on error); *dev = the
+// device ordinal if dev is not null.
+int sm_count(int* dev);
+
 // Default grid of a path/variant on the current device (SMs x CTAs per SM).
 int copy_wave_ctas(int path, int variant);
 
