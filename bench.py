@@ -18,7 +18,8 @@ in flight = 7.03 GiB) striped over 3 light-load peers.
   * N > 1 (torchrun, one process per GPU): every rank is a source striping
     its batch over all N-1 other ranks and an importer for theirs
     (mpress_init: POSIX-fd pool exchange + cuMemMap peer access over
-    NVLink); value = all ranks' swapped bytes / max-over-ranks time.
+    NVLink); value = one rank's swapped bytes / max-over-ranks time (per
+    source GPU, BASELINE.json's metric); all_ranks_gbs = the whole-job sum.
 value counts swapped tensor bytes, out + in (the round trip of P:332's
 "time cost", reading R15), per second.  Inputs (7 GiB) exceed the 126 MB L2,
 so no flush is needed between steps.
