@@ -33,16 +33,12 @@
 //   (cp.async.bulk, SASS UBLKCP): chunk loads land in a ring of shared-memory
 //   slots (mbarrier completion), then bulk stores drain them, so one SM keeps
 //   STAGES x piece bytes in flight with a single issuing thread.
-#include <cuda.h>
 #include <cuda_runtime.h>
 
 #include <algorithm>
 #include <atomic>
 #include <cstddef>
-#include <cstdlib>
-#include <cstring>
 #include <type_traits>
-#include <unordered_map>
 #include <mutex>
 #include <set>
 #include <utility>
@@ -704,77 +700,9 @@ uint32_t pace_ns_of(uint64_t pace_mbps, uint32_t shift, unsigned grid) {
   return (uint32_t)std::min<uint64_t>(std::max<uint64_t>(ns, 1), 0xFFFFFFFFull);
 }
 
-// Launch through the driver API (cuLaunchKernelEx, reached with
-// cudaGetDriverEntryPoint so the library still loads without a driver):
-// the runtime's cudaLaunchKernelEx spent ~3.6 us of host time per swap call
-// (profiles/r01/hostcost_v3.txt), most of a small swap's cost.
-// MPRESS_LAUNCH=runtime keeps the runtime call (A/B).
-struct DrvLaunch {
-  CUresult (*launch)(const CUlaunchConfig*, CUfunction, void**, void**) = nullptr;
-};
-
-const DrvLaunch& drv_launch() {
-  static const DrvLaunch d = [] {
-    DrvLaunch x;
-    const char* e = getenv("MPRESS_LAUNCH");
-    if (e && strcmp(e, "runtime") == 0) return x;
-    void* fn = nullptr;
-    cudaDriverEntryPointQueryResult q;
-    if (cudaGetDriverEntryPoint("cuLaunchKernelEx", &fn, cudaEnableDefault, &q) == cudaSuccess &&
-        q == cudaDriverEntryPointSuccess && fn)
-      x.launch = reinterpret_cast<CUresult (*)(const CUlaunchConfig*, CUfunction, void**, void**)>(fn);
-    else
-      cudaGetLastError();
-    return x;
-  }();
-  return d;
-}
-
-// The driver handle of a kernel in the current device's context (cached).
-CUfunction func_of(const void* k) {
-  static std::mutex mu;
-  static std::unordered_map<const void*, CUfunction> cache[64];
-  int dev = 0;
-  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return nullptr;
-  std::lock_guard<std::mutex> lk(mu);
-  auto it = cache[dev].find(k);
-  if (it != cache[dev].end()) return it->second;
-  cudaFunction_t f = nullptr;
-  if (cudaGetFuncBySymbol(&f, k) != cudaSuccess || !f) {
-    cudaGetLastError();
-    return nullptr;
-  }
-  cache[dev][k] = reinterpret_cast<CUfunction>(f);
-  return reinterpret_cast<CUfunction>(f);
-}
-
 template <typename K, typename Arg>
 int launch_kernel(K k, const Shape& sh, unsigned grid, bool pdl, cudaStream_t stream, Arg arg) {
   MP_TRY(prepare(k, sh));
-  const DrvLaunch& dl = drv_launch();
-  CUfunction f = dl.launch ? func_of(reinterpret_cast<const void*>(k)) : nullptr;
-  if (f) {
-    CUlaunchConfig cfg;
-    memset(&cfg, 0, sizeof cfg);
-    cfg.gridDimX = grid;
-    cfg.gridDimY = cfg.gridDimZ = 1;
-    cfg.blockDimX = (unsigned)sh.threads;
-    cfg.blockDimY = cfg.blockDimZ = 1;
-    cfg.sharedMemBytes = (unsigned)sh.smem;
-    cfg.hStream = reinterpret_cast<CUstream>(stream);
-    CUlaunchAttribute attr[1];
-    memset(attr, 0, sizeof attr);
-    attr[0].id = CU_LAUNCH_ATTRIBUTE_PROGRAMMATIC_STREAM_SERIALIZATION;
-    attr[0].value.programmaticStreamSerializationAllowed = 1;
-    cfg.attrs = attr;
-    cfg.numAttrs = pdl ? 1 : 0;
-    void* args[1] = {const_cast<void*>(static_cast<const void*>(&arg))};
-    HP_START();
-    const CUresult r = dl.launch(&cfg, f, args, nullptr);
-    HP_LAP(11, "launch: cuLaunchKernelEx");
-    if (r != CUDA_SUCCESS) return fail(MPRESS_ERR_CUDA, "swap kernel launch: CUresult %d", (int)r);
-    return MPRESS_OK;
-  }
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(grid);
   cfg.blockDim = dim3(sh.threads);
