@@ -87,9 +87,10 @@ def parse():
     ap.add_argument("--gemm-rounds", type=int, default=40,
                     help="paired alone / with-swap GEMM rounds (the slowdown's 95%% interval is bootstrapped "
                          "over them)")
-    ap.add_argument("--gemm-sustained-settle-s", type=float, default=3.0,
-                    help="minimum settle of the second 8192^3 GEMM-leg pass, which then goes on (up to 10x) "
-                         "until the GEMM runs in the power-capped sustained regime (0 = skip that pass)")
+    ap.add_argument("--gemm-window", type=int, default=200,
+                    help="GEMMs per window of the sustained-regime GEMM leg (gemm_windows)")
+    ap.add_argument("--gemm-window-rounds", type=int, default=12,
+                    help="alone / with-swap window pairs of the sustained-regime GEMM leg (0 = skip it)")
     ap.add_argument("--gemm-n", type=int, default=8192, help="GEMM size of the N>1 config-5 leg")
     ap.add_argument("--no-cfg5", action="store_true",
                     help="N>1: skip the config-5 leg (imbalanced swap + GEMM on every rank)")
@@ -610,15 +611,8 @@ def main():
         args.gemm_swap = cap_cal["chosen"]
     gemm = None if args.no_gemm else leg(gemm_interference, args, ctx, mp, world, source, per_copy, bw,
                                          sizes, src, dst, swap_stream, n, dist)
-    gemm_sus = None
-    if not (args.no_gemm or args.gemm_sustained_settle_s <= 0):
-        # the same leg after a long back-to-back GEMM settle, so the board sits
-        # at its power cap (the "sustained" regime of MEASURED_PEAKS.json)
-        burst_settle = args.gemm_settle_s
-        args.gemm_settle_s = args.gemm_sustained_settle_s
-        gemm_sus = leg(gemm_interference, args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap_stream,
-                       n, dist, False, "8192^3", True)
-        args.gemm_settle_s = burst_settle
+    gemm_sus = None if (args.no_gemm or args.gemm_window_rounds <= 0) else leg(
+        gemm_windows, args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap_stream, n, dist)
     gemm_fc1 = None if (args.no_gemm or args.no_gemm_fc1) else leg(
         gemm_interference, args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap_stream, n, dist, False,
         "gpt_fc1")
@@ -970,7 +964,7 @@ GEMM_SHAPES = {"8192^3": (8192, 8192, 8192),
 
 
 def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap, n, dist, ce=False,
-                      shape="8192^3", settle_until_sustained=False):
+                      shape="8192^3"):
     """Second half of the metric: slowdown of a bf16 GEMM (8192^3, the shape
     MEASURED_PEAKS.json is quoted on, or config 5's GPT FC1 stage GEMM) on the
     compute stream while swaps loop on the side stream with the grid capped
@@ -1023,28 +1017,13 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
         st["per_swap_ms"] = e0.elapsed_time(e1)
         # Settle the power state first: a B200 runs this GEMM at ~1670 TFLOP/s
         # in a burst and ~1400 sustained (MEASURED_PEAKS.json), and rounds that
-        # straddle the drop mix the two regimes into the ratio.  With
-        # settle_until_sustained (the second 8192^3 pass) the back-to-back
-        # GEMMs go on, up to 10 x the settle time, until one batch runs below
-        # the burst/sustained midpoint -- a fixed 6 s did not get there.
+        # straddle the drop mix the two regimes into the ratio.  (These short
+        # synchronised rounds let the board climb back to burst clocks; the
+        # power-capped regime is gemm_windows'.)
         t0 = time.time()
-        peaks, _ = measured_peaks()
-        mid = None
-        if settle_until_sustained and peaks.get("bf16_tflops") and peaks.get("bf16_tflops_sustained"):
-            mid = (peaks["bf16_tflops"] + peaks["bf16_tflops_sustained"]) / 2
-        while True:
-            evs = gemms()
+        while time.time() - t0 < args.gemm_settle_s:
+            gemms()
             torch.cuda.synchronize()
-            el = time.time() - t0
-            if mid is None:
-                if el >= args.gemm_settle_s:
-                    break
-                continue
-            ms = statistics.median(x.elapsed_time(y) for x, y in evs)
-            st["settle_tflops"] = 2 * M * N * K / (ms / 1e3) / 1e12
-            st["settle_s"] = el
-            if (el >= args.gemm_settle_s and st["settle_tflops"] < mid) or el >= 10 * args.gemm_settle_s:
-                break
 
     ratios = []
 
@@ -1115,8 +1094,7 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
             "regime": regime,
             "regime_rule": "alone TFLOP/s vs the midpoint of MEASURED_PEAKS.json bf16_tflops (burst) and "
                            "bf16_tflops_sustained",
-            "settle_s": st.get("settle_s", args.gemm_settle_s),
-            "settle_last_tflops": st.get("settle_tflops"),
+            "settle_s": args.gemm_settle_s,
             # each round pairs an alone and a with-swap run back to back, so
             # clock / power drift between rounds cancels in the round's ratio
             "slowdown": float(t[3]),
@@ -1139,6 +1117,117 @@ def gemm_interference(args, ctx, mp, world, source, per_copy, bw, sizes, src, ds
             "note": ("N=1 loopback: the swap's bytes also load the GEMM's HBM (2 B per swapped "
                      "byte), a harsher case than NVLink (1 B of source HBM per byte)") if n == 1 else
                     ("every rank swaps to all others while running the GEMM; max over ranks")}
+
+
+def gemm_windows(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap, n, dist):
+    """The GEMM leg in the power-capped ("sustained") regime.  The rounds of
+    gemm_interference synchronise between short GEMM runs, and those gaps let
+    the board climb back to burst clocks; here each round is an alone window
+    of W back-to-back 8192^3 GEMMs followed at once by a with-swap window of
+    W more (the paced capped swap looping beside it, started when the alone
+    window ends), both enqueued before one synchronise, so the GPU stays busy
+    and under its power cap (the protocol of tools/sweep.py power).  The
+    window time / W is the GEMM time; the ratio per round is paired; the
+    interval is bootstrapped over rounds.  After a settle that reaches the
+    sustained regime (below the burst/sustained midpoint)."""
+    import torch
+    comp = torch.cuda.current_stream()
+    M = K = N = 8192
+    W = args.gemm_window
+    L = _Local()
+    st = {}
+    ratios, alone, during, gbs = [], [], [], []
+
+    def setup():
+        st["a"] = torch.randn(M, K, dtype=torch.bfloat16, device="cuda")
+        st["b"] = torch.randn(K, N, dtype=torch.bfloat16, device="cuda")
+        st["c"] = torch.empty(M, N, dtype=torch.bfloat16, device="cuda")
+        st["pl"] = mp.plan(world, source, per_copy, bw, sizes)
+        st["prev"] = set_gemm_swap(ctx, mp, args.gemm_swap, gemm_pace_mbps(args))
+        h = ctx.swap_out(st["pl"], src[0], stream=swap)
+        ctx.swap_in(h, dst[0], stream=swap)
+        h.free()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(swap)
+        h = ctx.swap_out(st["pl"], src[0], stream=swap)
+        ctx.swap_in(h, dst[0], stream=swap)
+        e1.record(swap)
+        h.free()
+        torch.cuda.synchronize()
+        st["per_swap_ms"] = e0.elapsed_time(e1)
+        peaks, _ = measured_peaks()
+        mid = (peaks.get("bf16_tflops", 0) + peaks.get("bf16_tflops_sustained", 0)) / 2 or None
+        t0 = time.time()
+        while True:
+            a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a0.record(comp)
+            for _ in range(W):
+                torch.matmul(st["a"], st["b"], out=st["c"])
+            a1.record(comp)
+            torch.cuda.synchronize()
+            st["settle_tflops"] = 2 * M * N * K * W / (a0.elapsed_time(a1) / 1e3) / 1e12
+            st["settle_s"] = time.time() - t0
+            if (mid is None or st["settle_tflops"] < mid or st["settle_s"] > 30) and st["settle_s"] >= 2.0:
+                break
+
+    def round_():
+        a0, a1, b0, b1 = (torch.cuda.Event(enable_timing=True) for _ in range(4))
+        s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a0.record(comp)
+        for _ in range(W):
+            torch.matmul(st["a"], st["b"], out=st["c"])
+        a1.record(comp)
+        gemm_ms = statistics.median(alone) if alone else 0.8
+        n_swap = int(1.5 * W * gemm_ms / st["per_swap_ms"]) + 2
+        swap.wait_event(a1)                   # the swap window starts when the alone window ends
+        s0.record(swap)
+        for _ in range(n_swap):
+            h = ctx.swap_out(st["pl"], src[0], stream=swap)
+            ctx.swap_in(h, dst[0], stream=swap)
+            h.free()
+        s1.record(swap)
+        b0.record(comp)
+        for _ in range(W):
+            torch.matmul(st["a"], st["b"], out=st["c"])
+        b1.record(comp)
+        torch.cuda.synchronize()
+        a_ms = a0.elapsed_time(a1) / W
+        alone.append(a_ms)
+        if s0.elapsed_time(b0) >= 0 and b1.elapsed_time(s1) >= 0:   # the swap covered the whole window
+            d_ms = b0.elapsed_time(b1) / W
+            during.append(d_ms)
+            ratios.append(d_ms / a_ms - 1)
+            gbs.append(2 * n_swap * sum(sizes) / s0.elapsed_time(s1) / 1e6)
+
+    L(setup)
+    for _ in range(args.gemm_window_rounds):
+        L(round_)
+    if "prev" in st:
+        L(restore_swap, ctx, mp, st["prev"])
+    lo, hi = bootstrap_ci95(ratios)
+    t = torch.tensor([statistics.median(alone) if alone else float("nan"),
+                      statistics.median(during) if during else float("nan"),
+                      1.0 if L.err is not None else 0.0,
+                      statistics.median(ratios) if ratios else float("nan"), lo, hi], dtype=torch.float64)
+    if n > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    if float(t[2]) > 0:
+        return {"error": L.err or "another rank failed"}
+    a_ms = float(t[0])
+    a_tflops = 2 * M * N * K / (a_ms / 1e3) / 1e12
+    peaks, _ = measured_peaks()
+    mid = (peaks.get("bf16_tflops", 0) + peaks.get("bf16_tflops_sustained", 0)) / 2
+    return {"gemm": "bf16 8192x8192x8192 torch.matmul (cuBLAS), windows of %d back to back" % W,
+            "protocol": "per round: alone window then with-swap window, no synchronise between them",
+            "alone_ms": a_ms, "with_swap_ms": float(t[1]), "alone_tflops": a_tflops,
+            "regime": ("sustained" if a_tflops < mid else "burst") if mid else None,
+            "settle_s": st.get("settle_s"), "settle_last_tflops": st.get("settle_tflops"),
+            "slowdown": float(t[3]), "slowdown_ci95": [float(t[4]), float(t[5])],
+            "meets_10pct": float(t[5]) < 0.10, "rounds": len(ratios),
+            "slowdown_per_round": ratios, "swap_setting": args.gemm_swap,
+            "swap_pace_mbps": gemm_pace_mbps(args),
+            "swap_gbs_during": statistics.median(gbs) if gbs else None}
 
 
 def cfg5_leg(args, mp, rank, n, device, dist, ce=False):
