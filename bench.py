@@ -1187,6 +1187,7 @@ def gemm_windows(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, sw
             ctx.swap_in(h, dst[0], stream=swap)
             h.free()
         s1.record(swap)
+        comp.wait_event(s0)                   # the with-swap window starts once the swaps have
         b0.record(comp)
         for _ in range(W):
             torch.matmul(st["a"], st["b"], out=st["c"])
