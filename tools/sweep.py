@@ -8,6 +8,7 @@ keeps the driver's contract; this explains it.
   python tools/sweep.py sizes        # cfg4 sizes 4 KiB .. 4 GiB, 1/3/7 peers
   python tools/sweep.py gemm         # GEMM slowdown vs swap path x cap
   python tools/sweep.py power        # GEMM slowdown vs SM clock and board power
+  python tools/sweep.py windows      # GEMM slowdown in the power-capped regime (bench gemm_windows protocol)
 """
 import json
 import os
@@ -362,6 +363,77 @@ def power():
     ctx.finalize()
 
 
+def windows():
+    """GEMM slowdown in the power-capped regime (bench.py gemm_windows'
+    protocol): per round an alone window of W back-to-back bf16 8192^3 GEMMs,
+    then at once a with-swap window of W more beside the looping swap, one
+    synchronise per round; per setting `rounds` rounds after a settle.
+    WINDOW_COMBOS="direct:9:148:847059;ce:0:0:0" (path:variant:cap:pace)."""
+    import random
+    sizes = workloads.cfg2_sizes(1)
+    nbytes = sum(sizes)
+    ctx, pl, src, dst = setup(sizes, 3)
+    comp = torch.cuda.current_stream()
+    swap = torch.cuda.Stream()
+    M = 8192
+    W = int(os.environ.get("WINDOW", "200"))
+    rounds = int(os.environ.get("WINDOW_ROUNDS", "10"))
+    a = torch.randn(M, M, dtype=torch.bfloat16, device="cuda")
+    b = torch.randn(M, M, dtype=torch.bfloat16, device="cuda")
+    c = torch.empty(M, M, dtype=torch.bfloat16, device="cuda")
+    combos = [x.split(":") for x in os.environ.get(
+        "WINDOW_COMBOS", "direct:9:148:847059;direct:9:148:600000;direct:7:64:0;ce:0:0:0").split(";")]
+    t0 = __import__("time").time()
+    while __import__("time").time() - t0 < 3.0:          # settle into the power-capped regime
+        for _ in range(W):
+            torch.matmul(a, b, out=c)
+        torch.cuda.synchronize()
+    for name, var, cap, pace in combos:
+        ctx.set_option(mp.OPT_PATH, PATHS[name])
+        if name != "ce":
+            ctx.set_option(mp.OPT_VARIANT, int(var))
+        ctx.set_option(mp.OPT_MAX_CTAS, int(cap))
+        ctx.set_option(mp.OPT_PACE_MBPS, int(pace))
+        to, ti = time_swaps(ctx, pl, src, dst, 3, swap)
+        ratios, alone, gbs = [], [], []
+        for _ in range(rounds):
+            ev = [torch.cuda.Event(enable_timing=True) for _ in range(6)]
+            ev[0].record(comp)
+            for _ in range(W):
+                torch.matmul(a, b, out=c)
+            ev[1].record(comp)
+            gemm_ms = statistics.median(alone) if alone else 0.8
+            n_swap = int(1.5 * W * gemm_ms / (to + ti)) + 2
+            swap.wait_event(ev[1])
+            ev[2].record(swap)
+            for _ in range(n_swap):
+                h = ctx.swap_out(pl, src, stream=swap)
+                ctx.swap_in(h, dst, stream=swap)
+                h.free()
+            ev[3].record(swap)
+            comp.wait_event(ev[2])
+            ev[4].record(comp)
+            for _ in range(W):
+                torch.matmul(a, b, out=c)
+            ev[5].record(comp)
+            torch.cuda.synchronize()
+            am = ev[0].elapsed_time(ev[1]) / W
+            alone.append(am)
+            if ev[5].elapsed_time(ev[3]) >= 0:
+                ratios.append(ev[4].elapsed_time(ev[5]) / W / am - 1)
+                gbs.append(2 * n_swap * nbytes / ev[2].elapsed_time(ev[3]) / 1e6)
+        rng = random.Random(0)
+        meds = sorted(statistics.median(rng.choices(ratios, k=len(ratios))) for _ in range(2000)) if ratios else []
+        print(json.dumps({"sweep": "windows", "path": name, "variant": int(var), "max_ctas": int(cap),
+                          "pace_mbps": int(pace), "window": W, "rounds": len(ratios),
+                          "alone_tflops": 2 * M ** 3 / (statistics.median(alone) / 1e3) / 1e12,
+                          "slowdown": statistics.median(ratios) if ratios else None,
+                          "ci95": [meds[49], meds[1949]] if meds else None,
+                          "swap_gbs_during": statistics.median(gbs) if gbs else None,
+                          "swap_alone_gbs": 2 * nbytes / (to + ti) / 1e6}), flush=True)
+    ctx.finalize()
+
+
 if __name__ == "__main__":
     what = sys.argv[1] if len(sys.argv) > 1 else "paths"
-    {"paths": paths, "sizes": sizes_sweep, "gemm": gemm, "host": host, "power": power}[what]()
+    {"paths": paths, "sizes": sizes_sweep, "gemm": gemm, "host": host, "power": power, "windows": windows}[what]()
