@@ -438,7 +438,8 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
  * threads x 8 vectors (2 CTAs/SM by default), 1 = 512x8, 2 = 256x16,
  * 3 = 1024x4, 4 = 128x8 (16-byte vectors), 5 = 256x4, 6 = 256x8, 7 = 128x4,
  * 8 = 256x4 with L2 evict-first loads and stores, 9 = 128x8, 10 = 128x16, 11 = 64x16,
- * 12 = 128x8 with L2 evict-first loads and stores (32-byte vectors, used
+ * 12 = 128x8 with L2 evict-first loads and stores, 13 = 32x16 (one warp)
+ * (32-byte vectors, used
  * only when every address is 32-byte aligned, else the 16-byte shape);
  * bulk: 0 = 6 slots x 32 KiB, 1 = 12 x 16 KiB, 2 = 3 x 64 KiB (one CTA per
  * SM), 3 = 3 x 32 KiB (one per SM; twice as many fit), 4 = 4 x 16 KiB (three

@@ -557,7 +557,8 @@ struct Shape {
 // 7 (128,4,32) 8 (256,4,32 + L2 evict-first loads) 9 (128,8,32)
 // 10 (128,16,32) 11 (64,16,32) -- 32 / 64 KiB in flight per CTA with few
 // warps, for a capped grid beside a GEMM (its CTA leaves ~22.5K registers)
-// 12 (128,8,32 + L2 evict-first loads and stores)
+// 12 (128,8,32 + L2 evict-first loads and stores) 13 (32,16,32: one warp,
+// 16 KiB in flight -- the direct twin of the one-warp bulk shapes)
 // bulk (piece, stages, CTAs/SM): 0 (32K,6,1) 1 (16K,12,1) 2 (64K,3,1) 3 (32K,3,1)
 // 4 (16K,4,3) 5 (8K,2,1) 6 (4K,3,1) -- 5 and 6 use 16 / 12 KB of shared
 // memory, small enough to sit beside a cuBLAS GEMM CTA (214 KB)
@@ -565,7 +566,7 @@ constexpr Shape kDirect[kDirectVariants] = {
     {256, 15, 0, 2, 16, 0}, {512, 16, 0, 1, 16, 1}, {256, 16, 0, 2, 16, 2}, {1024, 16, 0, 1, 16, 3},
     {128, 14, 0, 4, 16, 4}, {256, 15, 0, 2, 32, 0}, {256, 16, 0, 2, 32, 2}, {128, 14, 0, 4, 32, 4},
     {256, 15, 0, 2, 32, 0}, {128, 15, 0, 4, 32, 4}, {128, 16, 0, 4, 32, 4}, {64, 15, 0, 8, 32, 4},
-    {128, 15, 0, 4, 32, 4}};
+    {128, 15, 0, 4, 32, 4}, {32, 14, 0, 8, 32, 4}};
 constexpr Shape kBulk[kBulkVariants] = {
     {32, 15, 6u << 15, 1, 16, 0}, {32, 14, 12u << 14, 1, 16, 1}, {32, 16, 3u << 16, 1, 16, 2},
     {32, 15, 3u << 15, 1, 16, 3}, {32, 14, 4u << 14, 3, 16, 4}, {32, 13, 2u << 13, 1, 16, 5},
@@ -623,6 +624,7 @@ std::conditional_t<G, KernelFnG<CAP>, KernelFn<CAP>> kernel_for(int path, int va
       case 10: k = MP_DIRECT(128, 16, 32, false); break;
       case 11: k = MP_DIRECT(64, 16, 32, false); break;
       case 12: k = MP_DIRECT(128, 8, 32, true); break;
+      case 13: k = MP_DIRECT(32, 16, 32, false); break;
       default: k = MP_DIRECT(256, 8, 16, false); break;
     }
   }

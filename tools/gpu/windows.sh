@@ -1,4 +1,6 @@
-# GEMM slowdown in the power-capped regime, several swap settings and the copy engines
+# GEMM slowdown in the power-capped regime: one-warp direct vs one-warp TMA beside the GEMM
 set -x
-WINDOW_ROUNDS=10 WINDOW_COMBOS="ce:0:0:0;direct:9:148:847059;bulk:5:148:847059;bulk:6:148:847059;bulk:5:74:847059;bulk:3:74:847059;direct:9:148:0;bulk:5:148:0;bulk:5:148:600000;direct:12:148:847059;ce:0:0:0;bulk:5:148:847059;direct:9:148:847059" \
-  timeout 1500 python tools/sweep.py windows > gpurun_out/windows2.jsonl 2> gpurun_out/windows2.err; echo rc $?
+timeout 600 python -m pytest tests/test_gpu_variants.py -m gpu -x -q > gpurun_out/pytest_v13.log 2>&1; echo pytest rc $?
+SWEEP_PATHS=direct SWEEP_VARIANTS=13,11 SWEEP_CAPS=74,148,296 timeout 600 python tools/sweep.py paths > gpurun_out/paths_v13.jsonl 2>&1
+WINDOW_ROUNDS=10 WINDOW_COMBOS="bulk:5:148:847059;direct:13:148:847059;direct:13:148:0;direct:11:148:847059;direct:13:296:847059;bulk:5:148:847059;direct:13:148:847059" \
+  timeout 1500 python tools/sweep.py windows > gpurun_out/windows3.jsonl 2> gpurun_out/windows3.err; echo rc $?
