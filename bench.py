@@ -891,8 +891,9 @@ def calibrate_gemm_cap(args, ctx, mp, world, source, per_copy, bw, sizes, src, d
     loopback at N = 1, NVLink at N > 1, where every remote access pays ~2x
     the latency, so a setting keeps fewer bytes in flight per µs): every
     candidate of --gemm-swap-candidates (ordered cheapest for the GEMM first:
-    one 128-thread direct CTA on every SM, then 96 and 64 of them, then
-    small-smem bulk CTAs) runs alone and unpaced, out + in, on every rank at
+    one-warp TMA CTAs with 16 KB of shared memory on every SM, then one
+    128-thread direct CTA on every SM, then 96 and 64 of them) runs alone and
+    unpaced, out + in, on every rank at
     once; the first whose slowest rank reaches --gemm-target-gbs / 0.85
     (headroom for the GEMM's contention) is chosen, else the fastest.  The
     GEMM leg then paces the chosen setting to that rate (gemm_pace_mbps).  Collective: every rank

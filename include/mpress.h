@@ -441,6 +441,9 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
  * 12 = 128x8 with L2 evict-first loads and stores, 13 = 32x16 (one warp)
  * (32-byte vectors, used
  * only when every address is 32-byte aligned, else the 16-byte shape);
+ * (beside a long bf16 GEMM under the power cap, MPRESS_PATH_BULK shape 5 on
+ * one CTA per SM cost the GEMM ~10% where the direct shapes cost ~17-21% at
+ * the same rate)
  * bulk: 0 = 6 slots x 32 KiB, 1 = 12 x 16 KiB, 2 = 3 x 64 KiB (one CTA per
  * SM), 3 = 3 x 32 KiB (one per SM; twice as many fit), 4 = 4 x 16 KiB (three
  * per SM),
