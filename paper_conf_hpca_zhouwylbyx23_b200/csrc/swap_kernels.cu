@@ -413,6 +413,7 @@ __device__ __forceinline__ void bulk_store(void* gdst, const void* smem, uint32_
 
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_read1() { asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 
 struct Piece {
@@ -451,8 +452,7 @@ __device__ __forceinline__ uint64_t shfl64(uint64_t v, int lane) {
 // <16-byte tail of a descriptor whose last chunk it resolved.  A ring in
 // shared memory remembers each slot's destination for its store.  Order:
 // piece k's load is issued once the store of piece k - STAGES has been read
-// out of its slot, keeping one store in flight behind the newest
-// (wait_group.read 1).
+// out of its slot (wait_group.read 0), so STAGES loads are in flight.
 template <int DIR, int SHIFT, int STAGES, int CAP>
 __device__ __forceinline__ void bulk_body(const CopyTable<CAP>& t) {
   constexpr uint32_t kSlot = 1u << SHIFT;
@@ -509,8 +509,19 @@ __device__ __forceinline__ void bulk_body(const CopyTable<CAP>& t) {
       if (lane == 0) {
         const uint32_t k = loaded;
         if (k >= STAGES) {
+#ifdef MPRESS_BULK_LAZY
           store_until(k - STAGES + 2 <= k ? k - STAGES + 2 : k);  // stores through piece k-STAGES+1
           bulk_wait_read1();  // all but the newest store have left smem: slot of k-STAGES is free
+#else
+          // only the store of piece k-STAGES (the slot's previous piece) is
+          // needed, then its smem read: STAGES loads stay in flight.  Round 1
+          // also stored piece k-STAGES+1 first, to keep one store in flight
+          // behind the newest -- which waited for load k-1 before issuing
+          // load k, leaving a 2-slot ring (shape 5, the one that fits beside
+          // a GEMM) with ~one load in flight.
+          store_until(k - STAGES + 1);
+          bulk_wait_read0();
+#endif
         }
         pace.wait();
         const uint32_t q = k % STAGES;

@@ -19,6 +19,10 @@ bw = workloads.bw_vector(world, 0, peers)
 pl = mp.plan(world, 0, spare, bw, sizes)
 part = [[0] * world for _ in range(world)]; part[0] = [u * 65536 for u in pl.units]
 ctx = mp.Context.local(world, 0, [0] * world, part)
+if os.environ.get("AB_PATH"):   # e.g. "bulk:5" (path:variant); default = AUTO
+    nm, var = os.environ["AB_PATH"].split(":")
+    ctx.set_option(mp.OPT_PATH, {"direct": mp.PATH_DIRECT, "bulk": mp.PATH_BULK}[nm])
+    ctx.set_option(mp.OPT_VARIANT, int(var))
 src = [torch.empty(s, dtype=torch.uint8, device="cuda") for s in sizes]
 for i, t in enumerate(src): synth_dev.fill(t, 1, i)
 dst = [torch.empty(s, dtype=torch.uint8, device="cuda") for s in sizes]
