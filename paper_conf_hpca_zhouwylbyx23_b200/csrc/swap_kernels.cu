@@ -452,10 +452,16 @@ __device__ __forceinline__ uint64_t shfl64(uint64_t v, int lane) {
 // <16-byte tail of a descriptor whose last chunk it resolved.  A ring in
 // shared memory remembers each slot's destination for its store.  Order:
 // piece k's load is issued once the store of piece k - STAGES has been read
-// out of its slot (wait_group.read 0), so STAGES loads are in flight.
+// out of its slot.  Small pieces (<= 4 KiB, kEager): issue only that store
+// and wait for its read (wait_group.read 0), so STAGES loads are in flight --
+// 3 x 4 KiB went from 625 to 1141 GB/s at 148 CTAs.  Larger pieces: also
+// store piece k-STAGES+1 and wait for all but the newest store's read
+// (read 1), keeping a store in flight -- for 3 x 32 KiB waiting on the
+// newest 32 KiB read cost 5% (profiles/r02/bulk_ring_ab.txt).
 template <int DIR, int SHIFT, int STAGES, int CAP>
 __device__ __forceinline__ void bulk_body(const CopyTable<CAP>& t) {
   constexpr uint32_t kSlot = 1u << SHIFT;
+  constexpr bool kEager = SHIFT <= 12;
   extern __shared__ __align__(128) uint8_t smem[];
   __shared__ __align__(8) uint64_t bars[STAGES];
   __shared__ uint8_t* ring_dst[STAGES];
@@ -509,19 +515,17 @@ __device__ __forceinline__ void bulk_body(const CopyTable<CAP>& t) {
       if (lane == 0) {
         const uint32_t k = loaded;
         if (k >= STAGES) {
-#ifdef MPRESS_BULK_LAZY
-          store_until(k - STAGES + 2 <= k ? k - STAGES + 2 : k);  // stores through piece k-STAGES+1
-          bulk_wait_read1();  // all but the newest store have left smem: slot of k-STAGES is free
-#else
-          // only the store of piece k-STAGES (the slot's previous piece) is
-          // needed, then its smem read: STAGES loads stay in flight.  Round 1
-          // also stored piece k-STAGES+1 first, to keep one store in flight
-          // behind the newest -- which waited for load k-1 before issuing
-          // load k, leaving a 2-slot ring (shape 5, the one that fits beside
-          // a GEMM) with ~one load in flight.
-          store_until(k - STAGES + 1);
-          bulk_wait_read0();
-#endif
+          if (kEager) {
+            // only the store of piece k-STAGES (the slot's previous piece),
+            // then its smem read: STAGES loads stay in flight
+            store_until(k - STAGES + 1);
+            bulk_wait_read0();
+          } else {
+            // also store piece k-STAGES+1 and wait only for all but the
+            // newest store's read: one store stays in flight behind it
+            store_until(k - STAGES + 2 <= k ? k - STAGES + 2 : k);  // stores through piece k-STAGES+1
+            bulk_wait_read1();  // all but the newest store have left smem: slot of k-STAGES is free
+          }
         }
         pace.wait();
         const uint32_t q = k % STAGES;
@@ -571,8 +575,9 @@ struct Shape {
 // 12 (128,8,32 + L2 evict-first loads and stores) 13 (32,16,32: one warp,
 // 16 KiB in flight -- the direct twin of the one-warp bulk shapes)
 // bulk (piece, stages, CTAs/SM): 0 (32K,6,1) 1 (16K,12,1) 2 (64K,3,1) 3 (32K,3,1)
-// 4 (16K,4,3) 5 (8K,2,1) 6 (4K,3,1) -- 5 and 6 use 16 / 12 KB of shared
-// memory, small enough to sit beside a cuBLAS GEMM CTA (214 KB)
+// 4 (16K,4,3) 5 (8K,2,1) 6 (4K,3,1) 7 (4K,4,1) -- 5, 6 and 7 use 16 / 12 /
+// 16 KB of shared memory, small enough to sit beside a cuBLAS GEMM CTA
+// (214 KB of the SM's 233.5 KB)
 constexpr Shape kDirect[kDirectVariants] = {
     {256, 15, 0, 2, 16, 0}, {512, 16, 0, 1, 16, 1}, {256, 16, 0, 2, 16, 2}, {1024, 16, 0, 1, 16, 3},
     {128, 14, 0, 4, 16, 4}, {256, 15, 0, 2, 32, 0}, {256, 16, 0, 2, 32, 2}, {128, 14, 0, 4, 32, 4},
@@ -581,7 +586,7 @@ constexpr Shape kDirect[kDirectVariants] = {
 constexpr Shape kBulk[kBulkVariants] = {
     {32, 15, 6u << 15, 1, 16, 0}, {32, 14, 12u << 14, 1, 16, 1}, {32, 16, 3u << 16, 1, 16, 2},
     {32, 15, 3u << 15, 1, 16, 3}, {32, 14, 4u << 14, 3, 16, 4}, {32, 13, 2u << 13, 1, 16, 5},
-    {32, 12, 3u << 12, 1, 16, 6}};
+    {32, 12, 3u << 12, 1, 16, 6}, {32, 12, 4u << 12, 1, 16, 7}};
 
 template <int CAP>
 using KernelFn = void (*)(CopyTable<CAP>);
@@ -619,6 +624,7 @@ std::conditional_t<G, KernelFnG<CAP>, KernelFn<CAP>> kernel_for(int path, int va
       case 4: k = MP_BULK(14, 4); break;
       case 5: k = MP_BULK(13, 2); break;
       case 6: k = MP_BULK(12, 3); break;
+      case 7: k = MP_BULK(12, 4); break;
       default: k = MP_BULK(15, 6); break;
     }
   } else {
