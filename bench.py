@@ -69,11 +69,11 @@ def parse():
                     help="swap grid cap (CTAs = SMs touched) while the concurrent GEMM runs (AUTO path -> "
                          "direct shape 9); 0 = calibrate: the first of --gemm-swap-candidates whose swap rate "
                          "on this run's links reaches --gemm-target-gbs / 0.85")
-    ap.add_argument("--gemm-swap-candidates", default="bulk:5:148,auto:-1:148,auto:-1:96,auto:-1:64",
+    ap.add_argument("--gemm-swap-candidates", default="bulk:7:148,auto:-1:148,auto:-1:96,auto:-1:64",
                     help="path:variant:max_ctas settings for the GEMM-concurrent swap, cheapest for the GEMM "
-                         "first: one-warp TMA CTAs (16 KB of shared memory) on every SM cost the power-capped "
-                         "GEMM ~10%% where 128-thread direct CTAs cost ~17%% at the same rate "
-                         "(profiles/r02/gemm_windows_power_capped.jsonl); among the direct settings one light "
+                         "first: one-warp TMA CTAs (4 x 4 KiB of shared memory) on every SM cost the "
+                         "power-capped GEMM ~12%% where 128-thread direct CTAs cost ~18%% at the same rate "
+                         "(profiles/r02/gemm_windows_*.jsonl); among the direct settings one light "
                          "CTA on every SM cost no more than 64 or 96 busier SMs (gemm_leg_settings.jsonl)")
     ap.add_argument("--gemm-target-gbs", type=float, default=720.0,
                     help="per-source swap rate the GEMM-concurrent swap should sustain (BJ:5: 80%% of 900)")

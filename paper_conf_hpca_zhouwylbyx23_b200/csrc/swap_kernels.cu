@@ -575,8 +575,8 @@ struct Shape {
 // 12 (128,8,32 + L2 evict-first loads and stores) 13 (32,16,32: one warp,
 // 16 KiB in flight -- the direct twin of the one-warp bulk shapes)
 // bulk (piece, stages, CTAs/SM): 0 (32K,6,1) 1 (16K,12,1) 2 (64K,3,1) 3 (32K,3,1)
-// 4 (16K,4,3) 5 (8K,2,1) 6 (4K,3,1) 7 (4K,4,1) -- 5, 6 and 7 use 16 / 12 /
-// 16 KB of shared memory, small enough to sit beside a cuBLAS GEMM CTA
+// 4 (16K,4,3) 5 (8K,2,1) 6 (4K,3,1) 7 (4K,4,1) 8 (2K,8,1) -- 5-8 use 16 / 12 /
+// 16 / 16 KB of shared memory, small enough to sit beside a cuBLAS GEMM CTA
 // (214 KB of the SM's 233.5 KB)
 constexpr Shape kDirect[kDirectVariants] = {
     {256, 15, 0, 2, 16, 0}, {512, 16, 0, 1, 16, 1}, {256, 16, 0, 2, 16, 2}, {1024, 16, 0, 1, 16, 3},
@@ -586,7 +586,7 @@ constexpr Shape kDirect[kDirectVariants] = {
 constexpr Shape kBulk[kBulkVariants] = {
     {32, 15, 6u << 15, 1, 16, 0}, {32, 14, 12u << 14, 1, 16, 1}, {32, 16, 3u << 16, 1, 16, 2},
     {32, 15, 3u << 15, 1, 16, 3}, {32, 14, 4u << 14, 3, 16, 4}, {32, 13, 2u << 13, 1, 16, 5},
-    {32, 12, 3u << 12, 1, 16, 6}, {32, 12, 4u << 12, 1, 16, 7}};
+    {32, 12, 3u << 12, 1, 16, 6}, {32, 12, 4u << 12, 1, 16, 7}, {32, 11, 8u << 11, 1, 16, 8}};
 
 template <int CAP>
 using KernelFn = void (*)(CopyTable<CAP>);
@@ -625,6 +625,7 @@ std::conditional_t<G, KernelFnG<CAP>, KernelFn<CAP>> kernel_for(int path, int va
       case 5: k = MP_BULK(13, 2); break;
       case 6: k = MP_BULK(12, 3); break;
       case 7: k = MP_BULK(12, 4); break;
+      case 8: k = MP_BULK(11, 8); break;
       default: k = MP_BULK(15, 6); break;
     }
   } else {

@@ -68,7 +68,7 @@ def paths():
     nbytes = sum(sizes)
     ctx, pl, src, dst = setup(sizes, 3)
     s = torch.cuda.Stream()
-    nvar = {"direct": 14, "bulk": 8, "ce": 1, "auto": 0}  # plus -1 = auto
+    nvar = {"direct": 14, "bulk": 9, "ce": 1, "auto": 0}  # plus -1 = auto
     only = os.environ.get("SWEEP_PATHS")        # e.g. "direct"
     var_sel = os.environ.get("SWEEP_VARIANTS")  # e.g. "0,5,6,8"
     cap_sel = os.environ.get("SWEEP_CAPS")      # e.g. "0,148,296"
