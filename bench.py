@@ -879,11 +879,19 @@ def restore_swap(ctx, mp, prev):
     ctx.set_option(mp.OPT_PACE_MBPS, prev[3])
 
 
-def gemm_pace_mbps(args):
+def gemm_pace_mbps(args, spec=None):
     """MB/s the GEMM-concurrent SM swap is paced to: the rate the calibration
     asks of it (--gemm-target-gbs / 0.85), so the swap takes only the
-    bandwidth its target needs; 0 with --gemm-no-pace."""
-    return 0 if args.gemm_no_pace else int(round(args.gemm_target_gbs / 0.85 * 1000))
+    bandwidth its target needs -- for the direct (LSU) kernels only,
+    whose cost to the GEMM rises with their rate (+12.8 / +16.1 / +21.9% at
+    381 / 555 / 737 GB/s); the TMA (bulk) kernels cost it about the same
+    paced or not (bulk 7: +11.7% at 670 GB/s paced and at 844 unpaced,
+    profiles/r02/gemm_windows_power_capped_bulk78.jsonl), so they run
+    unpaced and keep the rate.  0 with --gemm-no-pace."""
+    spec = spec if spec is not None else args.gemm_swap
+    if args.gemm_no_pace or spec.split(":")[0] in ("bulk", "ce"):
+        return 0
+    return int(round(args.gemm_target_gbs / 0.85 * 1000))
 
 
 def calibrate_gemm_cap(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap, n, dist):
