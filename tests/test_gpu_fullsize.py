@@ -142,7 +142,8 @@ src = [torch.empty(n, dtype=torch.uint8, device="cuda") for n in sizes]
 for i, t in enumerate(src):
     synth_dev.fill(t, 9, i)
 for path, variant, cap in ((mp.PATH_BULK, 0, 2), (mp.PATH_BULK, 3, 3), (mp.PATH_BULK, 5, 1),
-                           (mp.PATH_DIRECT, 5, 2), (mp.PATH_DIRECT, 7, 3)):
+                           (mp.PATH_BULK, 6, 2), (mp.PATH_BULK, 7, 3), (mp.PATH_BULK, 8, 1),
+                           (mp.PATH_DIRECT, 5, 2), (mp.PATH_DIRECT, 7, 3), (mp.PATH_DIRECT, 13, 2)):
     ctx.set_option(mp.OPT_PATH, path)
     ctx.set_option(mp.OPT_VARIANT, variant)
     ctx.set_option(mp.OPT_MAX_CTAS, cap)
