@@ -28,6 +28,9 @@
  *                       never blocks.
  *   mpress_autotune  -- times the two SM kernels on the context's own links
  *                       and sets the default path per direction and size.
+ *   mpress_set_option -- path, grid cap, kernel shape, chunk order, CTA
+ *                       split, PDL, and rate pacing (a swap hidden in
+ *                       its tensor's live interval needs no more bandwidth).
  *   Beyond the hot path: the multi-source and
  *   global planners, the device-stage mapping search, the 1F1B schedule and
  *   executor, the compaction decision rule, and a pinned host pool as a peer.
