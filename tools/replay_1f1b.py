@@ -55,7 +55,7 @@ def timed(fn, stream, reps=5):
     return statistics.median(ts[1:]) * 1e6  # ns
 
 
-def replay(S, e, M, scale, n_fwd_gemms, max_ctas, seed=7000, slack=0.5, pace_frac=0.0):
+def replay(S, e, M, scale, n_fwd_gemms, max_ctas, seed=7000, slack=0.5, pace_frac=0.0, path="auto:-1"):
     """pace_frac > 0: pace every swap launch (MPRESS_OPT_PACE_MBPS) to take
     pace_frac of the 1F1B period t_f + t_b, and give the scheduler those
     paced swap times.  In the steady state the swap-out stream and the
@@ -72,6 +72,11 @@ def replay(S, e, M, scale, n_fwd_gemms, max_ctas, seed=7000, slack=0.5, pace_fra
     part[0] = [M * u * mp.DEFAULT_GRANULE for u in pl.units]
     ctx = mp.Context.local(world, 0, [0] * world, part)
     ctx.set_option(mp.OPT_MAX_CTAS, max_ctas)
+    pname, pvar = path.split(":")
+    ctx.set_option(mp.OPT_PATH, {"auto": mp.PATH_AUTO, "direct": mp.PATH_DIRECT, "bulk": mp.PATH_BULK,
+                                 "ce": mp.PATH_CE}[pname])
+    if pname in ("direct", "bulk"):
+        ctx.set_option(mp.OPT_VARIANT, int(pvar))
     comp = torch.cuda.current_stream()
     s_out, s_in = torch.cuda.Stream(), torch.cuda.Stream()
     try:
@@ -175,7 +180,8 @@ def replay(S, e, M, scale, n_fwd_gemms, max_ctas, seed=7000, slack=0.5, pace_fra
         mb = sum(sizes)
         return {
             "stages": S, "stage": e, "micro_batches": M, "micro_batch_bytes": mb,
-            "swap_max_ctas": max_ctas, "swap_in_slack": slack, "pace_frac": pace_frac, "pace_mbps": pace_mbps,
+            "swap_max_ctas": max_ctas, "swap_path": path, "swap_in_slack": slack, "pace_frac": pace_frac,
+            "pace_mbps": pace_mbps,
             "t_fwd_ms": t_f / 1e6, "t_bwd_ms": t_b / 1e6, "t_out_ms": t_out / 1e6, "t_in_ms": t_in / 1e6,
             "schedule_params_ns": {"t_fwd": t_f, "t_bwd": t_b, "t_out": t_out, "t_in": t_in,
                                    "slack": int(slack * t_in)},
@@ -205,14 +211,17 @@ def main():
     ap.add_argument("--fwd-gemms", type=int, default=10)
     ap.add_argument("--max-ctas", type=int, default=64)
     ap.add_argument("--slack", type=float, default=0.5, help="swap-in lead, in units of t_in")
+    ap.add_argument("--path", nargs="+", default=["auto:-1"],
+                    help="swap path:variant settings to replay, e.g. auto:-1 bulk:7 ce:0")
     ap.add_argument("--pace-frac", type=float, nargs="+", default=[0.0],
                     help="0 = unpaced; f > 0 = pace each swap launch to take f x the 1F1B period t_f + t_b")
     args = ap.parse_args()
     for S in args.stages:
-        for f in args.pace_frac:
-            r = replay(S, 0, args.micro_batches, args.scale, args.fwd_gemms, args.max_ctas,
-                       slack=args.slack, pace_frac=f)
-            print(json.dumps(r), flush=True)
+        for path in args.path:
+            for f in args.pace_frac:
+                r = replay(S, 0, args.micro_batches, args.scale, args.fwd_gemms, args.max_ctas,
+                           slack=args.slack, pace_frac=f, path=path)
+                print(json.dumps(r), flush=True)
 
 
 if __name__ == "__main__":
