@@ -63,4 +63,8 @@ def test_round2_keys():
         assert lo <= g["slowdown"] <= hi and g["rounds"] >= 30
         assert g["regime"] in ("burst", "sustained")
         assert g["meets_10pct"] == (hi < 0.10)
-    assert d["gemm_slowdown"]["swap_pace_mbps"] > 0
+    # the direct (LSU) GEMM-concurrent swaps are paced, the TMA ones are not
+    g = d["gemm_slowdown"]
+    assert (g["swap_pace_mbps"] > 0) == (g["swap_setting"].split(":")[0] not in ("bulk", "ce"))
+    sus = d["gemm_slowdown_sustained"]
+    assert sus["rounds"] >= 10 and sus["slowdown_ci95"][0] <= sus["slowdown"] <= sus["slowdown_ci95"][1]
