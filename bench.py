@@ -659,6 +659,9 @@ def main():
             "duplex_gbs": duplex.get("duplex_gbs") if isinstance(duplex, dict) else None,
             "parity": "round trip bit-exact vs generator (all %d tensors x %d ranks)" % (47 * mb, n),
             "value_is": "per source GPU: one rank's swapped bytes (out + in) / max-over-ranks step time",
+            "paper_context": "context only, other hardware (BASELINE.md): Table III (P:323-332) D2D swaps of "
+                             "115-1152 MB in 3-27 ms on V100 DGX-1 over 4 NVLink2 links = 72-85 GB/s round trip; "
+                             "GPU-CPU swap 10.3-10.5 GB/s over PCIe3",
             "per_rank_gbs": value,
             "all_ranks_gbs": all_ranks_gbs,
             "transport": {mp.TRANSPORT_LOCAL: "local (mpress_init_local)",
