@@ -300,3 +300,39 @@ def test_autotune_waits_for_inflight_swap_in():
         assert all(synth_dev.check(t, 61, i) == 0 for i, t in enumerate(dst))
     finally:
         ctx.finalize()
+
+
+def test_peer_ptr_errors_and_identity():
+    """mpress_peer_ptr (the device address behind the element-wise stash
+    check): the bytes at the pointer are the ones mpress_peer_read returns;
+    unmapped peers and out-of-range offsets are refused."""
+    import numpy as np
+    from synth import device as synth_dev
+    world = 3
+    sizes = [1 << 20]
+    pl = mp.plan(world, 0, [0, 1 << 30, 0], [0, 1, 0], sizes)
+    part = [[0, 2 << 20, 0], [0] * 3, [0] * 3]
+    ctx = mp.Context.local(world, 0, [0] * world, part)
+    try:
+        src = [torch.empty(sizes[0], dtype=torch.uint8, device="cuda")]
+        synth_dev.fill(src[0], 71, 0)
+        h = ctx.swap_out(pl, src)
+        torch.cuda.synchronize()
+        off = h.slices()[1]
+        p = ctx.peer_ptr(1, off)
+        assert synth_dev.check_ptr(p, sizes[0], 71, 0) == 0
+        assert np.array_equal(np.frombuffer(ctx.peer_read(1, off, 4096), dtype=np.uint8),
+                              src[0][:4096].cpu().numpy())
+        with pytest.raises(mp.MPressError) as ei:
+            ctx.peer_ptr(2, 0)                     # no partition on peer 2
+        assert ei.value.code == mp.ERR_PEER
+        with pytest.raises(mp.MPressError) as ei:
+            ctx.peer_ptr(1, (2 << 20) + 1)         # past the partition
+        assert ei.value.code == mp.ERR_ARG
+        with pytest.raises(mp.MPressError):
+            ctx.peer_ptr(5, 0)
+        ctx.swap_in(h, src)
+        torch.cuda.synchronize()
+        h.free()
+    finally:
+        ctx.finalize()
