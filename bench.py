@@ -641,6 +641,12 @@ def main():
         cpu = leg(oracle_sample, args.cpu_seconds)
         planner = leg(planner_timing, mp, world, source, per_copy, bw, sizes)
 
+    # BASELINE.json's pairing: the swap sustains the target rate (80% of 900
+    # GB/s) beside the GEMM AND the GEMM slows by < 10% (upper 95% bound)
+    for g in (gemm, gemm_ce, gemm_fc1, gemm_sus):
+        if isinstance(g, dict) and g.get("swap_gbs_during") is not None and g.get("slowdown_ci95"):
+            g["meets_rate_target"] = g["swap_gbs_during"] >= args.gemm_target_gbs
+            g["meets_north_star_pair"] = bool(g["meets_rate_target"] and g.get("meets_10pct"))
     if rank == 0:
         line = {
             "metric": "D2D swap GB/s per source GPU (round trip, out+in)",
