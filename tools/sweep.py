@@ -163,11 +163,17 @@ def host():
         synth_dev.fill(src[0], 5, 0)
         dst = [torch.empty(size, dtype=torch.uint8, device="cuda")]
         torch.cuda.synchronize()
-        for name, cap in (("direct", 0), ("direct", 32), ("bulk", 0), ("ce", 0)):
+        combos = [("direct", -1, 0), ("direct", -1, 32), ("bulk", -1, 0), ("ce", 0, 0)]
+        if os.environ.get("HOST_COMBOS"):      # e.g. "bulk:7:148;direct:9:148"
+            combos = [(f[0], int(f[1]), int(f[2])) for f in
+                      (x.split(":") for x in os.environ["HOST_COMBOS"].split(";"))]
+        for name, var, cap in combos:
             ctx.set_option(mp.OPT_PATH, PATHS[name])
+            if name != "ce":
+                ctx.set_option(mp.OPT_VARIANT, var)
             ctx.set_option(mp.OPT_MAX_CTAS, cap)
             to, ti = time_swaps(ctx, pl, src, dst, 4, s)
-            print(json.dumps({"sweep": "host", "bytes": size, "path": name, "max_ctas": cap,
+            print(json.dumps({"sweep": "host", "bytes": size, "path": name, "variant": var, "max_ctas": cap,
                               "out_gbs": size / to / 1e6, "in_gbs": size / ti / 1e6}), flush=True)
         ctx.finalize()
 
