@@ -430,7 +430,9 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
  * MPRESS_AUTO_SMALL_BYTES per launch, bulk above), direct when the grid is
  * capped to <= one CTA per SM (its
  * 128-thread CTAs co-reside with a GEMM, bulk CTAs' shared memory does not)
- * or when a peer is a host pool.
+ * or when the launch mixes device peers and host pools, and the copy
+ * engines when every stripe of the launch goes to a host pool (over PCIe
+ * they beat every SM kernel shape, 56.9 vs 52.6 GB/s).
  * MPRESS_OPT_LAST_PATH (read-only) reports the path the last swap call ran.
  * Setting the path resets the variant to MPRESS_VARIANT_AUTO; under
  * MPRESS_PATH_AUTO only MPRESS_VARIANT_AUTO is accepted.

@@ -148,12 +148,21 @@ int run_copy(mpress_ctx_s* c, int dir, const std::vector<CopyDesc>& d,
     // measured faster on this context's links (before it runs: direct below
     // MPRESS_AUTO_SMALL_BYTES, bulk above -- TMA, +0.8% on B200 loopback);
     // direct when the grid is capped to <= one CTA per SM (small CTAs that
-    // co-reside with a GEMM) or a peer is pinned host memory
+    // co-reside with a GEMM) or the launch mixes device peers and pinned
+    // host pools; the copy engines when every stripe goes to a host pool
+    // (over PCIe every SM kernel shape stops at ~52.6 GB/s, the engines at
+    // ~56.9: profiles/r02/sweep_host_paths.jsonl)
     const int sms = sm_count(nullptr);
     const bool capped = c->max_ctas > 0 && c->max_ctas <= sms;
     uint64_t total = 0;
     for (const CopyDesc& x : d) total += x.len;
-    path = (capped || c->host_peer) ? MPRESS_PATH_DIRECT : c->auto_path[dir][total >= MPRESS_AUTO_SMALL_BYTES];
+    int host = 0;
+    if (c->host_peer)
+      for (int p : desc_peer) host += c->maps[p].host != nullptr;
+    if (host && host == (int)desc_peer.size())
+      path = MPRESS_PATH_CE;
+    else
+      path = (capped || host) ? MPRESS_PATH_DIRECT : c->auto_path[dir][total >= MPRESS_AUTO_SMALL_BYTES];
   }
   c->last_path = path;
   if (path != MPRESS_PATH_CE) {

@@ -88,3 +88,37 @@ def test_autotune_skips_host_pools():
         h.free()
     finally:
         ctx.finalize()
+
+
+def test_auto_picks_copy_engines_for_host_only_launches():
+    """MPRESS_PATH_AUTO per launch (round 2): every stripe to a host pool ->
+    the copy engines (faster than any SM kernel over PCIe); device peers only
+    -> the SM kernels even though the context also has a host pool; mixed ->
+    direct.  Bytes equal the oracle's byte model in all three."""
+    world = 3
+    part_bytes = 64 << 20
+    part = [[0, part_bytes, part_bytes], [0] * 3, [0] * 3]
+    ctx = mp.Context.local(world, 0, [0, 0, mp.DEVICE_HOST], part)
+    try:
+        sizes = [5 << 20, 4097]
+        for bw, want in (([0, 0, 1], mp.PATH_CE), ([0, 1, 0], None), ([0, 900, 55], mp.PATH_DIRECT)):
+            spare = [0, part_bytes if bw[1] else 0, part_bytes if bw[2] else 0]
+            o = oracle.plan(world, 0, spare, bw, sizes)
+            pl = mp.plan(world, 0, spare, bw, sizes)
+            src = U.make_inputs(sizes, 91)
+            h = ctx.swap_out(pl, src)
+            torch.cuda.synchronize()
+            ran = ctx.get_option(mp.OPT_LAST_PATH)
+            if want is None:
+                assert ran in (mp.PATH_DIRECT, mp.PATH_BULK)
+            else:
+                assert ran == want, (bw, ran)
+            U.check_stash(ctx, h, o, U.host_inputs(sizes, 91))
+            dst = [torch.zeros_like(t) for t in src]
+            ctx.swap_in(h, dst)
+            torch.cuda.synchronize()
+            h.free()
+            for d, e in zip(dst, U.host_inputs(sizes, 91)):
+                assert np.array_equal(d.cpu().numpy(), e)
+    finally:
+        ctx.finalize()
