@@ -23,6 +23,17 @@ in flight = 7.03 GiB) striped over 3 light-load peers.
 value counts swapped tensor bytes, out + in (the round trip of P:332's
 "time cost", reading R15), per second.  Inputs (7 GiB) exceed the 126 MB L2,
 so no flush is needed between steps.
+
+Beside the headline (each leg reports its own failure instead of losing the
+line): e2e through pinned host buffers; the duplex leg (two swap streams);
+the GEMM legs -- a calibrated GEMM-concurrent swap setting, then the bf16
+slowdown with a bootstrap 95% interval for 8192^3 (burst rounds and
+power-capped windows), the GPT FC1 stage GEMM and the copy engines, each
+with `meets_north_star_pair` (>= 720 GB/s beside the GEMM and < 10%); at
+N = 1 configs 1, 3 and 4 (single shot, back to back, graph-replayed), the
+oracle's cpu_baseline and the planner timing; at N > 1 config 4's single
+source rows (P = 1, 3, N-1) and config 5 (imbalanced sources + GEMMs on
+every rank).  `--impl reference` times the oracle instead.
 """
 import argparse
 import json
