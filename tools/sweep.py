@@ -291,11 +291,12 @@ def power():
 
     def window(setting):
         if setting:
-            name, var, cap = setting
+            name, var, cap, pace = setting
             ctx.set_option(mp.OPT_PATH, PATHS[name])
             if name != "ce":
                 ctx.set_option(mp.OPT_VARIANT, var)
             ctx.set_option(mp.OPT_MAX_CTAS, cap)
+            ctx.set_option(mp.OPT_PACE_MBPS, pace)
         per_pair = 0.0
         if setting:   # one pair alone sizes the swap batch that covers 20 GEMMs
             torch.cuda.synchronize()
@@ -342,7 +343,7 @@ def power():
         stop.set()
         th.join()
         keep = smp[len(smp) // 5:] or smp   # drop the ramp
-        row = {"sweep": "power", "setting": "alone" if not setting else "%s var=%d cap=%d" % setting,
+        row = {"sweep": "power", "setting": "alone" if not setting else "%s var=%d cap=%d pace=%d" % setting,
                "gemm_tflops": 2 * M ** 3 * n_gemm / (gms / 1e3) / 1e12,
                "sm_mhz_median": statistics.median(x for x, _ in keep),
                "power_w_median": statistics.median(w for _, w in keep), "samples": len(keep)}
@@ -353,12 +354,14 @@ def power():
         return row
 
     window(None)   # warm to the sustained power state
-    settings = [("direct", 7, 32), ("direct", 7, 64), ("direct", 9, 64), ("direct", 7, 148), ("ce", 0, 0)]
-    if os.environ.get("POWER_SETTINGS"):   # e.g. "direct:7:16,32,64;bulk:5:148;ce:0:0"
+    settings = [("direct", 7, 32, 0), ("direct", 7, 64, 0), ("direct", 9, 64, 0), ("direct", 7, 148, 0),
+                ("ce", 0, 0, 0)]
+    if os.environ.get("POWER_SETTINGS"):   # e.g. "direct:7:16,32,64;bulk:5:148;direct:9:148:847059;ce:0:0"
         settings = []
         for part in os.environ["POWER_SETTINGS"].split(";"):
-            nm, v, caps = part.split(":")
-            settings += [(nm, int(v), int(c)) for c in caps.split(",")]
+            f = part.split(":")
+            pace = int(f[3]) if len(f) > 3 else 0
+            settings += [(f[0], int(f[1]), int(c), pace) for c in f[2].split(",")]
     for st in settings:
         al = window(None)
         wi = window(st)
