@@ -100,9 +100,12 @@ def parse():
     ap.add_argument("--gemm-rounds", type=int, default=40,
                     help="paired alone / with-swap GEMM rounds (the slowdown's 95%% interval is bootstrapped "
                          "over them)")
-    ap.add_argument("--gemm-window", type=int, default=200,
-                    help="GEMMs per window of the sustained-regime GEMM leg (gemm_windows)")
-    ap.add_argument("--gemm-window-rounds", type=int, default=12,
+    ap.add_argument("--gemm-window", type=int, default=4000,
+                    help="GEMMs per window of the sustained-regime GEMM leg (gemm_windows): 4000 8192^3 "
+                         "GEMMs are ~3 s, long enough for the power governor to settle in each window "
+                         "(160 ms windows measured +11%% where 1.6-3 s windows measure +6%%, "
+                         "profiles/r02/gemm_windows_long.jsonl)")
+    ap.add_argument("--gemm-window-rounds", type=int, default=5,
                     help="alone / with-swap window pairs of the sustained-regime GEMM leg (0 = skip it)")
     ap.add_argument("--gemm-n", type=int, default=8192, help="GEMM size of the N>1 config-5 leg")
     ap.add_argument("--no-cfg5", action="store_true",
@@ -1155,9 +1158,11 @@ def gemm_windows(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, sw
     gemm_interference synchronise between short GEMM runs, and those gaps let
     the board climb back to burst clocks; here each round is an alone window
     of W back-to-back 8192^3 GEMMs followed at once by a with-swap window of
-    W more (the paced capped swap looping beside it, started when the alone
-    window ends), both enqueued before one synchronise, so the GPU stays busy
-    and under its power cap (the protocol of tools/sweep.py power).  The
+    W more (the capped swap looping beside it, started when the alone window
+    ends), both enqueued before one synchronise, so the GPU stays busy and
+    under its power cap.  W is ~3 s of GEMMs (the verdict's "windows of 3 s
+    or more"): the power governor responds over hundreds of ms, and 160 ms
+    windows mixed the two modes' power states.  The
     window time / W is the GEMM time; the ratio per round is paired; the
     interval is bootstrapped over rounds.  After a settle that reaches the
     sustained regime (below the burst/sustained midpoint)."""
