@@ -217,7 +217,8 @@ def test_bench_cfg5_leg_two_ranks_one_gpu():
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
            "--master-addr=127.0.0.1", "--master-port=%d" % _free_port(), "bench.py", "--gpus", "2",
-           "--steps", "2", "--warmup", "1", "--micro-batches", "1", "--e2e-steps", "1", "--gemm-n", "2048"]
+           "--steps", "2", "--warmup", "1", "--micro-batches", "1", "--e2e-steps", "1", "--gemm-n", "2048",
+           "--gemm-window", "200", "--gemm-window-rounds", "2"]
     r = subprocess.run(cmd, cwd=root, capture_output=True, text=True, timeout=900)
     assert r.returncode == 0, r.stderr[-3000:]
     line = json.loads([l for l in r.stdout.splitlines() if l.startswith("{")][-1])
