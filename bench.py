@@ -75,6 +75,8 @@ def parse():
                     help="MPRESS_OPT_SPLIT: 0 = contiguous block per CTA (default), 1 = grid stride (round 1)")
     ap.add_argument("--e2e-steps", type=int, default=16)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e-zero-copy", action="store_true",
+                    help="skip the e2e variant that hands pinned host tensors to the swap calls")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
     ap.add_argument("--gemm-cap", type=int, default=0,
                     help="swap grid cap (CTAs = SMs touched) while the concurrent GEMM runs (AUTO path -> "
@@ -617,6 +619,8 @@ def main():
             return {"error": "%s: %s" % (type(exc).__name__, exc)}
 
     e2e = leg(run_e2e, args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap_stream, n, dist)
+    e2e_zc = None if args.no_e2e_zero_copy else leg(run_e2e_zero_copy, args, ctx, mp, world, source, per_copy,
+                                                    bw, sizes, n, dist)
     duplex = None if args.no_duplex else leg(duplex_leg, ctx, mp, world, source, per_copy, bw, sizes, src, dst,
                                              n, dist)
     cap_cal = None
@@ -670,7 +674,7 @@ def main():
             "config": workload_config(args, n),
             "swap_path_ran": ran_by_dir, "autotune": autotune,
             "per_direction_gbs": per_dir,
-            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
+            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "e2e_zero_copy": e2e_zc,
             "gpu_launches": launches[0], "clocks": clk, "gemm_slowdown": gemm, "gemm_slowdown_ce": gemm_ce,
             "gemm_slowdown_gpt_fc1": gemm_fc1, "gemm_slowdown_sustained": gemm_sus,
             "gemm_cap_calibration": cap_cal,
@@ -1707,6 +1711,79 @@ def run_e2e(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, stream,
             "pcie": pcie,
             "frac_of_pcie_duplex": ((per / (ms / 1e3) / 1e9) / pcie["duplex_gbs"]
                                     if "duplex_gbs" in pcie else None)}
+
+
+def run_e2e_zero_copy(args, ctx, mp, world, source, per_copy, bw, sizes, n, dist):
+    """The same metric through the C ABI with the HOST buffers themselves as
+    the swap's tensors: pinned host memory is mapped into the device's
+    address space (UVA), so mpress_swap_out reads the micro-batch straight
+    from host memory over PCIe into the peers' stash and mpress_swap_in
+    writes it straight back into host memory -- no device staging buffers,
+    no separate copies.  Pipelined as the duplex leg: the swap-out of
+    micro-batch m+1 (PCIe reads) beside the swap-in of m (PCIe writes) on
+    two streams.  Every restored host byte is compared with the source."""
+    import numpy as np
+    import torch
+    from synth import device as synth_dev
+    mb = 2 if n == 1 else 1
+    nt = len(sizes)
+    L = _Local()
+    st = {}
+
+    def setup():
+        st["hsrc"] = [[torch.empty(x, dtype=torch.uint8, pin_memory=True) for x in sizes] for _ in range(mb)]
+        st["hdst"] = [[torch.empty(x, dtype=torch.uint8, pin_memory=True) for x in sizes] for _ in range(mb)]
+        for m in range(mb):
+            for i in range(nt):
+                t = torch.empty(sizes[i], dtype=torch.uint8, device="cuda")
+                synth_dev.fill(t, 9000 + m, i)
+                st["hsrc"][m][i].copy_(t)
+        st["s_out"], st["s_in"] = torch.cuda.Stream(), torch.cuda.Stream()
+        st["pl"] = mp.plan(world, source, per_copy, bw, sizes)
+
+    def step():
+        s_out, s_in = st["s_out"], st["s_in"]
+        hs = [ctx.swap_out(st["pl"], st["hsrc"][0], stream=s_out)]
+        for m in range(1, mb + 1):
+            if m < mb:
+                hs.append(ctx.swap_out(st["pl"], st["hsrc"][m], stream=s_out))
+            ctx.swap_in(hs[m - 1], st["hdst"][m - 1], stream=s_in)
+        return hs
+
+    def timed():
+        steps = max(1, args.e2e_steps)
+        for h in step():          # warm-up
+            h.free()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(st["s_out"])
+        st["s_in"].wait_stream(st["s_out"])
+        hs = []
+        for _ in range(steps):
+            hs += step()
+        st["s_out"].wait_stream(st["s_in"])
+        e1.record(st["s_out"])
+        torch.cuda.synchronize()
+        for h in hs:
+            h.free()
+        return e0.elapsed_time(e1) / steps
+
+    L(setup)
+    ms = L(timed)
+    t = torch.tensor([ms or 0.0, 1.0 if L.err is not None else 0.0], dtype=torch.float64)
+    if n > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    if float(t[1]) > 0:
+        return {"error": L.err or "another rank failed"}
+    ms = float(t[0])
+    ok = all(np.array_equal(st["hdst"][m][i].numpy(), st["hsrc"][m][i].numpy())
+             for m in range(mb) for i in range(nt))
+    per = 2 * mb * sum(sizes)
+    return {"value": per / (ms / 1e3) / 1e9, "unit": "GB/s", "micro_batches": mb, "ms_per_step": ms,
+            "h2d_bytes_per_step": mb * sum(sizes), "d2h_bytes_per_step": mb * sum(sizes),
+            "round_trip_ok": bool(ok),
+            "how": "pinned host tensors passed to mpress_swap_out / mpress_swap_in (UVA): the swap kernels "
+                   "read and write host memory over PCIe directly; out(m+1) || in(m) on two streams"}
 
 
 def leg_pcie(src, dst, hsrc, hdst, h2d, d2h, stream, reps=3):

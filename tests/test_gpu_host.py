@@ -122,3 +122,35 @@ def test_auto_picks_copy_engines_for_host_only_launches():
                 assert np.array_equal(d.cpu().numpy(), e)
     finally:
         ctx.finalize()
+
+
+@pytest.mark.parametrize("path", [mp.PATH_AUTO, mp.PATH_DIRECT, mp.PATH_BULK, mp.PATH_CE])
+def test_pinned_host_tensors_as_swap_buffers(path):
+    """Zero-copy e2e (bench `e2e_zero_copy`): pinned host tensors handed to
+    mpress_swap_out / mpress_swap_in directly (UVA) -- the kernels read the
+    host memory over PCIe into the device peers' stash and write it back;
+    the stash equals the oracle's byte model and the host round trip is the
+    identity."""
+    world, G = 3, 65536
+    sizes = [(3 << 20) + 48, 70001, 16]
+    spare, bw = [0, 1 << 30, 1 << 30], [0, 1, 2]
+    o = oracle.plan(world, 0, spare, bw, sizes, G)
+    pl = mp.plan(world, 0, spare, bw, sizes, G)
+    part = [[0] + [u * G for u in pl.units[1:]], [0] * 3, [0] * 3]
+    ctx = mp.Context.local(world, 0, [0] * world, part)
+    try:
+        ctx.set_option(mp.OPT_PATH, path)
+        host = U.host_inputs(sizes, 77)
+        hsrc = [torch.from_numpy(h.copy()).pin_memory() for h in host]
+        hdst = [torch.zeros(n, dtype=torch.uint8).pin_memory() for n in sizes]
+        s = torch.cuda.Stream()
+        h = ctx.swap_out(pl, hsrc, stream=s)
+        s.synchronize()
+        U.check_stash(ctx, h, o, host)
+        ctx.swap_in(h, hdst, stream=s)
+        s.synchronize()
+        h.free()
+        for d, e in zip(hdst, host):
+            assert np.array_equal(d.numpy(), e)
+    finally:
+        ctx.finalize()
