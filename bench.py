@@ -1725,7 +1725,7 @@ def run_e2e_zero_copy(args, ctx, mp, world, source, per_copy, bw, sizes, n, dist
     import numpy as np
     import torch
     from synth import device as synth_dev
-    mb = 2 if n == 1 else 1
+    mb = MICRO_BATCHES if n == 1 else 2   # as run_e2e: N ranks on one host do not pin N x 14 GiB
     nt = len(sizes)
     L = _Local()
     st = {}
