@@ -45,6 +45,14 @@ def check(t, seed, tensor_id, start=0, nbytes=None, stream=None):
     return r
 
 
+def fill_ptr(ptr, nbytes, seed, tensor_id, start=0, stream=None):
+    """Write generator bytes [start, start+nbytes) of tensor `tensor_id` at
+    device address `ptr` (e.g. a stash partition, for guard patterns)."""
+    rc = _get().synth_fill(ptr, nbytes, seed, tensor_id, start, _stream(stream))
+    if rc != 0:
+        raise RuntimeError("synth_fill failed: cuda error %d" % rc)
+
+
 def check_ptr(ptr, nbytes, seed, tensor_id, start=0, stream=None):
     """Number of bytes at device address `ptr` (nbytes of them) that differ
     from generator bytes [start, start+nbytes) of tensor `tensor_id`."""
