@@ -71,8 +71,9 @@ def parse():
     ap.add_argument("--pdl", type=int, default=1, choices=[0, 1, 2],
                     help="MPRESS_OPT_PDL: 0 never, 1 uncapped grids only (default), 2 always")
     ap.add_argument("--micro-batches", type=int, default=MICRO_BATCHES)
-    ap.add_argument("--split", type=int, default=0, choices=[0, 1],
-                    help="MPRESS_OPT_SPLIT: 0 = contiguous block per CTA (default), 1 = grid stride (round 1)")
+    ap.add_argument("--split", type=int, default=3, choices=[0, 1, 2, 3],
+                    help="MPRESS_OPT_SPLIT: 0 = contiguous block per CTA, 1 = grid stride (round 1), "
+                         "2 = dynamic claims, 3 = auto (dynamic for large TMA launches, default)")
     ap.add_argument("--e2e-steps", type=int, default=16)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e-zero-copy", action="store_true",
@@ -399,7 +400,7 @@ def workload_config(args, n):
     return {"workload": wl, "tensors_per_micro_batch": 47, "micro_batch_bytes": 900 << 20,
             "micro_batches": args.micro_batches, "peers": 3 if n == 1 else n - 1,
             "path": args.path, "variant": args.variant, "max_ctas": args.max_ctas, "pdl": 0 if args.no_pdl else args.pdl,
-            "split": ["blocked", "strided"][args.split],
+            "split": ["blocked", "strided", "dynamic", "auto"][args.split],
             "l2": "inputs %.2f GiB per rank > 126 MB L2: no flush needed" %
                   (args.micro_batches * 900 / 1024)}
 

@@ -27,7 +27,7 @@ OPT_LAST_PATH = 6  # read-only: path of the last swap call
 OPT_PDL = 7
 OPT_PACE_MBPS = 12
 OPT_SPLIT = 13
-SPLIT_BLOCKED, SPLIT_STRIDED = 0, 1
+SPLIT_BLOCKED, SPLIT_STRIDED, SPLIT_DYNAMIC, SPLIT_AUTO = 0, 1, 2, 3
 OPT_AUTO_OUT, OPT_AUTO_IN = 8, 9   # read-only: AUTO's uncapped-grid path per direction (large launches)
 OPT_AUTO_OUT_SMALL, OPT_AUTO_IN_SMALL = 10, 11   # ... for launches < AUTO_SMALL_BYTES
 AUTO_SMALL_BYTES = 32 << 20

@@ -105,7 +105,7 @@ struct mpress_ctx_s {
   int order = MPRESS_ORDER_INTERLEAVE;
   int pdl = 1;                        // MPRESS_OPT_PDL
   uint64_t pace_mbps = 0;             // MPRESS_OPT_PACE_MBPS (0 = unpaced)
-  int split = 0;                      // MPRESS_OPT_SPLIT
+  int split = MPRESS_SPLIT_AUTO;      // MPRESS_OPT_SPLIT
   // SM path MPRESS_PATH_AUTO takes for an uncapped grid, per direction
   // (kDirOut, kDirIn) and size class (a launch moving < MPRESS_AUTO_SMALL_BYTES,
   // or more); until mpress_autotune measures otherwise: direct for small
@@ -115,6 +115,7 @@ struct mpress_ctx_s {
   int last_launches = 0;
   std::vector<cudaStream_t> ce_streams;  // copy-engine comparator, one per peer
   mpress::TableRing* ring = nullptr;  // device-resident tables of large launches (lazy)
+  mpress::CounterRing* counters = nullptr;  // MPRESS_SPLIT_DYNAMIC claim counters (lazy)
   mpress::EvPool ev_pool = std::make_shared<std::vector<cudaEvent_t>>();
   std::set<mpress_handle_s*> handles;
   std::vector<mpress::CopyDesc> scratch_desc;  // per-call buffers, reused

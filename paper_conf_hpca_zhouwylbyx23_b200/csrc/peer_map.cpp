@@ -145,6 +145,7 @@ void destroy(mpress_ctx_s* c) {
   c->ev_pool->clear();
   for (auto s : c->ce_streams) if (s) cudaStreamDestroy(s);
   table_ring_destroy(c->ring);
+  counter_ring_destroy(c->counters);
   delete c;
 }
 
@@ -227,7 +228,10 @@ extern "C" int mpress_init_local(int world, int source, const int* devices,
     }
     init_partition(&c->parts[p], reinterpret_cast<uint8_t*>(c->maps[p].va), want);
   }
-  const int rc = preload_kernels();
+  int rc = preload_kernels();
+  // claim counters of MPRESS_SPLIT_DYNAMIC / AUTO launches, zeroed here (a
+  // blocking memset) so no swap call has to allocate or synchronise
+  if (rc == MPRESS_OK) rc = counter_ring_create(c->device, &c->counters);
   if (rc != MPRESS_OK) {
     destroy(c);
     return rc;
@@ -346,6 +350,7 @@ extern "C" int mpress_init(int device, int world, int rank, const uint64_t* part
     }
   }
   if (rc == MPRESS_OK) rc = preload_kernels();
+  if (rc == MPRESS_OK) rc = counter_ring_create(device, &c->counters);
   rc = agree(c, rc, "map its peers");
   if (rc != MPRESS_OK) {
     destroy(c);
@@ -486,8 +491,9 @@ extern "C" int mpress_set_option(mpress_ctx_t* c, int key, int64_t value) {
       c->pace_mbps = (uint64_t)value;
       return MPRESS_OK;
     case MPRESS_OPT_SPLIT:
-      if (value != MPRESS_SPLIT_BLOCKED && value != MPRESS_SPLIT_STRIDED)
-        return fail(MPRESS_ERR_ARG, "MPRESS_OPT_SPLIT is 0 (blocked) or 1 (strided), not %lld", (long long)value);
+      if (value < MPRESS_SPLIT_BLOCKED || value > MPRESS_SPLIT_AUTO)
+        return fail(MPRESS_ERR_ARG, "MPRESS_OPT_SPLIT is 0 (blocked), 1 (strided), 2 (dynamic) or 3 (auto), not %lld",
+                    (long long)value);
       c->split = (int)value;
       return MPRESS_OK;
     case MPRESS_OPT_VARIANT: {

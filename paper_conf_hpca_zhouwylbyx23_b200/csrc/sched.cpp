@@ -169,9 +169,14 @@ int run_copy(mpress_ctx_s* c, int dir, const std::vector<CopyDesc>& d,
     // Large tables live in device memory (TableRing), except under graph
     // capture: a replay would re-read a staging slot later launches reused.
     if (!graph && d.size() > (size_t)kParamDescMax && !c->ring) MP_TRY(table_ring_create(c->device, &c->ring));
+    // Claim counters likewise: a replayed launch would reuse a slot that
+    // later eager launches take (dynamic falls back to blocked there).
+    if (!graph && c->split >= MPRESS_SPLIT_DYNAMIC && !c->counters)
+      MP_TRY(counter_ring_create(c->device, &c->counters));
     return launch_copy(path, c->variant, dir, d.data(),
                        c->order == MPRESS_ORDER_INTERLEAVE ? desc_peer.data() : nullptr, d.size(), c->max_ctas,
-                       c->pdl, stream, &c->last_launches, graph ? nullptr : c->ring, c->pace_mbps, c->split);
+                       c->pdl, stream, &c->last_launches, graph ? nullptr : c->ring, c->pace_mbps, c->split,
+                       graph ? nullptr : c->counters);
   }
 
   // Copy-engine comparator (the prior-art mechanism):
@@ -562,6 +567,8 @@ extern "C" int mpress_autotune(mpress_ctx_t* c, uint64_t probe_bytes, int trials
   }
   // warm-up round (-1), then `trials` rounds alternating which path goes first
   const int paths[2] = {MPRESS_PATH_DIRECT, MPRESS_PATH_BULK};
+  if (rc == MPRESS_OK && c->split >= MPRESS_SPLIT_DYNAMIC && !c->counters)
+    rc = counter_ring_create(c->device, &c->counters);  // the probes run the context's split
   std::vector<float> t[2][2][2];  // [class][path][dir], ms per launch
   for (int r = -1; r < trials; ++r) {
     for (int cls = 0; cls < 2; ++cls) {
@@ -574,11 +581,13 @@ extern "C" int mpress_autotune(mpress_ctx_t* c, uint64_t probe_bytes, int trials
         cudaEventRecord(ev[0], stream);
         for (int i = 0; i < reps && rc == MPRESS_OK; ++i)
           rc = launch_copy(paths[pi], MPRESS_VARIANT_AUTO, kDirOut, dout[cls][i].data(), grp.data(),
-                           dout[cls][i].size(), 0, c->pdl, stream, &launches);
+                           dout[cls][i].size(), 0, c->pdl, stream, &launches, nullptr, 0, c->split,
+                           c->counters);
         cudaEventRecord(ev[1], stream);
         for (int i = 0; i < reps && rc == MPRESS_OK; ++i)
           rc = launch_copy(paths[pi], MPRESS_VARIANT_AUTO, kDirIn, din[cls][i].data(), grp.data(),
-                           din[cls][i].size(), 0, c->pdl, stream, &launches);
+                           din[cls][i].size(), 0, c->pdl, stream, &launches, nullptr, 0, c->split,
+                           c->counters);
         cudaEventRecord(ev[2], stream);
         cudaError_t e = cudaEventSynchronize(ev[2]);
         float a = 0, b = 0;

@@ -38,6 +38,7 @@
 #include <algorithm>
 #include <atomic>
 #include <cstddef>
+#include <cstdlib>
 #include <type_traits>
 #include <mutex>
 #include <set>
@@ -67,7 +68,8 @@ struct CopyTable {
   uint32_t rounds_log2;              // R = 2^rounds_log2 >= chunks of the largest group
   uint32_t pace_ns;                  // 0, or ns between the starts of one CTA's chunks (rate pacing)
   uint32_t split;                    // kSplitBlocked / kSplitStrided: positions -> CTAs (Cursor)
-  uint32_t pad[3];
+  uint32_t qlim;                     // MPRESS_SPLIT_DYNAMIC: smallest | largest claim << 16 (positions)
+  unsigned long long* dyn;           // MPRESS_SPLIT_DYNAMIC: {claimed, CTAs done} (CounterRing slot), else null
   uint32_t g_chunk[kGroups + 1];     // first chunk of each group (prefix)
   uint32_t g_desc[kGroups + 1];      // first descriptor of each group (prefix)
   uint32_t first_chunk[CAP + 1];     // first chunk of each descriptor (prefix)
@@ -165,6 +167,47 @@ struct Cursor {
       return true;
     }
     return false;
+  }
+};
+
+// MPRESS_SPLIT_DYNAMIC: a CTA claims blocks [s, s + q) of the launch's
+// positions from a counter (atomicAdd), claiming the next block while it
+// moves the current one so the atomic's latency hides behind the copies.
+// Guided self-scheduling: q = remaining / (2 x grid), clamped to [qmin,
+// QMAX], so the last blocks are a few chunks and SMs that run faster take
+// more.  Besides removing the tail, this keeps every CTA inside one moving
+// window of the sequence (all CTAs claim from the same front) instead of
+// 148 separate regions -- fewer pages touched at once.  Every CTA counts
+// itself done once its claims ran past the end; the last one resets the
+// slot for the next launch that takes it (kernel completion orders that
+// reset before any later launch, PDL included: griddepcontrol.wait waits for
+// completion and flush).
+template <uint32_t QMAX>
+struct DynClaim {
+  unsigned long long* ctr;
+  uint64_t P;
+  uint32_t qmin;
+  uint64_t next_s = 0;   // the prefetched claim (claiming thread)
+  uint32_t next_q = 0;
+  uint32_t qmax;
+  __device__ DynClaim(unsigned long long* c, uint64_t p, uint32_t qlim) : ctr(c), P(p) {
+    qmax = qlim >> 16;
+    qmax = qmax == 0 || qmax > QMAX ? QMAX : qmax;
+    qmin = qlim & 0xFFFFu;
+    qmin = qmin == 0 ? 1 : qmin > qmax ? qmax : qmin;
+  }
+  __device__ void claim(uint64_t seen) {
+    const uint64_t rem = seen < P ? P - seen : 0;
+    const uint64_t q = rem / (2ull * gridDim.x);
+    next_q = q < qmin ? qmin : q > qmax ? qmax : (uint32_t)q;
+    next_s = atomicAdd(ctr, (unsigned long long)next_q);
+  }
+  __device__ void done() {
+    __threadfence();
+    if (atomicAdd(ctr + 1, 1ull) == gridDim.x - 1ull) {
+      atomicExch(ctr, 0ull);
+      atomicExch(ctr + 1, 0ull);
+    }
   }
 };
 
@@ -309,8 +352,39 @@ __device__ __forceinline__ void direct_body(const CopyTable<CAP>& t) {
   // the stores first measured ~6% faster (tools/ab.py), so PF is off there.
   pdl_enter();
   Cursor<CAP> cur(t);
+  // MPRESS_SPLIT_DYNAMIC: thread 0 claims blocks of <= 16 positions for the
+  // CTA and hands them over through shared memory; every thread's cursor
+  // walks the same block, so they all run out -- and refill -- together.
+  const bool dyn = t.dyn != nullptr;
+  const uint64_t P = (uint64_t)t.n_groups << t.rounds_log2;
+  DynClaim<16> dc(t.dyn, P, t.qlim);
+  __shared__ uint64_t claim_s;
+  __shared__ uint32_t claim_q;
+  if (dyn) {
+    cur.init(0, 1, 0);
+    if (threadIdx.x == 0) dc.claim(0);
+  }
+  auto next = [&](uint32_t* cc, uint32_t* ss) -> bool {
+    while (!cur.next(cc, ss)) {
+      if (!dyn) return false;
+      __syncthreads();  // every thread has read the previous block
+      if (threadIdx.x == 0) {
+        claim_s = dc.next_s;
+        claim_q = dc.next_q;
+        if (dc.next_s < P) dc.claim(dc.next_s + dc.next_q);
+      }
+      __syncthreads();
+      const uint64_t b = claim_s;
+      if (b >= P) return false;
+      cur.init(b, 1, b + claim_q < P ? b + claim_q : P);
+    }
+    return true;
+  };
   uint32_t c, s;
-  if (!cur.next(&c, &s)) return;
+  if (!next(&c, &s)) {
+    if (dyn && threadIdx.x == 0) dc.done();
+    return;
+  }
   Span sp = span_of<kShift>(t, c, s);
   Pacer pace(t.pace_ns);
   uint64_t pol = 0;
@@ -326,13 +400,13 @@ __device__ __forceinline__ void direct_body(const CopyTable<CAP>& t) {
 #pragma unroll
       for (int j = 0; j < UNROLL; ++j) r[j] = Vec<VB, HINT>::ld(sv + j * THREADS);
       if (PF) {
-        more = cur.next(&c, &s);
+        more = next(&c, &s);
         if (more) nx = span_of<kShift>(t, c, s);
       }
 #pragma unroll
       for (int j = 0; j < UNROLL; ++j) Vec<VB, HINT>::st(dv + j * THREADS, r[j], pol);
       if (!PF) {
-        more = cur.next(&c, &s);
+        more = next(&c, &s);
         if (more) nx = span_of<kShift>(t, c, s);
       }
     } else {
@@ -344,12 +418,13 @@ __device__ __forceinline__ void direct_body(const CopyTable<CAP>& t) {
       for (uint32_t x = threadIdx.x; x < n16; x += THREADS) st_stream(dv + x, ld_stream(sv + x));
       const uint32_t tail = len & 15u;
       if (threadIdx.x < tail) sp.dst[(n16 << 4) + threadIdx.x] = sp.src[(n16 << 4) + threadIdx.x];
-      more = cur.next(&c, &s);
+      more = next(&c, &s);
       if (more) nx = span_of<kShift>(t, c, s);
     }
     if (!more) break;
     sp = nx;
   }
+  if (dyn && threadIdx.x == 0) dc.done();
 }
 
 // The table as a kernel parameter (constant bank) ...
@@ -488,6 +563,15 @@ __device__ __forceinline__ void bulk_body(const CopyTable<CAP>& t) {
   };
 
   Cursor<CAP> cur(t, lane, 32u);
+  // MPRESS_SPLIT_DYNAMIC: lane 0 claims blocks of <= 32 positions, one per
+  // resolver lane; a new block is taken when every lane's cursor is empty.
+  const bool dyn = t.dyn != nullptr;
+  const uint64_t P = (uint64_t)t.n_groups << t.rounds_log2;
+  DynClaim<32> dc(t.dyn, P, t.qlim);
+  if (dyn) {
+    cur.init(0, 1, 0);
+    if (lane == 0) dc.claim(0);
+  }
   for (;;) {
     uint32_t c, sd;
     const bool v = cur.next(&c, &sd);
@@ -505,7 +589,15 @@ __device__ __forceinline__ void bulk_body(const CopyTable<CAP>& t) {
     // compiled without a warp sync and saw only the lanes already done).
     __syncwarp();
     uint32_t mask = __ballot_sync(0xffffffffu, v);
-    if (!mask) break;
+    if (!mask) {
+      if (!dyn) break;
+      const uint64_t b = shfl64(dc.next_s, 0);
+      const uint32_t q = __shfl_sync(0xffffffffu, dc.next_q, 0);
+      if (b >= P) break;
+      if (lane == 0) dc.claim(b + q);
+      cur.init(b + lane, 32u, b + q < P ? b + q : P);
+      continue;
+    }
     while (mask) {
       const int j = __ffs(mask) - 1;
       mask &= mask - 1;
@@ -541,6 +633,7 @@ __device__ __forceinline__ void bulk_body(const CopyTable<CAP>& t) {
   if (lane == 0) {
     store_until(loaded);
     bulk_wait_all();
+    if (dyn) dc.done();
   }
 }
 
@@ -687,6 +780,8 @@ int build_table(CopyTable<CAP>& t, const CopyDesc* d, const int* gid, uint32_t n
   t.n = n;
   t.pace_ns = 0;
   t.split = 0;
+  t.qlim = 0;
+  t.dyn = nullptr;
   uint64_t chunks = 0;
   uint32_t ng = 0;
   for (uint32_t i = 0; i < n; ++i) {
@@ -742,10 +837,61 @@ int launch_kernel(K k, const Shape& sh, unsigned grid, bool pdl, cudaStream_t st
 }
 
 // One launch with the table as a kernel parameter.
+// MPRESS_SPLIT_DYNAMIC: the claim-counter slot of a launch of `chunks`
+// chunks over `grid` CTAs (*slot = -1 and a static split otherwise).
+// Tuning knobs of the dynamic split for A/B runs (tools/split_ab.py):
+// MPRESS_DYN_QMIN / _QMAX (smallest / largest claim, positions; 0 = the
+// default) and MPRESS_DYN_MIN (chunks per CTA below which a launch stays
+// blocked; 0 = the default).
+uint32_t env_u32(const char* name, uint32_t dflt) {
+  const char* v = getenv(name);
+  return v && *v ? (uint32_t)strtoul(v, nullptr, 10) : dflt;
+}
+
+int take_counter(CounterRing* r, int path, int split, uint32_t shift, uint64_t chunks, unsigned grid,
+                 unsigned long long** dyn, int* slot, uint32_t* split_out, uint32_t* qlim) {
+  static const uint32_t kQmin = env_u32("MPRESS_DYN_QMIN", 1);
+  static const uint32_t kQmax = env_u32("MPRESS_DYN_QMAX", 0);
+  static const uint32_t kMinPerCta = env_u32("MPRESS_DYN_MIN", 0);
+  *dyn = nullptr;
+  *slot = -1;
+  // largest claim ~128 KiB of pieces (4 x 32 KiB ... 32 x 4 KiB): a tight
+  // front, few enough atomics (tools/split_ab.py, profiles/r02/split_ab)
+  const uint32_t qmax = kQmax ? kQmax : std::min(32u, std::max(4u, (1u << 17) >> shift));
+  *qlim = (kQmin & 0xFFFFu) | (qmax << 16);
+  *split_out = (uint32_t)(split == MPRESS_SPLIT_STRIDED ? kSplitStrided : kSplitBlocked);
+  // AUTO: dynamic for TMA launches of >= kDynAutoChunksPerCta chunks per CTA;
+  // DYNAMIC: for any launch of >= kDynMinChunksPerCta chunks per CTA
+  const bool dynamic =
+      r && ((split == MPRESS_SPLIT_DYNAMIC &&
+             chunks >= (uint64_t)(kMinPerCta ? kMinPerCta : kDynMinChunksPerCta) * grid) ||
+            (split == MPRESS_SPLIT_AUTO && path == MPRESS_PATH_BULK &&
+             chunks >= (uint64_t)(kMinPerCta ? kMinPerCta : kDynAutoChunksPerCta) * grid));
+  if (!dynamic) return MPRESS_OK;
+  const int k = r->next;
+  if (r->armed[k]) {
+    const cudaError_t e = cudaEventSynchronize(r->ev[k]);   // blocks only if the ring wrapped
+    if (e != cudaSuccess) return fail(MPRESS_ERR_CUDA, "claim-counter ring: %s", cudaGetErrorString(e));
+    r->armed[k] = false;
+  }
+  r->next = (k + 1) % r->nslots;
+  *dyn = r->dev + (size_t)k * 16;
+  *slot = k;
+  return MPRESS_OK;
+}
+
+int arm_counter(CounterRing* r, int slot, cudaStream_t stream) {
+  if (slot < 0) return MPRESS_OK;
+  const cudaError_t e = cudaEventRecord(r->ev[slot], stream);
+  if (e != cudaSuccess) return fail(MPRESS_ERR_CUDA, "claim-counter event: %s", cudaGetErrorString(e));
+  r->armed[slot] = true;
+  return MPRESS_OK;
+}
+
 template <int CAP>
 int launch_batch(int path, int variant, int dir, const CopyDesc* d, const int* gid, uint32_t n,
-                 uint32_t shift, int cap, int sms, bool pdl, uint64_t pace_mbps, int split, cudaStream_t stream,
-                 bool* launched) {
+                 uint32_t shift, int cap, int sms, bool pdl, uint64_t pace_mbps, int split, CounterRing* cr,
+                 cudaStream_t stream, bool* launched) {
   CopyTable<CAP> t;
   uint64_t chunks = 0;
   *launched = false;
@@ -753,11 +899,12 @@ int launch_batch(int path, int variant, int dir, const CopyDesc* d, const int* g
   if (chunks == 0) return MPRESS_OK;
   const unsigned grid = (unsigned)std::min<uint64_t>(chunks, (uint64_t)cap);
   t.pace_ns = pace_ns_of(pace_mbps, shift, grid);
-  t.split = (uint32_t)split;
+  int slot;
+  MP_TRY(take_counter(cr, path, split, shift, chunks, grid, &t.dyn, &slot, &t.split, &t.qlim));
   const Shape& sh = shape_of(path, variant);
   MP_TRY(launch_kernel(kernel_for<CAP, false>(path, variant, dir, (int)grid <= sms), sh, grid, pdl, stream, t));
   *launched = true;
-  return MPRESS_OK;
+  return arm_counter(cr, slot, stream);
 }
 
 // One launch with the table device-resident (TableRing): built in a pinned
@@ -765,7 +912,7 @@ int launch_batch(int path, int variant, int dir, const CopyDesc* d, const int* g
 // read by the kernel through a pointer; the slot's event, recorded after the
 // kernel, guards both slots' reuse.
 int launch_batch_ring(TableRing* r, int path, int variant, int dir, const CopyDesc* d, const int* gid, uint32_t n,
-                      uint32_t shift, int cap, int sms, bool pdl, uint64_t pace_mbps, int split,
+                      uint32_t shift, int cap, int sms, bool pdl, uint64_t pace_mbps, int split, CounterRing* cr,
                       cudaStream_t stream, bool* launched) {
   using T = CopyTable<kMaxDescPerLaunch>;
   *launched = false;
@@ -783,7 +930,8 @@ int launch_batch_ring(TableRing* r, int path, int variant, int dir, const CopyDe
   r->next = (slot + 1) % r->nslots;
   const unsigned grid = (unsigned)std::min<uint64_t>(chunks, (uint64_t)cap);
   ht->pace_ns = pace_ns_of(pace_mbps, shift, grid);
-  ht->split = (uint32_t)split;
+  int cslot;
+  MP_TRY(take_counter(cr, path, split, shift, chunks, grid, &ht->dyn, &cslot, &ht->split, &ht->qlim));
   const size_t bytes = offsetof(T, d) + (size_t)n * sizeof(CopyDesc);
   cudaError_t e = cudaMemcpyAsync(dt, ht, bytes, cudaMemcpyHostToDevice, stream);
   if (e != cudaSuccess) return fail(MPRESS_ERR_CUDA, "descriptor upload: %s", cudaGetErrorString(e));
@@ -794,7 +942,7 @@ int launch_batch_ring(TableRing* r, int path, int variant, int dir, const CopyDe
   if (e != cudaSuccess) return fail(MPRESS_ERR_CUDA, "descriptor ring event: %s", cudaGetErrorString(e));
   r->armed[slot] = true;
   *launched = true;
-  return MPRESS_OK;
+  return arm_counter(cr, cslot, stream);
 }
 
 }  // namespace
@@ -901,9 +1049,41 @@ void table_ring_destroy(TableRing* r) {
   delete r;
 }
 
+int counter_ring_create(int device, CounterRing** out) {
+  *out = nullptr;
+  auto* r = new CounterRing();
+  r->device = device;
+  r->nslots = 256;
+  r->ev = new cudaEvent_t[r->nslots]();
+  r->armed = new bool[r->nslots]();
+  const size_t bytes = (size_t)r->nslots * 16 * sizeof(unsigned long long);
+  cudaError_t e = cudaMalloc(&r->dev, bytes);
+  if (e == cudaSuccess) e = cudaMemset(r->dev, 0, bytes);
+  if (e == cudaSuccess) e = cudaDeviceSynchronize();
+  for (int i = 0; i < r->nslots && e == cudaSuccess; ++i) e = cudaEventCreateWithFlags(&r->ev[i], cudaEventDisableTiming);
+  if (e != cudaSuccess) {
+    counter_ring_destroy(r);
+    return fail(MPRESS_ERR_CUDA, "claim-counter ring: %s", cudaGetErrorString(e));
+  }
+  *out = r;
+  return MPRESS_OK;
+}
+
+void counter_ring_destroy(CounterRing* r) {
+  if (!r) return;
+  for (int i = 0; i < r->nslots; ++i) {
+    if (r->armed[i]) cudaEventSynchronize(r->ev[i]);
+    if (r->ev[i]) cudaEventDestroy(r->ev[i]);
+  }
+  if (r->dev) cudaFree(r->dev);
+  delete[] r->ev;
+  delete[] r->armed;
+  delete r;
+}
+
 int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* group, size_t n,
                 int max_ctas, int pdl_mode, cudaStream_t stream, int* launches, TableRing* ring,
-                uint64_t pace_mbps, int split) {
+                uint64_t pace_mbps, int split, CounterRing* counters) {
   const int sms = sm_count(nullptr);
   if (sms <= 0) return fail(MPRESS_ERR_CUDA, "cannot query the SM count");
   // PDL (MPRESS_OPT_PDL): mode 1 only for an uncapped grid.  A capped swap
@@ -948,17 +1128,17 @@ int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* gr
     const int* g = group ? group + base : nullptr;
     bool launched = false;
     if (ring && m > (uint32_t)kParamDescMax)
-      MP_TRY(launch_batch_ring(ring, path, variant, dir, d + base, g, m, shift, cap, sms, pdl, pace_mbps, split, stream, &launched));
+      MP_TRY(launch_batch_ring(ring, path, variant, dir, d + base, g, m, shift, cap, sms, pdl, pace_mbps, split, counters, stream, &launched));
     else if (m <= 16)
-      MP_TRY(launch_batch<16>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, pace_mbps, split, stream, &launched));
+      MP_TRY(launch_batch<16>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, pace_mbps, split, counters, stream, &launched));
     else if (m <= 32)
-      MP_TRY(launch_batch<32>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, pace_mbps, split, stream, &launched));
+      MP_TRY(launch_batch<32>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, pace_mbps, split, counters, stream, &launched));
     else if (m <= 64)
-      MP_TRY(launch_batch<64>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, pace_mbps, split, stream, &launched));
+      MP_TRY(launch_batch<64>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, pace_mbps, split, counters, stream, &launched));
     else if (m <= 128)
-      MP_TRY(launch_batch<128>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, pace_mbps, split, stream, &launched));
+      MP_TRY(launch_batch<128>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, pace_mbps, split, counters, stream, &launched));
     else
-      MP_TRY(launch_batch<kMaxDescPerLaunch>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, pace_mbps, split, stream, &launched));
+      MP_TRY(launch_batch<kMaxDescPerLaunch>(path, variant, dir, d + base, g, m, shift, cap, sms, pdl, pace_mbps, split, counters, stream, &launched));
     if (launched && launches) ++*launches;
   }
   return MPRESS_OK;

@@ -46,6 +46,21 @@ constexpr int kParamDescMax = 128;
 int table_ring_create(int device, TableRing** out);
 void table_ring_destroy(TableRing* r);
 
+// Claim counters of MPRESS_SPLIT_DYNAMIC launches: one slot {claimed, CTAs
+// done} per launch (one 128-byte line each, so concurrent launches do not
+// share a line), zeroed at creation and reset by each launch's last CTA.  A
+// slot is reused once the event recorded after its launch has completed.
+struct CounterRing {
+  int device = -1;
+  int nslots = 0;
+  unsigned long long* dev = nullptr;  // nslots x 16 u64
+  cudaEvent_t* ev = nullptr;
+  bool* armed = nullptr;
+  int next = 0;
+};
+int counter_ring_create(int device, CounterRing** out);
+void counter_ring_destroy(CounterRing* r);
+
 // Enqueue kernels moving every descriptor on `stream`; `path` is
 // MPRESS_PATH_DIRECT or MPRESS_PATH_BULK, `variant` its kernel shape;
 // `max_ctas` caps the grid (0 = the variant's default grid); `pdl_mode`
@@ -57,11 +72,16 @@ void table_ring_destroy(TableRing* r);
 // `pace_mbps` (MPRESS_OPT_PACE_MBPS, 0 = off): the launch's CTAs space their
 // chunks so the whole launch moves at most pace_mbps MB/s.  `split`
 // (MPRESS_OPT_SPLIT): 0 = each CTA takes a contiguous block of the
-// interleaved chunk sequence, 1 = a grid stride over it (round 1).
+// interleaved chunk sequence, 1 = a grid stride over it (round 1), 2 =
+// blocks claimed from a counter in `counters` (null: as 0); a launch with
+// fewer than kDynMinChunksPerCta chunks per CTA runs as 0; 3 (AUTO) = 2 for
+// bulk-kernel launches of >= kDynAutoChunksPerCta chunks per CTA, else 0.
+constexpr int kDynMinChunksPerCta = 4;
+constexpr int kDynAutoChunksPerCta = 32;
 int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* group, size_t n,
                 int max_ctas, int pdl_mode,
                 cudaStream_t stream, int* launches, TableRing* ring = nullptr, uint64_t pace_mbps = 0,
-                int split = 0);
+                int split = 0, CounterRing* counters = nullptr);
 
 // SM count of the current device (cached per device; 0 on error); *dev = the
 // device ordinal if dev is not null.

@@ -19,8 +19,8 @@ a tensor id no swap uses).  After swap-out and after swap-in:
 
 Shapes: every MPRESS_OPT_VARIANT of the direct (14) and bulk (9) kernels,
 each at grids of 1 and 3 CTAs (many pieces per CTA: the bulk ring wraps,
-per-lane cursors finish at different times) and at its default grid, both CTA
-splits; the copy engines; AUTO; a > 128-descriptor launch (device-resident
+per-lane cursors finish at different times) and at its default grid, all
+three CTA splits (blocked, strided, dynamic claims); the copy engines; AUTO; a > 128-descriptor launch (device-resident
 tables); a pinned host-pool peer (NEXT-4)."""
 import random
 
@@ -153,9 +153,20 @@ def test_guard_bulk_every_shape(variant):
     _guarded_roundtrip(SIZES, mp.PATH_BULK, variant, caps=(1, 3, 0), seed=200 + variant)
 
 
+@pytest.mark.parametrize("split", [1, 2], ids=["strided", "dynamic"])
 @pytest.mark.parametrize("path", [mp.PATH_DIRECT, mp.PATH_BULK], ids=["direct", "bulk"])
-def test_guard_grid_stride_split(path):
-    _guarded_roundtrip(SIZES, path, caps=(2, 0), split=1, seed=300 + path)
+def test_guard_other_splits(path, split):
+    _guarded_roundtrip(SIZES, path, caps=(1, 2, 0), split=split, seed=300 + 10 * split + path)
+
+
+@pytest.mark.parametrize("variant", list(range(14)))
+def test_guard_dynamic_split_direct_every_shape(variant):
+    _guarded_roundtrip(SIZES, mp.PATH_DIRECT, variant, caps=(3, 0), split=2, seed=700 + variant)
+
+
+@pytest.mark.parametrize("variant", list(range(9)))
+def test_guard_dynamic_split_bulk_every_shape(variant):
+    _guarded_roundtrip(SIZES, mp.PATH_BULK, variant, caps=(3, 0), split=2, seed=800 + variant)
 
 
 @pytest.mark.parametrize("path", [mp.PATH_AUTO, mp.PATH_CE], ids=["auto", "ce"])
@@ -201,6 +212,6 @@ def test_guard_detects_a_stray_write():
         torch.cuda.synchronize()
         assert _check_stash(ctx, o, part_bytes, sl, 7)[1] >= 56
         assert src.guard_bad() >= 56
-        h.free()
+        h.free(force=True)
     finally:
         ctx.finalize()

@@ -47,7 +47,7 @@ def test_random_interleavings(seed):
                                                             mp.PATH_AUTO]))
                     ctx.set_option(mp.OPT_MAX_CTAS, rng.choice([0, 1, 7, 64]))
                     ctx.set_option(mp.OPT_PDL, rng.choice([0, 1, 2]))
-                    ctx.set_option(mp.OPT_SPLIT, rng.choice([mp.SPLIT_BLOCKED, mp.SPLIT_STRIDED]))
+                    ctx.set_option(mp.OPT_SPLIT, rng.choice([mp.SPLIT_BLOCKED, mp.SPLIT_STRIDED, mp.SPLIT_DYNAMIC, mp.SPLIT_AUTO]))
                     ctx.set_option(mp.OPT_PACE_MBPS, rng.choice([0, 0, 200_000, 2_000_000]))
                 src = [torch.empty(n, dtype=torch.uint8, device="cuda") for n in sizes]
                 for i, t in enumerate(src):

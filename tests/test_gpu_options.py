@@ -230,12 +230,12 @@ def test_pace_limits_rate_and_keeps_bytes(path, cap):
         ctx.finalize()
 
 
-@pytest.mark.parametrize("split", [0, 1], ids=["blocked", "strided"])
+@pytest.mark.parametrize("split", [0, 1, 2, 3], ids=["blocked", "strided", "dynamic", "auto"])
 @pytest.mark.parametrize("path,variant,cap", [(mp.PATH_DIRECT, 7, 5), (mp.PATH_DIRECT, 11, 128),
                                               (mp.PATH_DIRECT, 5, 0), (mp.PATH_BULK, 3, 0),
                                               (mp.PATH_BULK, 6, 7)])
 def test_split_modes_are_oracle_exact(split, path, variant, cap):
-    """MPRESS_OPT_SPLIT: both ways of sharing a launch's interleaved chunks
+    """MPRESS_OPT_SPLIT: every way of sharing a launch's interleaved chunks
     among CTAs write exactly the oracle's stash bytes and restore every
     tensor, with ragged stripes over three peers of unequal weight."""
     import oracle
@@ -265,7 +265,7 @@ def test_split_modes_are_oracle_exact(split, path, variant, cap):
         h.free()
         assert all(synth_dev.check(t, 41, i) == 0 for i, t in enumerate(dst))
         with pytest.raises(mp.MPressError):
-            ctx.set_option(mp.OPT_SPLIT, 2)
+            ctx.set_option(mp.OPT_SPLIT, 4)
     finally:
         ctx.finalize()
 
