@@ -501,10 +501,12 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
  * counter slot is reset by the launch's last CTA and reused once the event
  * recorded after the launch has fired; launches of < 4 chunks per CTA and
  * launches enqueued under graph capture run BLOCKED.
- * MPRESS_SPLIT_AUTO (3, default): DYNAMIC for TMA (bulk) kernel launches of
- * >= 32 chunks per CTA, BLOCKED otherwise (measured on B200 loopback: bulk
- * +3.8% at 900 MiB and 4 GiB, the direct kernel and launches of a few chunks
- * per CTA faster blocked). */
+ * MPRESS_SPLIT_AUTO (3, default): launches of < 32 chunks per CTA STRIDED on
+ * a full grid (>= one CTA per SM; BLOCKED on a capped one), larger ones
+ * DYNAMIC on the TMA (bulk) kernel and BLOCKED on the direct
+ * kernel (measured on B200 loopback: bulk +3.8% at 900 MiB and 4 GiB with
+ * the claims, launches of a few chunks per CTA +1-7% with the stride, the
+ * direct kernel's large launches fastest blocked). */
 #define MPRESS_OPT_SPLIT     13
 #define MPRESS_SPLIT_BLOCKED 0
 #define MPRESS_SPLIT_STRIDED 1

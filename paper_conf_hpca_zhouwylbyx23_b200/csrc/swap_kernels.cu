@@ -849,7 +849,7 @@ uint32_t env_u32(const char* name, uint32_t dflt) {
 }
 
 int take_counter(CounterRing* r, int path, int split, uint32_t shift, uint64_t chunks, unsigned grid,
-                 unsigned long long** dyn, int* slot, uint32_t* split_out, uint32_t* qlim) {
+                 bool full_grid, unsigned long long** dyn, int* slot, uint32_t* split_out, uint32_t* qlim) {
   static const uint32_t kQmin = env_u32("MPRESS_DYN_QMIN", 1);
   static const uint32_t kQmax = env_u32("MPRESS_DYN_QMAX", 0);
   static const uint32_t kMinPerCta = env_u32("MPRESS_DYN_MIN", 0);
@@ -859,9 +859,17 @@ int take_counter(CounterRing* r, int path, int split, uint32_t shift, uint64_t c
   // front, few enough atomics (tools/split_ab.py, profiles/r02/split_ab)
   const uint32_t qmax = kQmax ? kQmax : std::min(32u, std::max(4u, (1u << 17) >> shift));
   *qlim = (kQmin & 0xFFFFu) | (qmax << 16);
-  *split_out = (uint32_t)(split == MPRESS_SPLIT_STRIDED ? kSplitStrided : kSplitBlocked);
-  // AUTO: dynamic for TMA launches of >= kDynAutoChunksPerCta chunks per CTA;
-  // DYNAMIC: for any launch of >= kDynMinChunksPerCta chunks per CTA
+  // AUTO: launches of < kDynAutoChunksPerCta chunks per CTA take the grid
+  // stride (every CTA inside one window of the sequence: +4-7% at 64 MiB,
+  // +1-2% at 256 MiB over blocked on B200 loopback), larger TMA launches the
+  // dynamic claims, larger direct launches the blocked split (there the
+  // claims and the stride cost 2-12%: profiles/r02/split_ab/);
+  // DYNAMIC: claims for any launch of >= kDynMinChunksPerCta chunks per CTA
+  // (the stride only on a full grid: on a capped one the skipped positions
+  // of a multi-peer sequence alias with it, 8-12% slower at 32-64 CTAs)
+  const bool small = chunks < (uint64_t)kDynAutoChunksPerCta * grid;
+  const bool stride = split == MPRESS_SPLIT_STRIDED || (split == MPRESS_SPLIT_AUTO && small && full_grid);
+  *split_out = (uint32_t)(stride ? kSplitStrided : kSplitBlocked);
   const bool dynamic =
       r && ((split == MPRESS_SPLIT_DYNAMIC &&
              chunks >= (uint64_t)(kMinPerCta ? kMinPerCta : kDynMinChunksPerCta) * grid) ||
@@ -900,7 +908,7 @@ int launch_batch(int path, int variant, int dir, const CopyDesc* d, const int* g
   const unsigned grid = (unsigned)std::min<uint64_t>(chunks, (uint64_t)cap);
   t.pace_ns = pace_ns_of(pace_mbps, shift, grid);
   int slot;
-  MP_TRY(take_counter(cr, path, split, shift, chunks, grid, &t.dyn, &slot, &t.split, &t.qlim));
+  MP_TRY(take_counter(cr, path, split, shift, chunks, grid, (int)grid >= sms, &t.dyn, &slot, &t.split, &t.qlim));
   const Shape& sh = shape_of(path, variant);
   MP_TRY(launch_kernel(kernel_for<CAP, false>(path, variant, dir, (int)grid <= sms), sh, grid, pdl, stream, t));
   *launched = true;
@@ -931,7 +939,7 @@ int launch_batch_ring(TableRing* r, int path, int variant, int dir, const CopyDe
   const unsigned grid = (unsigned)std::min<uint64_t>(chunks, (uint64_t)cap);
   ht->pace_ns = pace_ns_of(pace_mbps, shift, grid);
   int cslot;
-  MP_TRY(take_counter(cr, path, split, shift, chunks, grid, &ht->dyn, &cslot, &ht->split, &ht->qlim));
+  MP_TRY(take_counter(cr, path, split, shift, chunks, grid, (int)grid >= sms, &ht->dyn, &cslot, &ht->split, &ht->qlim));
   const size_t bytes = offsetof(T, d) + (size_t)n * sizeof(CopyDesc);
   cudaError_t e = cudaMemcpyAsync(dt, ht, bytes, cudaMemcpyHostToDevice, stream);
   if (e != cudaSuccess) return fail(MPRESS_ERR_CUDA, "descriptor upload: %s", cudaGetErrorString(e));
