@@ -458,7 +458,9 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
  * (the only copy-engine variant);
  * MPRESS_VARIANT_AUTO (-1, default) = direct 9 when the grid is capped at
  * <= one CTA per SM (128-thread CTAs co-reside with a GEMM), else 5; bulk 3;
- * copy engines 0.
+ * on a full grid a launch of < 16 chunks per SM (< ~74 MiB) takes the
+ * deeper-ring shape instead (direct 1, bulk 0: more bytes in flight per SM
+ * for a launch that is mostly ramp and tail); copy engines 0.
  * MPRESS_OPT_ORDER: chunk order inside one launch -- 0 = interleave the
  * peers by a weighted round robin, so every peer link carries its share of
  * the swap at every moment (default; needed when several sources share

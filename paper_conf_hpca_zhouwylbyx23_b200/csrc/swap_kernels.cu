@@ -1117,6 +1117,21 @@ int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* gr
       variant = (max_ctas > 0 && max_ctas <= sms) ? 9 : 5;
     else
       variant = 3;
+    // Few chunks per SM on a full grid (< 16: a launch of < ~74 MiB): the
+    // whole launch is ramp and tail, and a deeper ring per SM wins -- bulk
+    // 6 x 32 KiB (shape 0) instead of 3 x 32 KiB, direct 512 x 8 x 16 B
+    // (shape 1, 64 KiB of loads per CTA) instead of 2 x 256 x 4 x 32 B: e.g.
+    // 32 MiB over 3 peers 2428 -> 3069 GB/s out (bulk), 2333 -> 2997
+    // (direct); 16 MiB 1827 -> 2232 in.  At 128 MiB (28 chunks per CTA) the
+    // default shapes are faster again (bulk 3005 vs 2746, direct 2918 vs 2842).
+    // (profiles/r02/small_shapes*.jsonl).
+    if (!capped) {
+      const uint32_t sh = shape_of(path, variant).shift;
+      uint64_t chunks = 0;
+      for (size_t i = 0; i < n; ++i) chunks += (d[i].len + (1ull << sh) - 1) >> sh;
+      if (chunks < (uint64_t)kDeepChunksPerCta * (uint64_t)sms)
+        variant = path == MPRESS_PATH_DIRECT ? 1 : 0;
+    }
   }
   const int nvar = path == MPRESS_PATH_BULK ? kBulkVariants : kDirectVariants;
   if (variant < 0 || variant >= nvar) return fail(MPRESS_ERR_ARG, "kernel variant %d out of range", variant);

@@ -78,6 +78,9 @@ void counter_ring_destroy(CounterRing* r);
 // bulk-kernel launches of >= kDynAutoChunksPerCta chunks per CTA, else 0.
 constexpr int kDynMinChunksPerCta = 4;
 constexpr int kDynAutoChunksPerCta = 32;
+// MPRESS_VARIANT_AUTO on a full grid: launches of fewer chunks per SM (of
+// the default shape) than this take the deeper-ring shape (bulk 0, direct 1).
+constexpr int kDeepChunksPerCta = 16;
 int launch_copy(int path, int variant, int dir, const CopyDesc* d, const int* group, size_t n,
                 int max_ctas, int pdl_mode,
                 cudaStream_t stream, int* launches, TableRing* ring = nullptr, uint64_t pace_mbps = 0,

@@ -6,7 +6,7 @@ only around the runs, so PDL chains the launches), splits alternating round
 by round.  Prints one JSON row per case with the median per-launch time and
 GB/s of each split.
 
-  python tools/split_ab.py [rounds]     # env SPLITS=0,2  PATHS=bulk,direct
+  python tools/split_ab.py [rounds]     # env SPLITS=0,2  PATHS=bulk,direct  VARIANTS=-1  CAPS=0  CASES=0,1
 """
 import json
 import os
@@ -29,10 +29,14 @@ CASES = [  # name, sizes, peers, launches per run
     ("16 MiB -> 3", [16 << 20], 3, 32),
     ("256 MiB -> 7", [256 << 20], 7, 8),
     ("4 GiB -> 7", [4 << 30], 7, 2),
+    ("4 MiB -> 7", [4 << 20], 7, 64),
+    ("32 MiB (8 x 4 MiB) -> 3", [4 << 20] * 8, 3, 32),
+    ("128 MiB -> 3", [128 << 20], 3, 16),
+    ("1 MiB -> 3", [1 << 20], 3, 64),
 ]
 
 
-def run_case(sizes, peers_n, R, path, splits, rounds, cap):
+def run_case(sizes, peers_n, R, path, splits, rounds, cap, variant=-1):
     world = peers_n + 1
     peers = list(range(1, world))
     spare = workloads.spare_vector(world, 0, peers, spare=64 << 30)
@@ -42,6 +46,7 @@ def run_case(sizes, peers_n, R, path, splits, rounds, cap):
     part[0] = [R * u * mp.DEFAULT_GRANULE for u in pl.units]
     ctx = mp.Context.local(world, 0, [0] * world, part)
     ctx.set_option(mp.OPT_PATH, PATHS[path])
+    ctx.set_option(mp.OPT_VARIANT, variant)
     ctx.set_option(mp.OPT_MAX_CTAS, cap)
     src = [torch.empty(s, dtype=torch.uint8, device="cuda") for s in sizes]
     for i, t in enumerate(src):
@@ -86,13 +91,16 @@ def main():
     splits = [int(x) for x in os.environ.get("SPLITS", "0,2").split(",")]
     caps = [int(x) for x in os.environ.get("CAPS", "0").split(",")]
     only = os.environ.get("CASES")
+    variants = [int(x) for x in os.environ.get("VARIANTS", "-1").split(",")]
     for path in os.environ.get("PATHS", "bulk,direct").split(","):
         for ci, (name, sizes, peers_n, R) in enumerate(CASES):
             if only and str(ci) not in only.split(","):
                 continue
             for cap in caps:
-                row = run_case(sizes, peers_n, R, path, splits, rounds, cap)
-                print(json.dumps({"case": name, "path": path, "max_ctas": cap, **row}), flush=True)
+                for var in variants:
+                    row = run_case(sizes, peers_n, R, path, splits, rounds, cap, var)
+                    print(json.dumps({"case": name, "path": path, "variant": var, "max_ctas": cap, **row}),
+                          flush=True)
 
 
 if __name__ == "__main__":
