@@ -52,6 +52,7 @@ MICRO_BATCHES = 8
 SPARE_PER_PEER = 24 * GiB          # cfg2: 24 GiB spare per peer
 FALLBACK_HBM = 6650.0              # B200_PROFILING.md fallback, GB/s
 NVLINK_GUIDE = 770.0               # B200_PROFILING.md's figure (peer copy per direction), not ours
+HBM_NOMINAL = 7700.0               # GB/s, B200 HBM3e nominal (B200_PROFILING.md: 7.7 TB/s HGX, 8 DGX)
 NVLINK_NOMINAL = 900.0
 
 
@@ -592,6 +593,11 @@ def main():
                 "kernel": "mp_swap_%s<%s>" % (ran, "kDirIn" if dom == "in" else "kDirOut"),
                 "algorithmic_bytes_per_launch": algo_bytes,
                 "avg_launch_ms": avg_ms, "peak_source": "%s hbm_gbs (MEASURED_PEAKS.json)" % peaks_src,
+                # the measured peak is torch's copy_ of 2 GiB (an elementwise
+                # LSU copy); the TMA kernel claiming from one moving front
+                # moves HBM faster than it, hence frac > 1;
+                # against the nominal 7.7 TB/s of B200 HBM3e (HGX):
+                "frac_of_nominal": achieved / HBM_NOMINAL,
                 # sampled launches: average kernel time x launches per step / step time
                 "share_of_step": (statistics.mean(dur["out"]) + statistics.mean(dur["in"])) * mb / ms_step
                 if ms_step > 0 else None,
