@@ -336,3 +336,43 @@ def test_peer_ptr_errors_and_identity():
         h.free()
     finally:
         ctx.finalize()
+
+
+def test_dynamic_claims_counter_ring_wraps_and_streams():
+    """MPRESS_SPLIT_DYNAMIC: 600 launches (more than the 256 claim-counter
+    slots, so every slot is reset by its launch's last CTA and reused) on two
+    streams at once, at 1 CTA (the claims' serial case) and 8 CTAs;
+    every restored byte equals the generator -- a slot left non-zero, or
+    shared by two concurrent launches, would skip or duplicate chunks."""
+    from synth import device as synth_dev
+    world = 3
+    sizes = [(1 << 20) + 4096 * 3 + 48, 333333]
+    spare, bw = [0, 1 << 30, 1 << 30], [0, 2, 1]
+    pl = mp.plan(world, 0, spare, bw, sizes)
+    part = [[0] * world for _ in range(world)]
+    part[0] = [8 * u * mp.DEFAULT_GRANULE for u in pl.units]
+    ctx = mp.Context.local(world, 0, [0] * world, part)
+    try:
+        ctx.set_option(mp.OPT_PATH, mp.PATH_BULK)
+        ctx.set_option(mp.OPT_SPLIT, mp.SPLIT_DYNAMIC)
+        src = [torch.empty(n, dtype=torch.uint8, device="cuda") for n in sizes]
+        for i, t in enumerate(src):
+            synth_dev.fill(t, 61, i)
+        torch.cuda.synchronize()
+        streams = [torch.cuda.Stream(), torch.cuda.Stream()]
+        for cap in (1, 8):
+            ctx.set_option(mp.OPT_MAX_CTAS, cap)
+            dsts = []     # all kept alive until the sync (used on side streams)
+            for k in range(150):
+                s = streams[k % 2]
+                dst = [torch.empty(n, dtype=torch.uint8, device="cuda") for n in sizes]
+                s.wait_stream(torch.cuda.current_stream())
+                h = ctx.swap_out(pl, src, stream=s)
+                ctx.swap_in(h, dst, stream=s)
+                h.free()
+                dsts.append(dst)
+            torch.cuda.synchronize()
+            for dst in dsts:
+                assert all(synth_dev.check(t, 61, i) == 0 for i, t in enumerate(dst)), cap
+    finally:
+        ctx.finalize()
