@@ -354,6 +354,16 @@ MPRESS_API int mpress_executor_before(mpress_executor_t* x, uint32_t op, void* c
 MPRESS_API int mpress_executor_after(mpress_executor_t* x, uint32_t op, void* compute_stream,
                                      void* const* activations);
 MPRESS_API int mpress_executor_release(mpress_executor_t* x, uint32_t micro_batch, void* stream);
+/* The executor's own swap options (MPRESS_OPT_PATH, _MAX_CTAS, _VARIANT,
+ * _ORDER, _PDL, _PACE_MBPS, _SPLIT; same values and validation as
+ * mpress_set_option): a copy of the context's taken at mpress_executor_create,
+ * so one pipeline stage can run its swaps on another transfer path or grid
+ * than the rest of the process -- the NEXT-2 replay measured no single path
+ * best for every stage (copy engines beside short GEMMs, the TMA kernel
+ * beside long ones).  A B200 addition (§9).
+ * Errors: MPRESS_ERR_ARG (not a swap option, bad value). */
+MPRESS_API int mpress_executor_set_option(mpress_executor_t* x, int option, int64_t value);
+MPRESS_API int mpress_executor_get_option(const mpress_executor_t* x, int option, int64_t* value);
 MPRESS_API int mpress_executor_free(mpress_executor_t* x);
 
 /* ---- peer-memory layer ----------------------------------------------------- */

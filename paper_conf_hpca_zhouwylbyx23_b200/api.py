@@ -46,7 +46,8 @@ EXPORTED = [
     "mpress_plan_from_units", "mpress_schedule_1f1b", "mpress_map_search",
     "mpress_compaction_plan", "mpress_executor_create", "mpress_executor_ops",
     "mpress_executor_slot", "mpress_executor_restore_to", "mpress_executor_before",
-    "mpress_executor_after", "mpress_executor_release", "mpress_executor_free", "mpress_init",
+    "mpress_executor_after", "mpress_executor_release", "mpress_executor_set_option",
+    "mpress_executor_get_option", "mpress_executor_free", "mpress_init",
     "mpress_init_local",
     "mpress_finalize", "mpress_stash_free", "mpress_set_option", "mpress_get_option", "mpress_autotune",
     "mpress_swap_out", "mpress_swap_in", "mpress_wait", "mpress_query", "mpress_handle_state",
@@ -118,6 +119,8 @@ def _load():
         "mpress_executor_before": (c_int, [P, c_uint32, P, POINTER(c_uint32), POINTER(c_uint32)]),
         "mpress_executor_after": (c_int, [P, c_uint32, P, P]),
         "mpress_executor_release": (c_int, [P, c_uint32, P]),
+        "mpress_executor_set_option": (c_int, [P, c_int, c_int64]),
+        "mpress_executor_get_option": (c_int, [P, c_int, POINTER(c_int64)]),
         "mpress_executor_free": (c_int, [P]),
         "mpress_compaction_plan": (c_int, [c_uint32, P, c_uint64, P, P, POINTER(c_uint64),
                                            POINTER(c_uint64)]),
@@ -459,6 +462,16 @@ class Executor:
         """mpress_executor_release: `stream` waits until micro-batch m's
         swap-out has read its activations, so they may be freed on it."""
         _check(lib.mpress_executor_release(self._h, m, _stream(stream)))
+
+    def set_option(self, key, value):
+        """mpress_executor_set_option: this executor's own swap options
+        (a copy of the context's taken at creation)."""
+        _check(lib.mpress_executor_set_option(self._h, key, int(value)))
+
+    def get_option(self, key):
+        v = c_int64()
+        _check(lib.mpress_executor_get_option(self._h, key, byref(v)))
+        return v.value
 
     def free(self):
         if self._h is not None:

@@ -82,6 +82,22 @@ struct Partition {
   std::deque<Fence> fences;           // in release order (oldest first)
 };
 
+// The options a swap launch runs with (mpress_set_option's swap keys): the
+// context's, or an executor's own copy (mpress_executor_set_option).
+struct SwapOpts {
+  int path = MPRESS_PATH_AUTO;
+  int max_ctas = 0;
+  int variant = MPRESS_VARIANT_AUTO;
+  int order = MPRESS_ORDER_INTERLEAVE;
+  int pdl = 1;                        // MPRESS_OPT_PDL
+  uint64_t pace_mbps = 0;             // MPRESS_OPT_PACE_MBPS (0 = unpaced)
+  int split = MPRESS_SPLIT_AUTO;      // MPRESS_OPT_SPLIT
+};
+// Set one swap option (validated); kNotSwapOption if `key` is not one.
+constexpr int kNotSwapOption = 1;
+int set_swap_option(SwapOpts* o, int key, int64_t value);
+int get_swap_option(const SwapOpts& o, int key, int64_t* value);  // kNotSwapOption if not one
+
 }  // namespace mpress
 
 struct mpress_handle_s;
@@ -97,15 +113,9 @@ struct mpress_ctx_s {
   mpress::Mapping own;                // multi-process: this rank's exported pool
   std::vector<mpress::Mapping> maps;  // [world] pool mappings used by this source
   std::vector<mpress::Partition> parts;  // [world]
-  int path = MPRESS_PATH_AUTO;
+  mpress::SwapOpts opt;               // the swap options (mpress_set_option)
   int last_path = -1;                 // path the last swap call ran (MPRESS_OPT_LAST_PATH)
   bool host_peer = false;             // a peer pool is pinned host memory (NEXT-4)
-  int max_ctas = 0;
-  int variant = MPRESS_VARIANT_AUTO;
-  int order = MPRESS_ORDER_INTERLEAVE;
-  int pdl = 1;                        // MPRESS_OPT_PDL
-  uint64_t pace_mbps = 0;             // MPRESS_OPT_PACE_MBPS (0 = unpaced)
-  int split = MPRESS_SPLIT_AUTO;      // MPRESS_OPT_SPLIT
   // SM path MPRESS_PATH_AUTO takes for an uncapped grid, per direction
   // (kDirOut, kDirIn) and size class (a launch moving < MPRESS_AUTO_SMALL_BYTES,
   // or more); until mpress_autotune measures otherwise: direct for small
@@ -148,4 +158,9 @@ struct mpress_handle_s {
 namespace mpress {
 // A pooled CUDA event (disable-timing) owned by reference; sched.cpp.
 EvRef take_event(mpress_ctx_s* c);
+// mpress_swap_out / mpress_swap_in with explicit options (the executor's);
+// sched.cpp.  The public calls pass the context's options.
+int swap_out_with(mpress_ctx_s* c, const SwapOpts& o, const mpress_plan_t* plan, void* const* tensors,
+                  void* stream, void* after, mpress_handle_t** out);
+int swap_in_with(mpress_ctx_s* c, const SwapOpts& o, mpress_handle_t* h, void* const* dst, void* stream);
 }  // namespace mpress

@@ -27,6 +27,10 @@ struct mpress_executor_s {
   std::vector<mpress_handle_t*> handle;      // per micro-batch
   std::vector<std::vector<void*>> restore;   // per micro-batch: destination pointers
   std::vector<mpress_1f1b_slot> slots;
+  // the options of this executor's swaps: the context's at creation, then
+  // mpress_executor_set_option (a stage picks its transfer path: the NEXT-2
+  // replay found no one path best for every stage)
+  mpress::SwapOpts opt;
 };
 
 using namespace mpress;
@@ -51,6 +55,10 @@ extern "C" int mpress_executor_create(mpress_ctx_t* ctx, const mpress_plan_t* pl
       return rc;
     }
     x->ctx = ctx;
+    {
+      std::lock_guard<std::mutex> lk(ctx->mu);
+      x->opt = ctx->opt;
+    }
     x->plan = plan;
     x->out_stream = static_cast<cudaStream_t>(out_stream);
     x->in_stream = static_cast<cudaStream_t>(in_stream);
@@ -137,7 +145,7 @@ extern "C" int mpress_executor_after(mpress_executor_t* x, uint32_t op, void* co
   if (x->kind[op] == 0) {  // F(m) produced the activations: swap them out
     if (!activations) return fail(MPRESS_ERR_ARG, "mpress_executor_after: F(%d) needs its activations", m);
     if (x->handle[m]) return fail(MPRESS_ERR_STATE, "mpress_executor_after: micro-batch %d already out", m);
-    MP_TRY(mpress_swap_out(c, x->plan, activations, x->out_stream, done.get(), &x->handle[m]));
+    MP_TRY(swap_out_with(c, x->opt, x->plan, activations, x->out_stream, done.get(), &x->handle[m]));
   }
   for (uint32_t mm : x->trig[op]) {  // swap-ins issued as late as still hidden
     if (!x->handle[mm]) return fail(MPRESS_ERR_STATE, "mpress_executor_after: micro-batch %u not swapped out", mm);
@@ -145,7 +153,7 @@ extern "C" int mpress_executor_after(mpress_executor_t* x, uint32_t op, void* co
       return fail(MPRESS_ERR_STATE, "mpress_executor_after: no restore buffers for micro-batch %u", mm);
     e = cudaStreamWaitEvent(x->in_stream, done.get(), 0);
     if (e != cudaSuccess) return fail(MPRESS_ERR_CUDA, "cudaStreamWaitEvent: %s", cudaGetErrorString(e));
-    MP_TRY(mpress_swap_in(c, x->handle[mm], x->restore[mm].data(), x->in_stream));
+    MP_TRY(swap_in_with(c, x->opt, x->handle[mm], x->restore[mm].data(), x->in_stream));
   }
   return MPRESS_OK;
 }
@@ -159,6 +167,18 @@ extern "C" int mpress_executor_release(mpress_executor_t* x, uint32_t micro_batc
   const cudaError_t e = cudaStreamWaitEvent(static_cast<cudaStream_t>(stream), h->out_done.get(), 0);
   if (e != cudaSuccess) return fail(MPRESS_ERR_CUDA, "mpress_executor_release: %s", cudaGetErrorString(e));
   return MPRESS_OK;
+}
+
+extern "C" int mpress_executor_set_option(mpress_executor_t* x, int key, int64_t value) {
+  if (!x) return fail(MPRESS_ERR_ARG, "mpress_executor_set_option: null executor");
+  const int rc = set_swap_option(&x->opt, key, value);
+  return rc == kNotSwapOption ? fail(MPRESS_ERR_ARG, "option %d is not a swap option", key) : rc;
+}
+
+extern "C" int mpress_executor_get_option(const mpress_executor_t* x, int key, int64_t* value) {
+  if (!x || !value) return fail(MPRESS_ERR_ARG, "mpress_executor_get_option: null argument");
+  const int rc = get_swap_option(x->opt, key, value);
+  return rc == kNotSwapOption ? fail(MPRESS_ERR_ARG, "option %d is not a swap option", key) : rc;
 }
 
 extern "C" int mpress_executor_slot(const mpress_executor_t* x, uint32_t micro_batch, mpress_1f1b_slot* slot) {

@@ -460,66 +460,82 @@ extern "C" int mpress_stash_free(const mpress_ctx_t* c, uint64_t* free_bytes) {
   return MPRESS_OK;
 }
 
-extern "C" int mpress_set_option(mpress_ctx_t* c, int key, int64_t value) {
-  if (!c) return fail(MPRESS_ERR_ARG, "mpress_set_option: null ctx");
-  std::lock_guard<std::mutex> lk(c->mu);
+namespace mpress {
+
+int set_swap_option(SwapOpts* o, int key, int64_t value) {
   switch (key) {
     case MPRESS_OPT_PATH:
       if (value != MPRESS_PATH_DIRECT && value != MPRESS_PATH_BULK && value != MPRESS_PATH_CE &&
           value != MPRESS_PATH_AUTO)
         return fail(MPRESS_ERR_ARG, "unknown path %lld", (long long)value);
-      c->path = (int)value;
-      c->variant = MPRESS_VARIANT_AUTO;  // variants are per path
+      o->path = (int)value;
+      o->variant = MPRESS_VARIANT_AUTO;  // variants are per path
       return MPRESS_OK;
     case MPRESS_OPT_MAX_CTAS:
       if (value < 0 || value > (1 << 20)) return fail(MPRESS_ERR_ARG, "bad max_ctas %lld", (long long)value);
-      c->max_ctas = (int)value;
+      o->max_ctas = (int)value;
       return MPRESS_OK;
     case MPRESS_OPT_PDL:
       if (value < 0 || value > 2) return fail(MPRESS_ERR_ARG, "MPRESS_OPT_PDL is 0, 1 or 2, not %lld", (long long)value);
-      c->pdl = (int)value;
+      o->pdl = (int)value;
       return MPRESS_OK;
     case MPRESS_OPT_ORDER:
       if (value != MPRESS_ORDER_INTERLEAVE && value != MPRESS_ORDER_PLAN)
         return fail(MPRESS_ERR_ARG, "unknown chunk order %lld", (long long)value);
-      c->order = (int)value;
+      o->order = (int)value;
       return MPRESS_OK;
     case MPRESS_OPT_PACE_MBPS:
       if (value < 0 || value > (int64_t)100000000)
         return fail(MPRESS_ERR_ARG, "MPRESS_OPT_PACE_MBPS is 0 (off) or a rate in MB/s up to 1e8, not %lld",
                     (long long)value);
-      c->pace_mbps = (uint64_t)value;
+      o->pace_mbps = (uint64_t)value;
       return MPRESS_OK;
     case MPRESS_OPT_SPLIT:
       if (value < MPRESS_SPLIT_BLOCKED || value > MPRESS_SPLIT_AUTO)
         return fail(MPRESS_ERR_ARG, "MPRESS_OPT_SPLIT is 0 (blocked), 1 (strided), 2 (dynamic) or 3 (auto), not %lld",
                     (long long)value);
-      c->split = (int)value;
+      o->split = (int)value;
       return MPRESS_OK;
     case MPRESS_OPT_VARIANT: {
-      const int nvar = c->path == MPRESS_PATH_BULK ? kBulkVariants
-                       : c->path == MPRESS_PATH_CE ? kCeVariants
-                       : c->path == MPRESS_PATH_AUTO ? 0 : kDirectVariants;
+      const int nvar = o->path == MPRESS_PATH_BULK ? kBulkVariants
+                       : o->path == MPRESS_PATH_CE ? kCeVariants
+                       : o->path == MPRESS_PATH_AUTO ? 0 : kDirectVariants;
       if (value != MPRESS_VARIANT_AUTO && (value < 0 || value >= nvar))
-        return fail(MPRESS_ERR_ARG, "variant %lld out of range for path %d", (long long)value, c->path);
-      c->variant = (int)value;
+        return fail(MPRESS_ERR_ARG, "variant %lld out of range for path %d", (long long)value, o->path);
+      o->variant = (int)value;
       return MPRESS_OK;
     }
   }
-  return fail(MPRESS_ERR_ARG, "unknown option %d", key);
+  return kNotSwapOption;
+}
+
+int get_swap_option(const SwapOpts& o, int key, int64_t* value) {
+  switch (key) {
+    case MPRESS_OPT_PATH: *value = o.path; return MPRESS_OK;
+    case MPRESS_OPT_MAX_CTAS: *value = o.max_ctas; return MPRESS_OK;
+    case MPRESS_OPT_VARIANT: *value = o.variant; return MPRESS_OK;
+    case MPRESS_OPT_ORDER: *value = o.order; return MPRESS_OK;
+    case MPRESS_OPT_PDL: *value = o.pdl; return MPRESS_OK;
+    case MPRESS_OPT_PACE_MBPS: *value = (int64_t)o.pace_mbps; return MPRESS_OK;
+    case MPRESS_OPT_SPLIT: *value = o.split; return MPRESS_OK;
+  }
+  return kNotSwapOption;
+}
+
+}  // namespace mpress
+
+extern "C" int mpress_set_option(mpress_ctx_t* c, int key, int64_t value) {
+  if (!c) return fail(MPRESS_ERR_ARG, "mpress_set_option: null ctx");
+  std::lock_guard<std::mutex> lk(c->mu);
+  const int rc = set_swap_option(&c->opt, key, value);
+  return rc == kNotSwapOption ? fail(MPRESS_ERR_ARG, "unknown option %d", key) : rc;
 }
 
 extern "C" int mpress_get_option(const mpress_ctx_t* c, int key, int64_t* value) {
   if (!c || !value) return fail(MPRESS_ERR_ARG, "mpress_get_option: null argument");
   std::lock_guard<std::mutex> lk(const_cast<mpress_ctx_t*>(c)->mu);  // set_option/autotune/run_copy write these
+  if (get_swap_option(c->opt, key, value) == MPRESS_OK) return MPRESS_OK;
   switch (key) {
-    case MPRESS_OPT_PATH: *value = c->path; return MPRESS_OK;
-    case MPRESS_OPT_MAX_CTAS: *value = c->max_ctas; return MPRESS_OK;
-    case MPRESS_OPT_VARIANT: *value = c->variant; return MPRESS_OK;
-    case MPRESS_OPT_ORDER: *value = c->order; return MPRESS_OK;
-    case MPRESS_OPT_PDL: *value = c->pdl; return MPRESS_OK;
-    case MPRESS_OPT_PACE_MBPS: *value = (int64_t)c->pace_mbps; return MPRESS_OK;
-    case MPRESS_OPT_SPLIT: *value = c->split; return MPRESS_OK;
     case MPRESS_OPT_TRANSPORT: *value = c->transport; return MPRESS_OK;
     case MPRESS_OPT_LAST_PATH: *value = c->last_path; return MPRESS_OK;
     case MPRESS_OPT_AUTO_OUT: *value = c->auto_path[mpress::kDirOut][1]; return MPRESS_OK;

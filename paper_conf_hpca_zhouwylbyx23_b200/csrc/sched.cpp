@@ -139,10 +139,10 @@ int record_done(mpress_ctx_s* c, cudaStream_t s, bool graph, EvRef* ev, EvRef* e
 }
 
 // Move every descriptor on `stream` with the context's path.
-int run_copy(mpress_ctx_s* c, int dir, const std::vector<CopyDesc>& d,
+int run_copy(mpress_ctx_s* c, const SwapOpts& o, int dir, const std::vector<CopyDesc>& d,
              const std::vector<int>& desc_peer, cudaStream_t stream, bool graph) {
   c->last_launches = 0;
-  int path = c->path;
+  int path = o.path;
   if (path == MPRESS_PATH_AUTO) {
     // full grid: per direction and size class, the kernel mpress_autotune
     // measured faster on this context's links (before it runs: direct below
@@ -153,7 +153,7 @@ int run_copy(mpress_ctx_s* c, int dir, const std::vector<CopyDesc>& d,
     // (over PCIe every SM kernel shape stops at ~52.6 GB/s, the engines at
     // ~56.9: profiles/r02/sweep_host_paths.jsonl)
     const int sms = sm_count(nullptr);
-    const bool capped = c->max_ctas > 0 && c->max_ctas <= sms;
+    const bool capped = o.max_ctas > 0 && o.max_ctas <= sms;
     uint64_t total = 0;
     for (const CopyDesc& x : d) total += x.len;
     int host = 0;
@@ -171,11 +171,11 @@ int run_copy(mpress_ctx_s* c, int dir, const std::vector<CopyDesc>& d,
     if (!graph && d.size() > (size_t)kParamDescMax && !c->ring) MP_TRY(table_ring_create(c->device, &c->ring));
     // Claim counters likewise: a replayed launch would reuse a slot that
     // later eager launches take (dynamic falls back to blocked there).
-    if (!graph && c->split >= MPRESS_SPLIT_DYNAMIC && !c->counters)
+    if (!graph && o.split >= MPRESS_SPLIT_DYNAMIC && !c->counters)
       MP_TRY(counter_ring_create(c->device, &c->counters));
-    return launch_copy(path, c->variant, dir, d.data(),
-                       c->order == MPRESS_ORDER_INTERLEAVE ? desc_peer.data() : nullptr, d.size(), c->max_ctas,
-                       c->pdl, stream, &c->last_launches, graph ? nullptr : c->ring, c->pace_mbps, c->split,
+    return launch_copy(path, o.variant, dir, d.data(),
+                       o.order == MPRESS_ORDER_INTERLEAVE ? desc_peer.data() : nullptr, d.size(), o.max_ctas,
+                       o.pdl, stream, &c->last_launches, graph ? nullptr : c->ring, o.pace_mbps, o.split,
                        graph ? nullptr : c->counters);
   }
 
@@ -216,12 +216,32 @@ int run_copy(mpress_ctx_s* c, int dir, const std::vector<CopyDesc>& d,
 
 using namespace mpress;
 
+namespace {
+int swap_out_locked(mpress_ctx_s* c, const SwapOpts& o, const mpress_plan_t* plan_, void* const* tensors,
+                    void* stream_, void* after, mpress_handle_t** out);
+}  // namespace
+
 extern "C" int mpress_swap_out(mpress_ctx_t* c, const mpress_plan_t* plan_, void* const* tensors,
                                void* stream_, void* after, mpress_handle_t** out) {
   if (!c || !plan_ || !out) return fail(MPRESS_ERR_ARG, "mpress_swap_out: null argument");
+  std::lock_guard<std::mutex> lk(c->mu);
+  return swap_out_locked(c, c->opt, plan_, tensors, stream_, after, out);
+}
+
+namespace mpress {
+int swap_out_with(mpress_ctx_s* c, const SwapOpts& o, const mpress_plan_t* plan_, void* const* tensors,
+                  void* stream_, void* after, mpress_handle_t** out) {
+  if (!c || !plan_ || !out) return fail(MPRESS_ERR_ARG, "mpress_swap_out: null argument");
+  std::lock_guard<std::mutex> lk(c->mu);
+  return swap_out_locked(c, o, plan_, tensors, stream_, after, out);
+}
+}  // namespace mpress
+
+namespace {
+int swap_out_locked(mpress_ctx_s* c, const SwapOpts& o, const mpress_plan_t* plan_, void* const* tensors,
+                    void* stream_, void* after, mpress_handle_t** out) {
   HP_START();
   *out = nullptr;
-  std::lock_guard<std::mutex> lk(c->mu);
   const uint64_t *units, *peer_bytes;
   const mpress_stripe* st;
   uint32_t n_st;
@@ -293,7 +313,7 @@ extern "C" int mpress_swap_out(mpress_ctx_t* c, const mpress_plan_t* plan_, void
   }
   if (after) cudaStreamWaitEvent(stream, static_cast<cudaEvent_t>(after), 0);
   HP_LAP(2, "out: descriptors");
-  rc = run_copy(c, kDirOut, d, dp, stream, graph);
+  rc = run_copy(c, o, kDirOut, d, dp, stream, graph);
   HP_LAP(3, "out: run_copy (launch)");
   if (rc == MPRESS_OK) rc = record_done(c, stream, graph, &h->out_done, &h->out_ext, "cudaEventRecord(out_done)");
   HP_LAP(4, "out: event record");
@@ -313,10 +333,26 @@ extern "C" int mpress_swap_out(mpress_ctx_t* c, const mpress_plan_t* plan_, void
   return MPRESS_OK;
 }
 
+int swap_in_locked(mpress_ctx_s* c, const SwapOpts& o, mpress_handle_t* h, void* const* dst, void* stream_);
+}  // namespace
+
 extern "C" int mpress_swap_in(mpress_ctx_t* c, mpress_handle_t* h, void* const* dst, void* stream_) {
   if (!c || !h) return fail(MPRESS_ERR_ARG, "mpress_swap_in: null argument");
-  HP_START();
   std::lock_guard<std::mutex> lk(c->mu);
+  return swap_in_locked(c, c->opt, h, dst, stream_);
+}
+
+namespace mpress {
+int swap_in_with(mpress_ctx_s* c, const SwapOpts& o, mpress_handle_t* h, void* const* dst, void* stream_) {
+  if (!c || !h) return fail(MPRESS_ERR_ARG, "mpress_swap_in: null argument");
+  std::lock_guard<std::mutex> lk(c->mu);
+  return swap_in_locked(c, o, h, dst, stream_);
+}
+}  // namespace mpress
+
+namespace {
+int swap_in_locked(mpress_ctx_s* c, const SwapOpts& o, mpress_handle_t* h, void* const* dst, void* stream_) {
+  HP_START();
   if (h->ctx != c || !c->handles.count(h)) return fail(MPRESS_ERR_ARG, "mpress_swap_in: handle not of this context");
   if (h->state != MPRESS_STATE_OUT_PENDING && h->state != MPRESS_STATE_OUT)
     return fail(MPRESS_ERR_STATE, "mpress_swap_in: handle is in state %d, not swapped out", h->state);
@@ -344,7 +380,7 @@ extern "C" int mpress_swap_in(mpress_ctx_t* c, mpress_handle_t* h, void* const* 
   }
   if (h->graph || !same_stream(h->out_stream, stream)) cudaStreamWaitEvent(stream, h->out_done.get(), 0);
   HP_LAP(5, "in: checks + capture query + desc");
-  int rc = run_copy(c, kDirIn, d, dp, stream, h->graph);
+  int rc = run_copy(c, o, kDirIn, d, dp, stream, h->graph);
   HP_LAP(6, "in: run_copy (launch)");
   if (rc != MPRESS_OK) return rc;
   EvRef in_done, in_ext;
@@ -376,6 +412,7 @@ extern "C" int mpress_swap_in(mpress_ctx_t* c, mpress_handle_t* h, void* const* 
   HP_LAP(8, "in: fences + slice release");
   return MPRESS_OK;
 }
+}  // namespace
 
 extern "C" int mpress_wait(mpress_ctx_t* c, mpress_handle_t* h, void* consumer) {
   if (!c || !h || h->ctx != c) return fail(MPRESS_ERR_ARG, "mpress_wait: bad argument");
@@ -567,7 +604,7 @@ extern "C" int mpress_autotune(mpress_ctx_t* c, uint64_t probe_bytes, int trials
   }
   // warm-up round (-1), then `trials` rounds alternating which path goes first
   const int paths[2] = {MPRESS_PATH_DIRECT, MPRESS_PATH_BULK};
-  if (rc == MPRESS_OK && c->split >= MPRESS_SPLIT_DYNAMIC && !c->counters)
+  if (rc == MPRESS_OK && c->opt.split >= MPRESS_SPLIT_DYNAMIC && !c->counters)
     rc = counter_ring_create(c->device, &c->counters);  // the probes run the context's split
   std::vector<float> t[2][2][2];  // [class][path][dir], ms per launch
   for (int r = -1; r < trials; ++r) {
@@ -581,12 +618,12 @@ extern "C" int mpress_autotune(mpress_ctx_t* c, uint64_t probe_bytes, int trials
         cudaEventRecord(ev[0], stream);
         for (int i = 0; i < reps && rc == MPRESS_OK; ++i)
           rc = launch_copy(paths[pi], MPRESS_VARIANT_AUTO, kDirOut, dout[cls][i].data(), grp.data(),
-                           dout[cls][i].size(), 0, c->pdl, stream, &launches, nullptr, 0, c->split,
+                           dout[cls][i].size(), 0, c->opt.pdl, stream, &launches, nullptr, 0, c->opt.split,
                            c->counters);
         cudaEventRecord(ev[1], stream);
         for (int i = 0; i < reps && rc == MPRESS_OK; ++i)
           rc = launch_copy(paths[pi], MPRESS_VARIANT_AUTO, kDirIn, din[cls][i].data(), grp.data(),
-                           din[cls][i].size(), 0, c->pdl, stream, &launches, nullptr, 0, c->split,
+                           din[cls][i].size(), 0, c->opt.pdl, stream, &launches, nullptr, 0, c->opt.split,
                            c->counters);
         cudaEventRecord(ev[2], stream);
         cudaError_t e = cudaEventSynchronize(ev[2]);

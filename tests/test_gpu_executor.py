@@ -147,3 +147,50 @@ def test_executor_release_then_reuse():
         ex.free()
     finally:
         ctx.finalize()
+
+
+@pytest.mark.parametrize("path", [mp.PATH_CE, mp.PATH_BULK, mp.PATH_DIRECT], ids=["ce", "bulk", "direct"])
+def test_executor_own_swap_options(path):
+    """mpress_executor_set_option: the executor's swaps run on its own path
+    (OPT_LAST_PATH after a step) while the context keeps its own (a plain
+    swap afterwards runs the context's); options are copied at creation,
+    validated like mpress_set_option, and non-swap options are refused."""
+    M = 2
+    ctx, pl, sizes = _setup(M)
+    s_out, s_in = torch.cuda.Stream(), torch.cuda.Stream()
+    comp = torch.cuda.current_stream()
+    try:
+        ctx.set_option(mp.OPT_MAX_CTAS, 5)
+        ex = mp.Executor(ctx, pl, 2, 0, M, 10_000, 20_000, 5_000, 5_000, s_out, s_in)
+        assert ex.get_option(mp.OPT_MAX_CTAS) == 5            # copied from the context
+        assert ex.get_option(mp.OPT_PATH) == mp.PATH_AUTO
+        ex.set_option(mp.OPT_PATH, path)
+        ex.set_option(mp.OPT_MAX_CTAS, 0)
+        assert ctx.get_option(mp.OPT_PATH) == mp.PATH_AUTO    # the context is unchanged
+        assert ctx.get_option(mp.OPT_MAX_CTAS) == 5
+        with pytest.raises(mp.MPressError) as ei:
+            ex.set_option(mp.OPT_TRANSPORT, 0)                 # not a swap option
+        assert ei.value.code == mp.ERR_ARG
+        with pytest.raises(mp.MPressError):
+            ex.set_option(mp.OPT_VARIANT, 99)
+        src = [[torch.empty(n, dtype=torch.uint8, device="cuda") for n in sizes] for _ in range(M)]
+        dst = [[torch.zeros(n, dtype=torch.uint8, device="cuda") for n in sizes] for _ in range(M)]
+        for m in range(M):
+            for i, t in enumerate(src[m]):
+                synth_dev.fill(t, 70 + m, i)
+            ex.restore_to(m, dst[m])
+        for j in range(ex.ops):
+            kind, m = ex.before(j, comp)
+            ex.after(j, comp, src[m] if kind == "F" else None)
+        torch.cuda.synchronize()
+        assert ctx.get_option(mp.OPT_LAST_PATH) == path
+        for m in range(M):
+            for i, t in enumerate(dst[m]):
+                assert synth_dev.check(t, 70 + m, i) == 0, (m, i)
+        h = ctx.swap_out(pl, src[0])                            # a plain swap: the context's options
+        torch.cuda.synchronize()
+        assert ctx.get_option(mp.OPT_LAST_PATH) in (mp.PATH_DIRECT, mp.PATH_BULK)   # AUTO at 5 CTAs
+        h.free(force=True)
+        ex.free()
+    finally:
+        ctx.finalize()
