@@ -37,7 +37,7 @@ def setup(sizes, peers_n, copies=1):
     part[0] = [copies * u * mp.DEFAULT_GRANULE for u in pl.units]
     ctx = mp.Context.local(world, 0, [0] * world, part)
     ctx.set_option(mp.OPT_PDL, int(os.environ.get("SWEEP_PDL", "1")))
-    ctx.set_option(mp.OPT_SPLIT, int(os.environ.get("SWEEP_SPLIT", "0")))
+    ctx.set_option(mp.OPT_SPLIT, int(os.environ.get("SWEEP_SPLIT", "3")))
     src = [torch.empty(s, dtype=torch.uint8, device="cuda") for s in sizes]
     for i, t in enumerate(src):
         synth_dev.fill(t, 77, i)
