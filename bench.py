@@ -619,11 +619,18 @@ def main():
 
     # The legs below add context to the headline; a failure in one is
     # reported in its key instead of losing the measured line.
+    leg_wall = {}
+
     def leg(fn, *a):
+        t0 = time.time()
         try:
             return fn(*a)
         except Exception as exc:  # pragma: no cover - reported, not hidden
             return {"error": "%s: %s" % (type(exc).__name__, exc)}
+        finally:
+            name = (fn.__name__ + ("_ce" if any(x is True for x in a[-2:]) else "") +
+                    ("_fc1" if any(isinstance(x, str) and x == "gpt_fc1" for x in a) else ""))
+            leg_wall[name] = round(time.time() - t0, 2)
 
     e2e = leg(run_e2e, args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap_stream, n, dist)
     e2e_zc = None if args.no_e2e_zero_copy else leg(run_e2e_zero_copy, args, ctx, mp, world, source, per_copy,
@@ -633,8 +640,10 @@ def main():
     cap_cal = None
     args.gemm_swap = "auto:-1:%d" % (args.gemm_cap if args.gemm_cap > 0 else 148)
     if not args.no_gemm and args.gemm_cap <= 0:
+        t0 = time.time()
         cap_cal = calibrate_gemm_cap(args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap_stream, n,
                                      dist)
+        leg_wall["calibrate_gemm_cap"] = round(time.time() - t0, 2)
         args.gemm_swap = cap_cal["chosen"]
     gemm = None if args.no_gemm else leg(gemm_interference, args, ctx, mp, world, source, per_copy, bw,
                                          sizes, src, dst, swap_stream, n, dist)
@@ -687,6 +696,7 @@ def main():
             "gemm_cap_calibration": cap_cal,
             "planner": planner, "other_configs": others, "cfg5": cfg5, "cfg5_ce": cfg5_ce,
             "single_source": single, "duplex": duplex,
+            "leg_wall_s": leg_wall,
             "duplex_gbs": duplex.get("duplex_gbs") if isinstance(duplex, dict) else None,
             "parity": "round trip bit-exact vs generator (all %d tensors x %d ranks)" % (47 * mb, n),
             "value_is": "per source GPU: one rank's swapped bytes (out + in) / max-over-ranks step time",
@@ -1732,7 +1742,9 @@ def run_e2e_zero_copy(args, ctx, mp, world, source, per_copy, bw, sizes, n, dist
     import numpy as np
     import torch
     from synth import device as synth_dev
-    mb = MICRO_BATCHES if n == 1 else 2   # as run_e2e: N ranks on one host do not pin N x 14 GiB
+    # as run_e2e: N ranks on one host do not pin N x 14 GiB; never more
+    # micro-batches than the partitions hold (out(m+1) beside in(m) needs 2)
+    mb = min(args.micro_batches, MICRO_BATCHES if n == 1 else 2)
     nt = len(sizes)
     L = _Local()
     st = {}
