@@ -20,7 +20,7 @@ from synth import splitmix64_bytes, workloads
 pytestmark = pytest.mark.gpu
 
 
-def _sampled_roundtrip(world, source, spare, bw, sizes, seed, samples=64, path=None):
+def _sampled_roundtrip(world, source, spare, bw, sizes, seed, samples=64, path=None, variant=-1, max_ctas=0):
     o = oracle.plan(world, source, spare, bw, sizes)
     pl = mp.plan(world, source, spare, bw, sizes)
     assert pl.stripes == [tuple(s) for s in o["stripes"]]
@@ -31,6 +31,9 @@ def _sampled_roundtrip(world, source, spare, bw, sizes, seed, samples=64, path=N
     try:
         if path is not None:
             ctx.set_option(mp.OPT_PATH, path)
+            if variant >= 0:
+                ctx.set_option(mp.OPT_VARIANT, variant)
+        ctx.set_option(mp.OPT_MAX_CTAS, max_ctas)
         src = []
         for i, n in enumerate(sizes):
             t = torch.empty(n, dtype=torch.uint8, device="cuda")
@@ -117,3 +120,18 @@ def test_stripe_longer_than_4gib(path):
     chunk arithmetic), with a ragged tail."""
     spare = [0, 8 << 30]
     _sampled_roundtrip(2, 0, spare, [0, 1], [(6 << 30) + 17], seed=4100, path=path)
+
+
+@pytest.mark.parametrize("path,variant,cap", [(mp.PATH_BULK, 7, 148), (mp.PATH_AUTO, -1, 64)],
+                         ids=["gemm_leg_bulk7x148", "auto_capped64"])
+def test_config2_micro_batch_gemm_leg_settings(path, variant, cap):
+    """BJ:8 / BJ:11: one full Bert stage-0 micro-batch (47 tensors, 900 MiB)
+    over 3 peers in the launch configurations the bench's GEMM legs time
+    (the one-warp TMA shape on every SM, with the AUTO split's dynamic
+    claims; AUTO capped at 64 CTAs = direct shape 9): every stash byte
+    against the oracle's byte model, every restored byte."""
+    peers = [1, 2, 3]
+    spare = workloads.spare_vector(4, 0, peers, spare=4 << 30)
+    bw = workloads.bw_vector(4, 0, peers)
+    _sampled_roundtrip(4, 0, spare, bw, workloads.cfg2_sizes(1), seed=2100 + cap, path=path, variant=variant,
+                       max_ctas=cap)
