@@ -15,17 +15,19 @@
 //     With several sources swapping at once (config 5, or every rank of the
 //     N-GPU bench) each peer's NVLink ingress is then shared by all sources
 //     all the time instead of every source converging on its first peer;
-//   * the CTAs walk that interleaved sequence with a grid stride, so any grid
-//     size is load-balanced and adjacent chunks are in flight on different
-//     SMs at once;
+//   * the CTAs share that interleaved sequence by MPRESS_OPT_SPLIT: a
+//     contiguous block each, a grid stride, or blocks claimed from a
+//     per-launch counter so all CTAs work on one moving front of it (AUTO:
+//     the stride for short launches, the claims for long TMA launches --
+//     see Cursor and DynClaim below);
 //   * the grid is capped (MPRESS_OPT_MAX_CTAS) so a concurrent GEMM keeps
 //     most SMs;
 //   * every address is 16-B aligned (tensor pointers are checked; stripe
 //     offsets are multiples of 256, R6), so bodies move int4 / bulk pieces and
 //     only the last <16 bytes of a tensor take a byte loop.
 //
-// PATH_DIRECT: THREADS threads, each issuing UNROLL independent 16-B loads
-//   before its UNROLL stores, L1 bypassed on both sides.  Peer addresses
+// PATH_DIRECT: THREADS threads, each issuing UNROLL independent 16- or 32-B
+//   loads before its UNROLL stores, L1 bypassed on both sides.  Peer addresses
 //   route over NVLink by their VA; loads of peer memory bypass the local L2
 //   (B300_MICROARCH.md "NVLink"), so the depth of outstanding loads sets
 //   swap-in bandwidth (Little's law).
