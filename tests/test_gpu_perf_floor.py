@@ -1,6 +1,7 @@
 """Performance floors on one B200 (loopback peers): generous lower bounds that
-only a gross regression would break -- the measured values are ~1.25-1.3x
-above them (profiles/r02/).  The bench, not these tests, is the
+only a gross regression would break -- the measured values are ~1.65x
+above them (profiles/r02/), so a slower box or a noisy neighbour does not
+trip them.  The bench, not these tests, is the
 measurement."""
 import statistics
 
@@ -32,8 +33,9 @@ def _rate(ctx, pl, src, dst, s, nbytes, reps=10):
 
 def test_cfg2_micro_batch_round_trip_floor():
     """One Bert stage-0 micro-batch (47 tensors, 900 MiB) over 3 loopback
-    peers, default path and grid: >= 2500 GB/s of swapped bytes (measured
-    ~3150-3200; roofline 3276 = half the measured HBM copy bandwidth)."""
+    peers, default path and grid: >= 2000 GB/s of swapped bytes (measured
+    ~3330-3350 with the AUTO split; half the measured HBM copy bandwidth is
+    ~3270)."""
     sizes = workloads.cfg2_sizes(1)
     peers = [1, 2, 3]
     spare = workloads.spare_vector(4, 0, peers, spare=24 << 30)
@@ -52,18 +54,18 @@ def test_cfg2_micro_batch_round_trip_floor():
         ps, pd = mp.pointers(src), mp.pointers(dst)
         gbs = _rate(ctx, pl, ps, pd, s, sum(sizes))
         assert all(synth_dev.check(d, 90, i) == 0 for i, d in enumerate(dst))
-        assert gbs >= 2500, "cfg2 round trip %.0f GB/s (floor 2500)" % gbs
+        assert gbs >= 2000, "cfg2 round trip %.0f GB/s (floor 2000)" % gbs
         # the capped direct shape (AUTO at 64 CTAs: 128 x 8 x 32 B, shape 9)
         # alone: measured ~1830 (round 1's shape 7: ~1120)
         ctx.set_option(mp.OPT_MAX_CTAS, 64)
         capped = _rate(ctx, pl, ps, pd, s, sum(sizes))
-        assert capped >= 1400, "capped round trip %.0f GB/s (floor 1400)" % capped
+        assert capped >= 1100, "capped round trip %.0f GB/s (floor 1100)" % capped
         # the TMA shape the bench runs beside a GEMM (bulk 7, one CTA per SM):
         # measured ~1280
         ctx.set_option(mp.OPT_PATH, mp.PATH_BULK)
         ctx.set_option(mp.OPT_VARIANT, 7)
         ctx.set_option(mp.OPT_MAX_CTAS, 148)
         tma = _rate(ctx, pl, ps, pd, s, sum(sizes))
-        assert tma >= 1000, "bulk 7 x 148 round trip %.0f GB/s (floor 1000)" % tma
+        assert tma >= 760, "bulk 7 x 148 round trip %.0f GB/s (floor 760)" % tma
     finally:
         ctx.finalize()
