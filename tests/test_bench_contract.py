@@ -70,3 +70,5 @@ def test_round2_keys():
     # the power-capped leg: >= 5 paired windows of ~3 s (the verdict's "windows of 3 s or more")
     assert sus["rounds"] >= 5 and sus["slowdown_ci95"][0] <= sus["slowdown"] <= sus["slowdown_ci95"][1]
     assert sus["alone_ms"] * int(sus["gemm"].split("windows of ")[1].split()[0]) >= 2500
+    if "fallback" in sus:   # re-measured with --gemm-sus-fallback: the first setting missed the rate
+        assert sus["first_setting"]["swap_gbs_during"] < 720 and sus["swap_setting"] != sus["first_setting"]["swap_setting"]
