@@ -658,7 +658,8 @@ def main():
     # again with --gemm-sus-fallback (unpaced), and the first result is kept
     # in the line.  Every rank sees the slowest rank's rate, so all agree.
     if (isinstance(gemm_sus, dict) and gemm_sus.get("swap_gbs_during") is not None and args.gemm_sus_fallback
-            and gemm_sus["swap_gbs_during"] < args.gemm_target_gbs and args.gemm_cap <= 0):
+            and gemm_sus["swap_gbs_during"] < args.gemm_target_gbs and args.gemm_cap <= 0
+            and gemm_sus.get("swap_setting") != args.gemm_sus_fallback):
         alt = leg(gemm_windows, args, ctx, mp, world, source, per_copy, bw, sizes, src, dst, swap_stream, n, dist,
                   args.gemm_sus_fallback, 0)
         if isinstance(alt, dict) and "error" not in alt:
