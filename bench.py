@@ -84,9 +84,11 @@ def parse():
                     help="swap grid cap (CTAs = SMs touched) while the concurrent GEMM runs (AUTO path -> "
                          "direct shape 9); 0 = calibrate: the first of --gemm-swap-candidates whose swap rate "
                          "on this run's links reaches --gemm-target-gbs / 0.85")
-    ap.add_argument("--gemm-swap-candidates", default="bulk:7:148,auto:-1:148,auto:-1:96,auto:-1:64",
+    ap.add_argument("--gemm-swap-candidates", default="bulk:9:148,bulk:7:148,auto:-1:148,auto:-1:96,auto:-1:64",
                     help="path:variant:max_ctas settings for the GEMM-concurrent swap, cheapest for the GEMM "
-                         "first: one-warp TMA CTAs (4 x 4 KiB of shared memory) on every SM cost the "
+                         "first: bulk 9 = a TMA warp (4 x 4 KiB of shared memory) plus an LSU warp per SM, "
+                         "1.4x bulk 7's rate at the same burst-GEMM cost (profiles/r02/hybrid/); "
+                         "one-warp TMA CTAs (4 x 4 KiB of shared memory) on every SM cost the "
                          "power-capped GEMM ~12%% where 128-thread direct CTAs cost ~18%% at the same rate "
                          "(profiles/r02/gemm_windows_*.jsonl); among the direct settings one light "
                          "CTA on every SM cost no more than 64 or 96 busier SMs (gemm_leg_settings.jsonl)")

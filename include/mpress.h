@@ -462,8 +462,10 @@ MPRESS_API int mpress_stash_free(const mpress_ctx_t* ctx, uint64_t* free_bytes);
  * bulk: 0 = 6 slots x 32 KiB, 1 = 12 x 16 KiB, 2 = 3 x 64 KiB (one CTA per
  * SM), 3 = 3 x 32 KiB (one per SM; twice as many fit), 4 = 4 x 16 KiB (three
  * per SM),
- * 5 = 2 x 8 KiB, 6 = 3 x 4 KiB, 7 = 4 x 4 KiB, 8 = 8 x 2 KiB (one per SM;
- * small enough to share an SM with a GEMM CTA);
+ * 5 = 2 x 8 KiB, 6 = 3 x 4 KiB, 7 = 4 x 4 KiB, 8 = 8 x 2 KiB, 9 = 4 x 4 KiB
+ * plus a second warp copying 4 x 4 KiB through registers, both claiming
+ * work under the dynamic split (one per SM; small enough to share an SM
+ * with a GEMM CTA);
  * copy engines: 0 = cudaMemcpyAsync per stripe on one side stream per peer
  * (the only copy-engine variant);
  * MPRESS_VARIANT_AUTO (-1, default) = direct 9 when the grid is capped at

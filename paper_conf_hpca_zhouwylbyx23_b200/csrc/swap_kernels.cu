@@ -192,7 +192,9 @@ struct DynClaim {
   uint64_t next_s = 0;   // the prefetched claim (claiming thread)
   uint32_t next_q = 0;
   uint32_t qmax;
-  __device__ DynClaim(unsigned long long* c, uint64_t p, uint32_t qlim) : ctr(c), P(p) {
+  uint64_t workers;      // claimants in the launch: CTAs, or warps of a two-warp CTA
+  __device__ DynClaim(unsigned long long* c, uint64_t p, uint32_t qlim, uint64_t w = 0)
+      : ctr(c), P(p), workers(w ? w : gridDim.x) {
     qmax = qlim >> 16;
     qmax = qmax == 0 || qmax > QMAX ? QMAX : qmax;
     qmin = qlim & 0xFFFFu;
@@ -200,13 +202,13 @@ struct DynClaim {
   }
   __device__ void claim(uint64_t seen) {
     const uint64_t rem = seen < P ? P - seen : 0;
-    const uint64_t q = rem / (2ull * gridDim.x);
+    const uint64_t q = rem / (2ull * workers);
     next_q = q < qmin ? qmin : q > qmax ? qmax : (uint32_t)q;
     next_s = atomicAdd(ctr, (unsigned long long)next_q);
   }
   __device__ void done() {
     __threadfence();
-    if (atomicAdd(ctr + 1, 1ull) == gridDim.x - 1ull) {
+    if (atomicAdd(ctr + 1, 1ull) == workers - 1ull) {
       atomicExch(ctr, 0ull);
       atomicExch(ctr + 1, 0ull);
     }
@@ -518,6 +520,71 @@ __device__ __forceinline__ uint64_t shfl64(uint64_t v, int lane) {
   return ((uint64_t)hi << 32) | lo;
 }
 
+// Bulk shape 9 (beside a GEMM): a second warp in the CTA copies pieces
+// through registers (LDG/STG, 4 pieces x 2^SHIFT bytes in flight) while the
+// first drives the TMA ring, both claiming their own blocks from the
+// launch's counter -- twice the bytes in flight per SM inside the shared
+// memory a GEMM CTA leaves.  Only with the dynamic claims; under a static
+// split (small launches, graph capture) the TMA warp moves everything.
+template <int SHIFT, int CAP>
+__device__ __forceinline__ void bulk_lsu_warp(const CopyTable<CAP>& t, uint64_t workers) {
+  constexpr uint32_t kVec = (1u << SHIFT) / 16u / 32u;  // 16-byte vectors per lane per piece
+  constexpr int kPieces = 4;
+  const uint32_t lane = threadIdx.x & 31u;
+  if (!t.dyn) return;
+  const uint64_t P = (uint64_t)t.n_groups << t.rounds_log2;
+  DynClaim<32> dc(t.dyn, P, t.qlim, workers);
+  if (lane == 0) dc.claim(0);
+  Cursor<CAP> cur(t, lane, 32u);
+  for (;;) {
+    const uint64_t b = shfl64(dc.next_s, 0);
+    const uint32_t q = __shfl_sync(0xffffffffu, dc.next_q, 0);
+    if (b >= P) break;
+    if (lane == 0) dc.claim(b + q);
+    cur.init(b + lane, 32u, b + q < P ? b + q : P);   // q <= 32: one position per lane at most
+    uint32_t c, sd;
+    const bool v = cur.next(&c, &sd);
+    Piece mine{nullptr, nullptr, 0};
+    if (v) {
+      mine = bulk_piece<SHIFT>(t, c, sd);
+      if (c + 1 == t.first_chunk[sd + 1]) {  // last chunk of descriptor sd: its tail
+        const CopyDesc& d = t.d[sd];
+        for (uint64_t x = d.len & ~15ull; x < d.len; ++x)
+          static_cast<uint8_t*>(d.dst)[x] = static_cast<const uint8_t*>(d.src)[x];
+      }
+    }
+    __syncwarp();
+    uint32_t mask = __ballot_sync(0xffffffffu, mine.bytes != 0);
+    while (mask) {
+      const int4* src[kPieces];
+      int4* dst[kPieces];
+      uint32_t nv[kPieces];
+#pragma unroll
+      for (int p = 0; p < kPieces; ++p) {
+        const int j = mask ? __ffs(mask) - 1 : 0;
+        const bool has = mask != 0;
+        if (has) mask &= mask - 1;
+        src[p] = reinterpret_cast<const int4*>(shfl64(reinterpret_cast<uint64_t>(mine.src), j));
+        dst[p] = reinterpret_cast<int4*>(shfl64(reinterpret_cast<uint64_t>(mine.dst), j));
+        const uint32_t nb = __shfl_sync(0xffffffffu, mine.bytes, j);
+        nv[p] = has ? nb >> 4 : 0u;
+      }
+      int4 r[kPieces][kVec];
+#pragma unroll
+      for (int p = 0; p < kPieces; ++p)
+#pragma unroll
+        for (uint32_t k = 0; k < kVec; ++k)
+          if (lane + 32u * k < nv[p]) r[p][k] = ld_stream(src[p] + lane + 32u * k);
+#pragma unroll
+      for (int p = 0; p < kPieces; ++p)
+#pragma unroll
+        for (uint32_t k = 0; k < kVec; ++k)
+          if (lane + 32u * k < nv[p]) st_stream(dst[p] + lane + 32u * k, r[p][k]);
+    }
+  }
+  if (lane == 0) dc.done();
+}
+
 // One warp per CTA: lane 0 streams pieces of 2^SHIFT bytes through STAGES
 // shared-memory slots with the SM's bulk-copy engine (cp.async.bulk G->S with
 // mbarrier completion, then S->G bulk stores).  The 32 lanes resolve the
@@ -535,7 +602,7 @@ __device__ __forceinline__ uint64_t shfl64(uint64_t v, int lane) {
 // store piece k-STAGES+1 and wait for all but the newest store's read
 // (read 1), keeping a store in flight -- for 3 x 32 KiB waiting on the
 // newest 32 KiB read cost 5% (profiles/r02/bulk_ring_ab.txt).
-template <int DIR, int SHIFT, int STAGES, int CAP>
+template <int DIR, int SHIFT, int STAGES, int CAP, int LSU>
 __device__ __forceinline__ void bulk_body(const CopyTable<CAP>& t) {
   constexpr uint32_t kSlot = 1u << SHIFT;
   constexpr bool kEager = SHIFT <= 12;
@@ -543,9 +610,14 @@ __device__ __forceinline__ void bulk_body(const CopyTable<CAP>& t) {
   __shared__ __align__(8) uint64_t bars[STAGES];
   __shared__ uint8_t* ring_dst[STAGES];
   __shared__ uint32_t ring_bytes[STAGES];
-  const uint32_t lane = threadIdx.x;
+  const uint32_t lane = threadIdx.x & 31u;
+  const uint64_t workers = (uint64_t)gridDim.x * (1 + LSU);
 
   pdl_enter();
+  if (LSU && threadIdx.x >= 32) {
+    bulk_lsu_warp<SHIFT, CAP>(t, workers);
+    return;
+  }
   if (lane == 0) {
     for (int k = 0; k < STAGES; ++k) mbar_init(&bars[k], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -569,7 +641,7 @@ __device__ __forceinline__ void bulk_body(const CopyTable<CAP>& t) {
   // resolver lane; a new block is taken when every lane's cursor is empty.
   const bool dyn = t.dyn != nullptr;
   const uint64_t P = (uint64_t)t.n_groups << t.rounds_log2;
-  DynClaim<32> dc(t.dyn, P, t.qlim);
+  DynClaim<32> dc(t.dyn, P, t.qlim, workers);
   if (dyn) {
     cur.init(0, 1, 0);
     if (lane == 0) dc.claim(0);
@@ -639,16 +711,16 @@ __device__ __forceinline__ void bulk_body(const CopyTable<CAP>& t) {
   }
 }
 
-template <int DIR, int SHIFT, int STAGES, int CAP>
-__global__ void __launch_bounds__(32)
+template <int DIR, int SHIFT, int STAGES, int CAP, int LSU>
+__global__ void __launch_bounds__(32 * (1 + LSU))
 mp_swap_bulk(const __grid_constant__ CopyTable<CAP> t) {
-  bulk_body<DIR, SHIFT, STAGES, CAP>(t);
+  bulk_body<DIR, SHIFT, STAGES, CAP, LSU>(t);
 }
 
-template <int DIR, int SHIFT, int STAGES, int CAP>
-__global__ void __launch_bounds__(32)
+template <int DIR, int SHIFT, int STAGES, int CAP, int LSU>
+__global__ void __launch_bounds__(32 * (1 + LSU))
 mp_swap_bulk_g(const CopyTable<CAP>* __restrict__ tp) {
-  bulk_body<DIR, SHIFT, STAGES, CAP>(*tp);
+  bulk_body<DIR, SHIFT, STAGES, CAP, LSU>(*tp);
 }
 
 // ---------------------------------------------------------------- variants
@@ -670,9 +742,10 @@ struct Shape {
 // 12 (128,8,32 + L2 evict-first loads and stores) 13 (32,16,32: one warp,
 // 16 KiB in flight -- the direct twin of the one-warp bulk shapes)
 // bulk (piece, stages, CTAs/SM): 0 (32K,6,1) 1 (16K,12,1) 2 (64K,3,1) 3 (32K,3,1)
-// 4 (16K,4,3) 5 (8K,2,1) 6 (4K,3,1) 7 (4K,4,1) 8 (2K,8,1) -- 5-8 use 16 / 12 /
-// 16 / 16 KB of shared memory, small enough to sit beside a cuBLAS GEMM CTA
-// (214 KB of the SM's 233.5 KB)
+// 4 (16K,4,3) 5 (8K,2,1) 6 (4K,3,1) 7 (4K,4,1) 8 (2K,8,1) 9 (4K,4,1 plus an
+// LSU warp with 4 x 4 KiB in registers, dynamic claims only) -- 5-9 use 16 /
+// 12 / 16 / 16 / 16 KB of shared memory, small enough to sit beside a cuBLAS
+// GEMM CTA (214 KB of the SM's 233.5 KB)
 constexpr Shape kDirect[kDirectVariants] = {
     {256, 15, 0, 2, 16, 0}, {512, 16, 0, 1, 16, 1}, {256, 16, 0, 2, 16, 2}, {1024, 16, 0, 1, 16, 3},
     {128, 14, 0, 4, 16, 4}, {256, 15, 0, 2, 32, 0}, {256, 16, 0, 2, 32, 2}, {128, 14, 0, 4, 32, 4},
@@ -681,7 +754,8 @@ constexpr Shape kDirect[kDirectVariants] = {
 constexpr Shape kBulk[kBulkVariants] = {
     {32, 15, 6u << 15, 1, 16, 0}, {32, 14, 12u << 14, 1, 16, 1}, {32, 16, 3u << 16, 1, 16, 2},
     {32, 15, 3u << 15, 1, 16, 3}, {32, 14, 4u << 14, 3, 16, 4}, {32, 13, 2u << 13, 1, 16, 5},
-    {32, 12, 3u << 12, 1, 16, 6}, {32, 12, 4u << 12, 1, 16, 7}, {32, 11, 8u << 11, 1, 16, 8}};
+    {32, 12, 3u << 12, 1, 16, 6}, {32, 12, 4u << 12, 1, 16, 7}, {32, 11, 8u << 11, 1, 16, 8},
+    {64, 12, 4u << 12, 1, 16, 9}};
 
 template <int CAP>
 using KernelFn = void (*)(CopyTable<CAP>);
@@ -690,10 +764,10 @@ using KernelFnG = void (*)(const CopyTable<CAP>*);
 
 // Entry point of one instantiation; `if constexpr` keeps the pointer-table
 // (G) kernels from being instantiated for the capacities that never use them.
-template <int CAP, bool G, int D, int SH, int ST>
+template <int CAP, bool G, int D, int SH, int ST, int LSU = 0>
 void* bulk_ptr() {
-  if constexpr (G) return reinterpret_cast<void*>(mp_swap_bulk_g<D, SH, ST, CAP>);
-  else return reinterpret_cast<void*>(mp_swap_bulk<D, SH, ST, CAP>);
+  if constexpr (G) return reinterpret_cast<void*>(mp_swap_bulk_g<D, SH, ST, CAP, LSU>);
+  else return reinterpret_cast<void*>(mp_swap_bulk<D, SH, ST, CAP, LSU>);
 }
 template <int CAP, bool G, int D, int T, int U, int VB, bool H, bool PF>
 void* direct_ptr() {
@@ -721,6 +795,7 @@ std::conditional_t<G, KernelFnG<CAP>, KernelFn<CAP>> kernel_for(int path, int va
       case 6: k = MP_BULK(12, 3); break;
       case 7: k = MP_BULK(12, 4); break;
       case 8: k = MP_BULK(11, 8); break;
+      case 9: k = o ? bulk_ptr<CAP, G, kDirOut, 12, 4, 1>() : bulk_ptr<CAP, G, kDirIn, 12, 4, 1>(); break;
       default: k = MP_BULK(15, 6); break;
     }
   } else {

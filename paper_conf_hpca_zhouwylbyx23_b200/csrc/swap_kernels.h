@@ -19,7 +19,7 @@ struct CopyDesc {
 
 constexpr int kMaxDescPerLaunch = 1024;  // fits the 32 KB kernel-parameter space
 constexpr int kDirectVariants = 14;      // MPRESS_OPT_VARIANT range, direct path
-constexpr int kBulkVariants = 9;         // MPRESS_OPT_VARIANT range, bulk path
+constexpr int kBulkVariants = 10;        // MPRESS_OPT_VARIANT range, bulk path
 constexpr int kCeVariants = 1;           // copy engines: 0 = cudaMemcpyAsync per stripe, per-peer streams
 
 enum CopyDir { kDirOut = 0, kDirIn = 1 };

@@ -148,7 +148,7 @@ def test_guard_direct_every_shape(variant):
     _guarded_roundtrip(SIZES, mp.PATH_DIRECT, variant, caps=(1, 3, 0), seed=100 + variant)
 
 
-@pytest.mark.parametrize("variant", range(9))
+@pytest.mark.parametrize("variant", range(10))
 def test_guard_bulk_every_shape(variant):
     _guarded_roundtrip(SIZES, mp.PATH_BULK, variant, caps=(1, 3, 0), seed=200 + variant)
 
@@ -164,7 +164,7 @@ def test_guard_dynamic_split_direct_every_shape(variant):
     _guarded_roundtrip(SIZES, mp.PATH_DIRECT, variant, caps=(3, 0), split=2, seed=700 + variant)
 
 
-@pytest.mark.parametrize("variant", list(range(9)))
+@pytest.mark.parametrize("variant", list(range(10)))
 def test_guard_dynamic_split_bulk_every_shape(variant):
     _guarded_roundtrip(SIZES, mp.PATH_BULK, variant, caps=(3, 0), split=2, seed=800 + variant)
 

@@ -27,7 +27,7 @@ def test_options_and_stash_free():
         ctx.set_option(mp.OPT_PATH, mp.PATH_BULK)
         assert ctx.get_option(mp.OPT_VARIANT) == mp.VARIANT_AUTO   # reset with the path
         with pytest.raises(mp.MPressError):
-            ctx.set_option(mp.OPT_VARIANT, 9)                        # bulk has 9 shapes (0-8)
+            ctx.set_option(mp.OPT_VARIANT, 10)                       # bulk has 10 shapes (0-9)
         assert ctx.stash_free() == [0, 4 << 20, 4 << 20]
         src = [torch.zeros(sizes[0], dtype=torch.uint8, device="cuda")]
         h = ctx.swap_out(pl, src)

@@ -16,7 +16,7 @@ SIZES = [1000, 70000, 300, (1 << 20) + 48, 17, 65536 * 3]
 
 
 @pytest.mark.parametrize("path,variant", [(mp.PATH_DIRECT, v) for v in range(14)] +
-                         [(mp.PATH_BULK, v) for v in range(9)] +
+                         [(mp.PATH_BULK, v) for v in range(10)] +
                          [(mp.PATH_CE, 0)])
 @pytest.mark.parametrize("misalign", [0, 16])
 def test_variant_roundtrip(path, variant, misalign):
