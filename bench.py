@@ -84,18 +84,20 @@ def parse():
                     help="swap grid cap (CTAs = SMs touched) while the concurrent GEMM runs (AUTO path -> "
                          "direct shape 9); 0 = calibrate: the first of --gemm-swap-candidates whose swap rate "
                          "on this run's links reaches --gemm-target-gbs / 0.85")
-    ap.add_argument("--gemm-swap-candidates", default="bulk:9:148,bulk:7:148,auto:-1:148,auto:-1:96,auto:-1:64",
+    ap.add_argument("--gemm-swap-candidates", default="bulk:7:148,bulk:9:148,auto:-1:148,auto:-1:96,auto:-1:64",
                     help="path:variant:max_ctas settings for the GEMM-concurrent swap, cheapest for the GEMM "
-                         "first: bulk 9 = a TMA warp (4 x 4 KiB of shared memory) plus an LSU warp per SM, "
-                         "1.4x bulk 7's rate at the same burst-GEMM cost (profiles/r02/hybrid/); "
+                         "first: one-warp TMA CTAs (bulk 7); bulk 9 = that TMA warp plus a register-copy warp "
+                         "per SM, 1.4x bulk 7's rate but a wider spread of burst-GEMM cost (+3..+13%%, "
+                         "profiles/r02/hybrid/); "
                          "one-warp TMA CTAs (4 x 4 KiB of shared memory) on every SM cost the "
                          "power-capped GEMM ~12%% where 128-thread direct CTAs cost ~18%% at the same rate "
                          "(profiles/r02/gemm_windows_*.jsonl); among the direct settings one light "
                          "CTA on every SM cost no more than 64 or 96 busier SMs (gemm_leg_settings.jsonl)")
-    ap.add_argument("--gemm-sus-fallback", default="auto:-1:64",
+    ap.add_argument("--gemm-sus-fallback", default="bulk:9:148",
                     help="swap setting (path:variant:max_ctas, unpaced) for the power-capped GEMM leg when the "
-                         "calibrated one moves less than --gemm-target-gbs there (empty: none); direct shape 9 on "
-                         "64 SMs moved 1121 GB/s at +7.8%% [7.6, 8.0] in 3 s windows (profiles/r02/gemm_windows_3s.jsonl)")
+                         "calibrated one moves less than --gemm-target-gbs there (empty: none); bulk 9 (TMA warp + "
+                         "register-copy warp) moved 998-1107 GB/s at +5.3..+5.8%% in 3 s windows, direct 9 on 64 "
+                         "SMs 1109-1128 at +7.6..+9.1%% (profiles/r02/hybrid/, gemm_windows_fallback_caps.jsonl)")
     ap.add_argument("--gemm-target-gbs", type=float, default=720.0,
                     help="per-source swap rate the GEMM-concurrent swap should sustain (BJ:5: 80%% of 900)")
     ap.add_argument("--gemm-no-pace", action="store_true",
