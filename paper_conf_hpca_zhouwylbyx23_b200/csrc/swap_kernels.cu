@@ -526,6 +526,12 @@ __device__ __forceinline__ uint64_t shfl64(uint64_t v, int lane) {
 // launch's counter -- twice the bytes in flight per SM inside the shared
 // memory a GEMM CTA leaves.  Only with the dynamic claims; under a static
 // split (small launches, graph capture) the TMA warp moves everything.
+// Registers decide whether it co-resides with the GEMM at all: a cuBLAS
+// CTA's 8 warps x 168 registers leave 5632 of each SM sub-partition's 16K,
+// so a warp of this kernel must stay at <= 176 registers (it uses 168; a
+// build at 180 lost co-residency and cost the GEMM +80%,
+// profiles/r02/hybrid/pace_180regs_gemm.jsonl).  Not paced (pacing keeps
+// CTAs resident while they sleep, which costs a GEMM more than it saves).
 template <int SHIFT, int CAP>
 __device__ __forceinline__ void bulk_lsu_warp(const CopyTable<CAP>& t, uint64_t workers) {
   constexpr uint32_t kVec = (1u << SHIFT) / 16u / 32u;  // 16-byte vectors per lane per piece
@@ -711,14 +717,16 @@ __device__ __forceinline__ void bulk_body(const CopyTable<CAP>& t) {
   }
 }
 
+// (LSU: at least 6 CTAs' worth of registers per SM = <= 168 registers per
+// thread, the co-residency bound with a GEMM CTA -- see bulk_lsu_warp)
 template <int DIR, int SHIFT, int STAGES, int CAP, int LSU>
-__global__ void __launch_bounds__(32 * (1 + LSU))
+__global__ void __launch_bounds__(32 * (1 + LSU), LSU ? 6 : 1)
 mp_swap_bulk(const __grid_constant__ CopyTable<CAP> t) {
   bulk_body<DIR, SHIFT, STAGES, CAP, LSU>(t);
 }
 
 template <int DIR, int SHIFT, int STAGES, int CAP, int LSU>
-__global__ void __launch_bounds__(32 * (1 + LSU))
+__global__ void __launch_bounds__(32 * (1 + LSU), LSU ? 6 : 1)
 mp_swap_bulk_g(const CopyTable<CAP>* __restrict__ tp) {
   bulk_body<DIR, SHIFT, STAGES, CAP, LSU>(*tp);
 }
